@@ -1,0 +1,368 @@
+/*
+ * ft2_oracle.c -- plain, slow, obviously-correct CPU oracle for FT2's hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this library.  The
+ * product path (paper_conf_hpdc_sunzmg00y25_b200/, libft2.so) never links,
+ * imports or calls it, and this file shares no code, header, table or
+ * constant generator with csrc/.
+ *
+ * Source of every definition: /root/reference/PAPER.md (FT2, HPDC'25), cited
+ * as L<line> plus section; where the paper is silent the reading is the one
+ * listed in DESIGN.md "Readings" (A1..A21).
+ *
+ * Representation (R0): bf16 values are handled as their uint16 bit patterns;
+ * every comparison is done on the order key
+ *     key(b) = (b & 0x8000) ? (~b & 0xFFFF) : (b | 0x8000)
+ * which is a total order on non-NaN values (-Inf < ... < -0 < +0 < ... < +Inf).
+ * Floating point appears only in bound scaling (R3, fp32 as the reading fixes)
+ * and in the reference GEMM (R8, fp64 accumulation).  Compiled with
+ * -O2 -fno-fast-math -ffp-contract=off so every fp op is a single IEEE op.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <string.h>
+
+#define EXPORT __attribute__((visibility("default")))
+
+/* ------------------------------------------------------------------ R0 --- */
+/* bf16 layout 1/8/7 (PAPER.md L185 describes the FP16 1/5/10 analogue). */
+
+EXPORT int ft2o_isnan(uint16_t b) { return (b & 0x7FFF) > 0x7F80; }
+EXPORT int ft2o_isinf(uint16_t b) { return (b & 0x7FFF) == 0x7F80; }
+EXPORT int ft2o_isfinite(uint16_t b) { return (b & 0x7F80) != 0x7F80; }
+
+EXPORT uint16_t ft2o_key(uint16_t b) {
+    return (b & 0x8000) ? (uint16_t)(~b & 0xFFFF) : (uint16_t)(b | 0x8000);
+}
+
+EXPORT uint16_t ft2o_unkey(uint16_t k) {
+    return (k & 0x8000) ? (uint16_t)(k & 0x7FFF) : (uint16_t)(~k & 0xFFFF);
+}
+
+EXPORT double ft2o_bf16_to_f64(uint16_t b) {
+    uint32_t u = (uint32_t)b << 16;
+    float f;
+    memcpy(&f, &u, 4);
+    return (double)f;
+}
+
+/* Round-to-nearest-even of an arbitrary double to bf16 (NaN -> 0x7FC0).
+ * Written from the definition: find the representable neighbours' spacing at
+ * the value's binade and round the scaled significand with rint() (the
+ * default FE_TONEAREST mode is ties-to-even).  Used for R8 (fp64 GEMM -> bf16)
+ * and for fp32 inputs (exact promotion to double). */
+EXPORT uint16_t ft2o_f64_to_bf16_rne(double d) {
+    if (isnan(d)) return 0x7FC0;
+    uint16_t sign = signbit(d) ? 0x8000 : 0x0000;
+    double a = fabs(d);
+    if (isinf(a)) return sign | 0x7F80;
+    if (a < ldexp(1.0, -126)) {
+        /* subnormal range: spacing 2^-133; rint(a * 2^133) in [0, 128] */
+        double q = rint(ldexp(a, 133));
+        return sign | (uint16_t)q; /* q == 128 encodes the smallest normal */
+    }
+    int e;
+    double m = frexp(a, &e); /* a = m * 2^e, m in [0.5, 1) */
+    double q = rint(ldexp(m, 8)); /* significand with 7 fraction bits, [128, 256] */
+    int E = e - 1;
+    if (q == 256.0) { q = 128.0; E += 1; }
+    if (E + 127 >= 255) return sign | 0x7F80; /* overflow -> Inf */
+    return sign | (uint16_t)(((E + 127) << 7) | ((int)q - 128));
+}
+
+/* Directed rounding of a double to bf16: dir = -1 toward -Inf, +1 toward +Inf.
+ * Used by R3 (bounds are rounded outward, reading A10).  Defined from RNE:
+ * take the nearest value, and step one ulp outward if it lies on the wrong
+ * side of d. */
+static uint16_t next_up_bf16(uint16_t b) { /* next representable toward +Inf */
+    uint16_t k = ft2o_key(b);
+    return ft2o_unkey((uint16_t)(k + 1));
+}
+static uint16_t next_down_bf16(uint16_t b) {
+    uint16_t k = ft2o_key(b);
+    return ft2o_unkey((uint16_t)(k - 1));
+}
+EXPORT uint16_t ft2o_f64_to_bf16_dir(double d, int dir) {
+    uint16_t r = ft2o_f64_to_bf16_rne(d);
+    double rv = ft2o_bf16_to_f64(r);
+    if (dir < 0 && rv > d) r = next_down_bf16(r);
+    if (dir > 0 && rv < d) r = next_up_bf16(r);
+    return r;
+}
+
+/* ------------------------------------------------------------------ R3 --- */
+/* Bound scaling, PAPER.md L229-L233 (Sec. 4.2.1, TA#6): "the scaling factor is
+ * set to 2".  Reading A2: widen away from the interval, i.e. lo <= 0 is
+ * multiplied by c and lo > 0 divided by c (and symmetrically for hi).  The
+ * product/quotient is formed in fp32 (one IEEE op), then rounded outward to
+ * bf16 (A10) and saturated to +-max finite 0x7F7F (A8). */
+EXPORT uint16_t ft2o_scale_bound(uint16_t raw, float c, int is_hi) {
+    float x = (float)ft2o_bf16_to_f64(raw);
+    volatile float s;
+    if (is_hi) s = (x >= 0.0f) ? x * c : x / c;
+    else       s = (x <= 0.0f) ? x * c : x / c;
+    uint16_t r = ft2o_f64_to_bf16_dir((double)s, is_hi ? +1 : -1);
+    if (r == 0x7F80) r = 0x7F7F; /* +Inf -> +max finite */
+    if (r == 0xFF80) r = 0xFF7F; /* -Inf -> -max finite */
+    return r;
+}
+
+/* ------------------------------------------------------------------ R5 --- */
+/* Check-and-clip of one value, PAPER.md L259-L261 (Sec. 4.3: "FT2 checks all
+ * the neuron values within each critical layer"), L261/L270 (TA#8: out-of-bound
+ * values are clipped to the bound), L191/L198 (NaN corrected to 0), L272
+ * (torch.clamp + torch.nan_to_num).  Reading A5: NaN -> clamp(+0, lo, hi);
+ * A6: +-Inf -> hi/lo through the clamp; A7: a value equal to a bound is in
+ * bounds, order = key order. Returns the corrected bits. */
+EXPORT uint16_t ft2o_clip_value(uint16_t y, uint16_t lo, uint16_t hi) {
+    uint16_t x = ft2o_isnan(y) ? 0x0000 : y; /* nan_to_num(nan=0.0) */
+    uint16_t k = ft2o_key(x);
+    if (k < ft2o_key(lo)) return lo;
+    if (k > ft2o_key(hi)) return hi;
+    return x;
+}
+
+/* In-place check-and-clip of y[rows][n] (row stride ld).  Row r belongs to
+ * sequence row_to_seq[r]; bounds[2*s] = lo_s, bounds[2*s+1] = hi_s.
+ * count[s] += number of elements whose bits changed (R5: corrected <=> y' != y).
+ * Rows whose sequence is out of [0, num_seqs) are skipped. */
+EXPORT void ft2o_protect(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
+                         const int32_t* row_to_seq, const uint16_t* bounds,
+                         int32_t num_seqs, uint32_t* count) {
+    for (int64_t r = 0; r < rows; ++r) {
+        int32_t s = row_to_seq ? row_to_seq[r] : (num_seqs == 1 ? 0 : (int32_t)r);
+        if (s < 0 || s >= num_seqs) continue;
+        uint16_t lo = bounds[2 * s], hi = bounds[2 * s + 1];
+        for (int64_t j = 0; j < n; ++j) {
+            uint16_t v = y[r * ld + j];
+            uint16_t w = ft2o_clip_value(v, lo, hi);
+            if (w != v) {
+                y[r * ld + j] = w;
+                if (count) count[s] += 1;
+            }
+        }
+    }
+}
+
+/* ------------------------------------------------------------- R2/R3/R4 --- */
+/* First-token bound profiling, PAPER.md L150 ("obtain bounds while generating
+ * the first token"), L221-L233 (Sec. 4.2), L332 ("two bound values are stored
+ * for each layer").  Readings A1 (one pair per sequence), A3/A4 (non-finite
+ * values excluded from the reduction), A9 (no finite value -> lo = hi = +0),
+ * A18 (only rows inside seq_offsets ranges count).
+ *
+ * y: [rows][n] bits, stride ld.  seq_offsets: [S+1] row offsets (NULL = one
+ * sequence covering all rows).  Outputs per sequence s:
+ *   raw_keys[2s] = key(min finite) or -1, raw_keys[2s+1] = key(max finite) or -1
+ *   bounds[2s], bounds[2s+1] = R3-scaled lo, hi (bf16 bits)
+ *   nonfinite[s] = number of non-finite elements
+ * If correct_nonfinite, R4 applies R5 to the prefill output with the fresh
+ * bounds ("NaN can always be detected and
+ * corrected" during the first token). */
+EXPORT void ft2o_bounds(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
+                        const int32_t* seq_offsets, int32_t num_seqs, float scale,
+                        int32_t correct_nonfinite, uint16_t* bounds, int32_t* raw_keys,
+                        uint32_t* nonfinite) {
+    for (int32_t s = 0; s < num_seqs; ++s) {
+        int64_t r0 = seq_offsets ? seq_offsets[s] : 0;
+        int64_t r1 = seq_offsets ? seq_offsets[s + 1] : rows;
+        int have = 0;
+        uint16_t kmin = 0, kmax = 0;
+        uint32_t nf = 0;
+        for (int64_t r = r0; r < r1; ++r) {
+            for (int64_t j = 0; j < n; ++j) {
+                uint16_t v = y[r * ld + j];
+                if (!ft2o_isfinite(v)) { nf++; continue; }
+                uint16_t k = ft2o_key(v);
+                if (!have || k < kmin) kmin = k;
+                if (!have || k > kmax) kmax = k;
+                have = 1;
+            }
+        }
+        uint16_t lo, hi;
+        if (have) {
+            lo = ft2o_scale_bound(ft2o_unkey(kmin), scale, 0);
+            hi = ft2o_scale_bound(ft2o_unkey(kmax), scale, 1);
+        } else {
+            lo = hi = 0x0000; /* A9 */
+        }
+        if (raw_keys) {
+            raw_keys[2 * s] = have ? (int32_t)kmin : -1;
+            raw_keys[2 * s + 1] = have ? (int32_t)kmax : -1;
+        }
+        if (bounds) { bounds[2 * s] = lo; bounds[2 * s + 1] = hi; }
+        if (nonfinite) nonfinite[s] = nf;
+        if (correct_nonfinite) {
+            for (int64_t r = r0; r < r1; ++r)
+                for (int64_t j = 0; j < n; ++j)
+                    y[r * ld + j] = ft2o_clip_value(y[r * ld + j], lo, hi);
+        }
+    }
+}
+
+/* Bounds from raw keys (the TP path): raw_keys as produced by
+ * ft2o_bounds (-1 = no finite value). */
+EXPORT void ft2o_bounds_from_keys(const int32_t* raw_keys, int32_t num_seqs, float scale,
+                                  uint16_t* bounds) {
+    for (int32_t s = 0; s < num_seqs; ++s) {
+        int32_t a = raw_keys[2 * s], b = raw_keys[2 * s + 1];
+        if (a < 0 || b < 0) { bounds[2 * s] = bounds[2 * s + 1] = 0; continue; }
+        bounds[2 * s] = ft2o_scale_bound(ft2o_unkey((uint16_t)a), scale, 0);
+        bounds[2 * s + 1] = ft2o_scale_bound(ft2o_unkey((uint16_t)b), scale, 1);
+    }
+}
+
+/* --------------------------------------------------------------- Philox --- */
+/* Philox4x32-10 (Salmon, Moraes, Dror, Shaw, SC'11), the counter-based
+ * generator the fault-site reading R6 uses. */
+static void mulhilo32(uint32_t a, uint32_t b, uint32_t* hi, uint32_t* lo) {
+    uint64_t p = (uint64_t)a * (uint64_t)b;
+    *hi = (uint32_t)(p >> 32);
+    *lo = (uint32_t)p;
+}
+EXPORT void ft2o_philox4x32_10(const uint32_t ctr_in[4], const uint32_t key_in[2], uint32_t out[4]) {
+    uint32_t c[4] = {ctr_in[0], ctr_in[1], ctr_in[2], ctr_in[3]};
+    uint32_t k0 = key_in[0], k1 = key_in[1];
+    for (int r = 0; r < 10; ++r) {
+        if (r > 0) { k0 += 0x9E3779B9u; k1 += 0xBB67AE85u; }
+        uint32_t hi0, lo0, hi1, lo1;
+        mulhilo32(0xD2511F53u, c[0], &hi0, &lo0);
+        mulhilo32(0xCD9E8D57u, c[2], &hi1, &lo1);
+        uint32_t n0 = hi1 ^ c[1] ^ k0, n1 = lo1, n2 = hi0 ^ c[3] ^ k1, n3 = lo0;
+        c[0] = n0; c[1] = n1; c[2] = n2; c[3] = n3;
+    }
+    out[0] = c[0]; out[1] = c[1]; out[2] = c[2]; out[3] = c[3];
+}
+
+/* --------------------------------------------------------------- R6 ------ */
+/* Fault sites, PAPER.md L84 (Sec. 2.2: 1-bit, 2-bit, EXP fault models), L88
+ * ("only one error occurs per inference"), L90 ("the location ... is
+ * identified by the layer ID, neuron ID, and bit locations"), L95 (uniformly
+ * distributed location; linear layers of the decoder blocks).  Readings A11
+ * (layer-then-neuron uniform, or size-weighted neuron-uniform), A12 (step
+ * uniform over 0..S, 0 = prefill with a uniform prompt token), A13 (2-bit =
+ * two distinct uniform positions; EXP = uniform over the exponent field).
+ *
+ * Site layout matches include/ft2.h's ft2_fault_site bit for bit, but the
+ * struct is restated here (no shared header). */
+typedef struct {
+    uint32_t trial;
+    uint16_t step, layer;
+    uint32_t token, col;
+    uint32_t xor_mask;
+    uint8_t model, nbits, pad[2];
+} ft2o_site;
+
+static uint32_t draw_below(uint32_t u, uint32_t n) { /* floor(u * n / 2^32) */
+    return (uint32_t)(((uint64_t)u * (uint64_t)n) >> 32);
+}
+
+/* dtype: 0 bf16 (16 bits, exponent bits 7..14), 1 fp16 (10..14), 2 fp32 (23..30) */
+EXPORT void ft2o_make_sites(uint64_t seed, uint64_t trial0, int32_t n_trials, int32_t model,
+                            int32_t dtype, int32_t n_steps, int32_t prompt_len, int32_t n_layers,
+                            const int32_t* layer_width, int32_t layer_uniform, int32_t step_policy,
+                            ft2o_site* out) {
+    uint32_t width_bits = (dtype == 2) ? 32u : 16u;
+    uint32_t exp_lo = (dtype == 0) ? 7u : (dtype == 1) ? 10u : 23u;
+    uint32_t exp_n = (dtype == 0) ? 8u : (dtype == 1) ? 5u : 8u;
+    uint64_t total_neurons = 0;
+    for (int32_t l = 0; l < n_layers; ++l) total_neurons += (uint64_t)layer_width[l];
+    for (int32_t i = 0; i < n_trials; ++i) {
+        uint64_t t = trial0 + (uint64_t)i;
+        uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
+        uint32_t c0[4] = {(uint32_t)t, (uint32_t)(t >> 32), 0u, 0x46543200u};
+        uint32_t c1[4] = {(uint32_t)t, (uint32_t)(t >> 32), 1u, 0x46543200u};
+        uint32_t u[4], v[4];
+        ft2o_philox4x32_10(c0, key, u);
+        ft2o_philox4x32_10(c1, key, v);
+        ft2o_site s;
+        memset(&s, 0, sizeof(s));
+        s.trial = (uint32_t)t;
+        uint32_t step;
+        if (step_policy == 1) step = 1u + (uint32_t)(t % (uint64_t)n_steps); /* one per decode step */
+        else step = draw_below(u[0], (uint32_t)n_steps + 1u);               /* A12 */
+        s.step = (uint16_t)step;
+        uint32_t layer, col;
+        if (layer_uniform) {
+            layer = draw_below(u[1], (uint32_t)n_layers);
+            col = draw_below(u[2], (uint32_t)layer_width[layer]);
+        } else {
+            /* neuron-uniform over all layers' outputs: one draw in [0, total) */
+            uint64_t g = ((uint64_t)u[1] * total_neurons) >> 32;
+            layer = 0;
+            while (g >= (uint64_t)layer_width[layer]) { g -= (uint64_t)layer_width[layer]; layer++; }
+            col = (uint32_t)g;
+        }
+        s.layer = (uint16_t)layer;
+        s.col = col;
+        s.token = (step == 0) ? draw_below(v[0], (uint32_t)prompt_len) : 0u;
+        uint32_t mask;
+        if (model == 0) {        /* 1-bit */
+            mask = 1u << draw_below(u[3], width_bits);
+            s.nbits = 1;
+        } else if (model == 1) { /* 2-bit: two distinct positions */
+            uint32_t b1 = draw_below(u[3], width_bits);
+            uint32_t b2p = draw_below(v[1], width_bits - 1u);
+            uint32_t b2 = b2p + (b2p >= b1 ? 1u : 0u);
+            mask = (1u << b1) | (1u << b2);
+            s.nbits = 2;
+        } else {                 /* EXP: one bit of the exponent field */
+            mask = 1u << (exp_lo + draw_below(u[3], exp_n));
+            s.nbits = 1;
+        }
+        s.xor_mask = mask;
+        s.model = (uint8_t)model;
+        out[i] = s;
+    }
+}
+
+/* --------------------------------------------------------------- R7 ------ */
+/* Injection, PAPER.md L90 (hook flips bits of the selected neuron in the
+ * layer output).  Site i belongs to batch slot i; its row is
+ * base_row[i] (or i if base_row is NULL) plus the prompt token when the
+ * current step is the prefill (step 0).  Sites that do not match
+ * (cur_step, cur_layer) or fall outside y are ignored. */
+EXPORT void ft2o_inject(uint16_t* y, int64_t rows, int64_t n, int64_t ld, const ft2o_site* sites,
+                        int32_t n_sites, int32_t cur_layer, int32_t cur_step, const int32_t* base_row) {
+    for (int32_t i = 0; i < n_sites; ++i) {
+        const ft2o_site* s = &sites[i];
+        if ((int32_t)s->step != cur_step || (int32_t)s->layer != cur_layer) continue;
+        int64_t row = (base_row ? base_row[i] : i) + (cur_step == 0 ? (int64_t)s->token : 0);
+        if (row < 0 || row >= rows || (int64_t)s->col >= n) continue;
+        y[row * ld + s->col] ^= (uint16_t)s->xor_mask;
+    }
+}
+
+/* --------------------------------------------------------------- R8 ------ */
+/* Reference linear layer for the fused path: y = x W^T + b (nn.Linear),
+ * accumulated in fp64 (independent of summation order), rounded once to bf16.
+ * x: [M][K] (ldx), w: [N][K] (ldw), bias: [N] or NULL, y: [M][N] (ldy). */
+EXPORT void ft2o_linear_f64(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
+                            const uint16_t* bias, int32_t M, int32_t N, int32_t K,
+                            double* y_f64, uint16_t* y_bf16, int64_t ldy) {
+    for (int32_t m = 0; m < M; ++m) {
+        for (int32_t j = 0; j < N; ++j) {
+            double acc = 0.0;
+            for (int32_t k = 0; k < K; ++k)
+                acc += ft2o_bf16_to_f64(x[(int64_t)m * ldx + k]) * ft2o_bf16_to_f64(w[(int64_t)j * ldw + k]);
+            if (bias) acc += ft2o_bf16_to_f64(bias[j]);
+            if (y_f64) y_f64[(int64_t)m * ldy + j] = acc;
+            if (y_bf16) y_bf16[(int64_t)m * ldy + j] = ft2o_f64_to_bf16_rne(acc);
+        }
+    }
+}
+
+/* Full oracle layer (R8 then R7 then R5): linear -> bf16 -> inject -> check. */
+EXPORT void ft2o_protected_linear(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
+                                  const uint16_t* bias, int32_t M, int32_t N, int32_t K,
+                                  uint16_t* y, int64_t ldy, const int32_t* row_to_seq,
+                                  const uint16_t* bounds, int32_t num_seqs, uint32_t* count,
+                                  const ft2o_site* sites, int32_t n_sites, int32_t cur_layer,
+                                  int32_t cur_step, const int32_t* base_row) {
+    ft2o_linear_f64(x, ldx, w, ldw, bias, M, N, K, 0, y, ldy);
+    if (sites && n_sites > 0) ft2o_inject(y, M, N, ldy, sites, n_sites, cur_layer, cur_step, base_row);
+    if (bounds) ft2o_protect(y, M, N, ldy, row_to_seq, bounds, num_seqs, count);
+}
+
+EXPORT int32_t ft2o_site_size(void) { return (int32_t)sizeof(ft2o_site); }
