@@ -1,0 +1,233 @@
+/*
+ * ft2.h -- C ABI of libft2.so, the B200 (sm_100a) implementation of FT2's
+ * online range restriction (Sun et al., "FT2: First-Token-Inspired Online
+ * Fault Tolerance on Critical Layers for Generative Large Language Models",
+ * HPDC'25).  Citations are to /root/reference/PAPER.md as L<line> (section).
+ *
+ * The method (Sec. 4): (1) pick the critical linear
+ * layers of the model (L149, L212; host-side); (2) while the
+ * first token is generated (prefill) reduce each protected layer's output to
+ * two bounds, widened by a factor 2 (L150, L221-L233, L332); (3) on every later
+ * token check every neuron of each protected layer's output against those
+ * bounds: out-of-bound values are clipped to the bound, NaN is corrected to 0
+ * (L151, L191, L198, L259-L272).  Faults for evaluation are 1-bit, 2-bit or
+ * exponent-bit flips of one neuron of one linear layer's output (L84, L90, L95).
+ *
+ * Conventions (all entry points):
+ *  - Pointers are DEVICE pointers unless stated otherwise.  Every call is
+ *    asynchronous on `stream` (a cudaStream_t passed as void*; NULL = legacy
+ *    default stream), is CUDA-graph capturable, never allocates device memory,
+ *    never synchronises, never throws.
+ *  - The caller owns every buffer (tensors, bounds, counters, sites,
+ *    workspace).  The library keeps no per-call state; the only global state
+ *    is a host-side cache of TMA descriptors (mutex-protected) and a launch
+ *    counter.
+ *  - Errors are reported synchronously from argument checks:
+ *      NULL required pointer, negative sizes, ld < n, num_seqs < 1, a
+ *      non-finite or < 1 scale                       -> FT2_ERR_INVALID_ARG
+ *      base pointer not 16-byte aligned, or ld % 8 != 0 (bf16)
+ *                                                    -> FT2_ERR_MISALIGNED
+ *      dtype other than FT2_BF16, shapes outside the stated limits
+ *                                                    -> FT2_ERR_UNSUPPORTED
+ *      kernel launch failure (cudaGetLastError)      -> FT2_ERR_CUDA
+ *    A zero-size tensor returns FT2_OK without launching.  Faults inside a
+ *    kernel surface at the caller's next synchronisation, as with CUDA.
+ *  - Counters accumulate (the caller zeroes them), so one counter can span a
+ *    whole request.
+ *  - Tensors are row-major: element (r, j) of an ft2_tensor lives at
+ *    data + (r * ld + j) * sizeof(dtype).
+ *  - Values are compared on the total order of reading A7:
+ *    -Inf < ... < -0 < +0 < ... < +Inf; a value equal to a bound is in bounds.
+ */
+#ifndef FT2_H_
+#define FT2_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    FT2_OK = 0,
+    FT2_ERR_INVALID_ARG = 1,
+    FT2_ERR_MISALIGNED = 2,
+    FT2_ERR_UNSUPPORTED = 3,
+    FT2_ERR_CUDA = 4
+} ft2_status;
+
+/* Activation dtype.  BF16 is implemented; FP16/FP32 (the paper's FP16 main
+ * precision L282 and its FP32 study L334) return FT2_ERR_UNSUPPORTED in this
+ * release. */
+typedef enum { FT2_BF16 = 0, FT2_FP16 = 1, FT2_FP32 = 2 } ft2_dtype;
+
+/* Fault models, PAPER.md L84 (Sec. 2.2): single-bit flip, double-bit flip,
+ * single-bit flip in the exponent bits. */
+typedef enum { FT2_FAULT_1BIT = 0, FT2_FAULT_2BIT = 1, FT2_FAULT_EXP = 2 } ft2_fault_model;
+
+/* Epilogue of ft2_protect_fused_gemm. */
+typedef enum {
+    FT2_GEMM_PLAIN = 0, /* y = x W^T + b (+ faults), no check: the unprotected baseline */
+    FT2_GEMM_CHECK = 1  /* ... then the check-and-clip of ft2_protect on the bf16 result */
+} ft2_gemm_mode;
+
+typedef struct {
+    void* data;       /* device pointer, 16-byte aligned */
+    int64_t rows;     /* number of rows (tokens) */
+    int64_t n;        /* elements per row (output neurons); multiple of 8 for bf16 */
+    int64_t ld;       /* row stride in elements, >= n, multiple of 8 for bf16 */
+    ft2_dtype dtype;
+} ft2_tensor;
+
+/* One fault-injection site: "the location ... is identified by
+ * the layer ID, neuron ID, and bit locations"; extended with the trial id, the
+ * token step (0 = prefill) and the prompt token for prefill faults. 24 bytes. */
+typedef struct {
+    uint32_t trial;    /* global trial id */
+    uint16_t step;     /* 0 = prefill (first token), s >= 1 = decode step s */
+    uint16_t layer;    /* linear-layer id in [0, n_layers) (block-major) */
+    uint32_t token;    /* prompt token (row offset) when step == 0, else 0 */
+    uint32_t col;      /* output neuron within the layer */
+    uint32_t xor_mask; /* bits to flip in the element's bit pattern */
+    uint8_t model;     /* ft2_fault_model */
+    uint8_t nbits;     /* popcount(xor_mask) */
+    uint8_t pad[2];
+} ft2_fault_site;
+
+/* Where faults can land (linear layers of the decoder blocks,
+ * uniformly distributed locations).  layer_width is a HOST array. */
+typedef struct {
+    int32_t n_steps;            /* decode steps S; sites draw step in [0, S] */
+    int32_t prompt_len;         /* prefill tokens T (token drawn in [0, T) for step 0) */
+    int32_t n_layers;           /* linear layers L (<= FT2_MAX_SITE_LAYERS) */
+    const int32_t* layer_width; /* host, [n_layers] output neurons per layer */
+    int32_t layer_uniform;      /* 1: layer uniform then neuron uniform (reading A11, default);
+                                   0: neuron-uniform over all layer outputs */
+    int32_t step_policy;        /* 0: step uniform in [0, S] (reading A12);
+                                   1: step = 1 + trial mod S (one fault per decode step, config C1) */
+} ft2_site_geometry;
+
+#define FT2_MAX_SITE_LAYERS 1024
+#define FT2_MAX_SEQS 65535
+
+/* ------------------------------------------------------------------------ */
+/* Bytes of workspace ft2_bounds_from_prefill needs for num_seqs sequences.
+ * The workspace must be zero-filled once before its first use; every call
+ * leaves it zero-filled again (self-cleaning), so it can be reused and
+ * captured in CUDA graphs.  One workspace must not be used by two calls that
+ * may run concurrently. */
+size_t ft2_workspace_bytes(int32_t num_seqs);
+
+/* First-token bound profiling: PAPER.md L150 ("obtain bounds while generating
+ * the first token"), L221-L233 (Sec. 4.2; bounds scaled by 2, TA#6), L332 (two
+ * bound values per protected layer), L225/L237/L241 (NaN in the first token is
+ * detected and corrected).
+ *
+ * y            [rows x n] prefill output of one protected layer.  Rows
+ *              [seq_offsets[s], seq_offsets[s+1]) belong to sequence s
+ *              (seq_offsets: device int32 [num_seqs+1], non-decreasing; NULL =
+ *              one sequence of all rows).  Rows outside every range (padding)
+ *              are ignored (reading A18).  Modified in place only when
+ *              correct_nonfinite = 1, and then only its non-finite elements.
+ * scale        widening factor c >= 1 (paper: 2).  lo <= 0 is multiplied by c,
+ *              lo > 0 divided (symmetrically for hi), in fp32, rounded outward
+ *              to bf16 and saturated to +-max finite (readings A2, A8, A10).
+ * finalize     1: write bounds_out.  0: only write keys_out (raw order keys for
+ *              a tensor-parallel MAX all-reduce, then ft2_bounds_finalize).
+ * correct_nonfinite  1 (requires finalize = 1): after the bounds are known,
+ *              NaN -> clamp(+0, lo, hi), +Inf -> hi, -Inf -> lo (readings A3-A6).
+ * bounds_out   [num_seqs x 2] bf16 (lo, hi) per sequence, or NULL if finalize = 0.
+ *              A sequence without finite values gets lo = hi = +0 (reading A9).
+ * keys_out     NULL or int32 [num_seqs x 2]: keys_out[2s] = 0xFFFF - key(lo_raw),
+ *              keys_out[2s+1] = key(hi_raw), -1 where the sequence has no finite
+ *              value; element-wise MAX of these over shards gives the keys of
+ *              the unsharded tensor (min/max are exact and associative).
+ * nonfinite_count  NULL or uint32 [num_seqs]: WRITTEN with the number of
+ *              non-finite elements of each sequence.
+ * workspace    ft2_workspace_bytes(num_seqs) bytes, see above.
+ * Limits: num_seqs <= FT2_MAX_SEQS, rows * n / 8 < 2^31. */
+ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int32_t num_seqs,
+                                   float scale, int32_t finalize, int32_t correct_nonfinite,
+                                   void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
+                                   void* workspace, void* stream);
+
+/* Bounds from (all-reduced) keys in the ft2_bounds_from_prefill keys_out
+ * encoding: the second half of the tensor-parallel path. */
+ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scale,
+                               ft2_dtype dtype, void* bounds_out, void* stream);
+
+/* Online range restriction of one protected layer's output: PAPER.md L151,
+ * L259-L261 (Sec. 4.3: check every neuron after each critical layer), L261/L270
+ * (TA#8: clip out-of-bound values to the bound), L191/L198 (NaN -> 0), L272
+ * (clamp + nan_to_num fused).  In place on y:
+ *   y' = clamp(isnan(y) ? +0 : y, lo_s, hi_s),   s = sequence of the row.
+ * row_to_seq   device int32 [rows] row -> sequence, or NULL: row r -> sequence
+ *              r when num_seqs == rows, every row -> sequence 0 when num_seqs
+ *              == 1 (otherwise FT2_ERR_INVALID_ARG).  Rows mapped outside
+ *              [0, num_seqs) are left untouched.
+ * bounds       [num_seqs x 2] bf16 (lo, hi) with key(lo) <= key(hi), finite.
+ * corrected_count  NULL or uint32 [num_seqs]: += number of elements whose bits
+ *              changed (= NaN, +-Inf or out of bounds).
+ * Only vectors containing a corrected element are written back. */
+ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* bounds,
+                       int32_t num_seqs, uint32_t* corrected_count, void* stream);
+
+/* Critical linear layer with the check fused into the GEMM epilogue (tcgen05
+ * MMA, TMEM accumulators, TMA-fed shared-memory pipeline on sm_100a):
+ *   y[m, j] = check(inject(bf16_rne(sum_k x[m, k] * w[j, k] + bias[j])))
+ * x [M x K] (ldx), w [N x K] (ldw, nn.Linear layout), bias [N] or NULL, y [M x N]
+ * (ldy), all bf16, fp32 accumulation.  The K reduction is complete before the
+ * epilogue (split-K partial sums are combined first: clipping is non-linear).
+ * mode         FT2_GEMM_PLAIN or FT2_GEMM_CHECK.
+ * col_begin/col_end  the protected column slice [col_begin, col_end) (e.g. V of
+ *              a fused QKV projection); 0/N = the whole output.
+ * row_to_seq, bounds, num_seqs, corrected_count  as in ft2_protect (used by CHECK).
+ * sites/n_sites/cur_layer/cur_step/base_row  optional fault injection applied
+ *              to the bf16 result before the check (order: GEMM -> bias -> bf16 ->
+ *              inject -> check; readings A19, A20), as in ft2_inject_faults.
+ * workspace/ws_bytes  scratch of ft2_gemm_workspace_bytes(M, N, K) bytes (may be 0).
+ * Limits: K % 8 == 0, ldx/ldw/ldy % 8 == 0, 16-byte aligned bases, M, N >= 1. */
+size_t ft2_gemm_workspace_bytes(int32_t M, int32_t N, int32_t K);
+ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw,
+                                  const void* bias, void* y, int64_t ldy, int32_t M, int32_t N,
+                                  int32_t K, ft2_gemm_mode mode, int32_t col_begin, int32_t col_end,
+                                  const int32_t* row_to_seq, const void* bounds, int32_t num_seqs,
+                                  uint32_t* corrected_count, const ft2_fault_site* sites,
+                                  int32_t n_sites, int32_t cur_layer, int32_t cur_step,
+                                  const int32_t* base_row, void* workspace, size_t ws_bytes,
+                                  void* stream);
+
+/* Seeded fault sites for trials [trial0, trial0 + n_trials) (reading R6:
+ * Philox4x32-10 keyed by seed, counter = trial id; uniform step, layer, neuron
+ * and bit position(s) per PAPER.md L84, L90, L95).  Bit-exact with the CPU
+ * oracle; any trial range can be generated independently (campaign sharding).
+ * geom is a HOST pointer; sites_out is device [n_trials]. */
+ft2_status ft2_make_fault_sites(uint64_t seed, uint64_t trial0, int32_t n_trials,
+                                ft2_fault_model model, ft2_dtype dtype,
+                                const ft2_site_geometry* geom, ft2_fault_site* sites_out,
+                                void* stream);
+
+/* Apply the sites whose (step, layer) equals (cur_step, cur_layer) to y:
+ * y[row, col] ^= xor_mask with row = (base_row ? base_row[i] : i) +
+ * (cur_step == 0 ? token : 0) for site i (site i belongs to batch slot i;
+ * pass seq_offsets as base_row during prefill).  Out-of-range sites are
+ * ignored.  PAPER.md L90 (hook-based neuron bit flips). */
+ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t n_sites,
+                             int32_t cur_layer, int32_t cur_step, const int32_t* base_row,
+                             void* stream);
+
+/* Human-readable status. */
+const char* ft2_status_string(ft2_status s);
+
+/* Number of kernels this library has launched since it was loaded (host-side
+ * counter; launches recorded into a CUDA graph count once, at capture). */
+uint64_t ft2_launch_count(void);
+
+/* Library version string ("ft2-b200 <semver> sm_100a"). */
+const char* ft2_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FT2_H_ */

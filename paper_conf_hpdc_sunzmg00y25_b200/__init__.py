@@ -1,0 +1,16 @@
+"""FT2 on B200: online range restriction of critical LLM layers (sm_100a).
+
+Product package.  It never imports ``oracle/``; compute runs only in
+``lib/libft2.so`` (built from ``csrc/`` for sm_100a).  Importing the package
+loads the library and raises if it is missing -- there is no CPU fallback.
+"""
+from ._lib import load as _load
+
+_load()
+
+from . import ft2  # noqa: E402,F401
+from .ft2 import (bounds_finalize, bounds_from_prefill, inject_faults, launch_count,  # noqa: E402,F401
+                  make_fault_sites, make_workspace, protect, protect_fused_gemm, version, workspace_bytes)
+
+__all__ = ["bounds_from_prefill", "bounds_finalize", "protect", "protect_fused_gemm", "make_fault_sites",
+           "inject_faults", "make_workspace", "workspace_bytes", "launch_count", "version"]

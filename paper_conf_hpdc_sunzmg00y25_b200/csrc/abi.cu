@@ -1,0 +1,237 @@
+// abi.cu -- the C ABI of libft2.so (include/ft2.h): argument validation,
+// status codes, launch bookkeeping.  All compute happens in the kernels of
+// bounds.cu, protect.cu, faults.cu and gemm_sm100.cu.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cmath>
+
+#include "ft2_internal.h"
+
+namespace ft2impl {
+
+int num_sms() {
+    static int cached[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (cached[dev] == 0) {
+        int n = 0;
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        cached[dev] = n > 0 ? n : 148;
+    }
+    return cached[dev];
+}
+
+}  // namespace ft2impl
+
+using namespace ft2impl;
+
+static std::atomic<uint64_t> g_launches{0};
+
+static inline bool al16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+static ft2_status check_tensor(const ft2_tensor& t, bool allow_null_if_empty = true) {
+    if (t.rows < 0 || t.n < 0 || t.ld < t.n) return FT2_ERR_INVALID_ARG;
+    if (t.dtype != FT2_BF16) return FT2_ERR_UNSUPPORTED;
+    if (t.rows == 0 || t.n == 0) return FT2_OK;
+    if (t.data == nullptr) return FT2_ERR_INVALID_ARG;
+    if (!al16(t.data) || (t.n % 8) != 0 || (t.ld % 8) != 0) return FT2_ERR_MISALIGNED;
+    (void)allow_null_if_empty;
+    return FT2_OK;
+}
+
+static inline ft2_status finish(cudaError_t e, int launches) {
+    g_launches.fetch_add((uint64_t)launches, std::memory_order_relaxed);
+    if (e != cudaSuccess) {
+        cudaGetLastError();  // clear the sticky-free launch error
+        return FT2_ERR_CUDA;
+    }
+    return FT2_OK;
+}
+
+extern "C" {
+
+size_t ft2_workspace_bytes(int32_t num_seqs) {
+    if (num_seqs < 1) num_seqs = 1;
+    return bounds_ws_bytes(num_seqs);
+}
+
+ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int32_t num_seqs, float scale,
+                                   int32_t finalize, int32_t correct_nonfinite, void* bounds_out,
+                                   int32_t* keys_out, uint32_t* nonfinite_count, void* workspace,
+                                   void* stream) {
+    ft2_status s = check_tensor(y);
+    if (s != FT2_OK) return s;
+    if (num_seqs < 1 || num_seqs > FT2_MAX_SEQS) return num_seqs < 1 ? FT2_ERR_INVALID_ARG : FT2_ERR_UNSUPPORTED;
+    if (!(std::isfinite(scale)) || scale < 1.0f) return FT2_ERR_INVALID_ARG;
+    if (workspace == nullptr) return FT2_ERR_INVALID_ARG;
+    if (finalize && bounds_out == nullptr) return FT2_ERR_INVALID_ARG;
+    if (!finalize && keys_out == nullptr) return FT2_ERR_INVALID_ARG;
+    if (correct_nonfinite && !finalize) return FT2_ERR_INVALID_ARG;
+    if (seq_offsets == nullptr && num_seqs != 1) return FT2_ERR_INVALID_ARG;
+    if (((uintptr_t)workspace & 7u) != 0 || (bounds_out && ((uintptr_t)bounds_out & 3u) != 0))
+        return FT2_ERR_MISALIGNED;
+    if ((y.rows * (y.n / 8)) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
+    if (y.rows == 0 || y.n == 0) {
+        // nothing to reduce: every sequence is empty (reading A9) -- still a
+        // well-defined result, produced by the finalize kernel on "no value" keys
+        // would need a buffer; report OK without touching outputs.
+        return FT2_OK;
+    }
+    BoundsArgs a;
+    a.y = static_cast<uint16_t*>(y.data);
+    a.ld = y.ld;
+    a.rows = y.rows;
+    a.n = y.n;
+    a.seq_offsets = seq_offsets;
+    a.S = num_seqs;
+    a.scale = scale;
+    a.finalize = finalize ? 1 : 0;
+    a.correct = correct_nonfinite ? 1 : 0;
+    a.bounds_out = static_cast<uint16_t*>(bounds_out);
+    a.keys_out = keys_out;
+    a.nonfinite_out = nonfinite_count;
+    a.ws = static_cast<uint32_t*>(workspace);
+    int nl = 0;
+    cudaError_t e = launch_bounds(a, static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scale, ft2_dtype dtype,
+                               void* bounds_out, void* stream) {
+    if (keys == nullptr || bounds_out == nullptr || num_seqs < 1) return FT2_ERR_INVALID_ARG;
+    if (!(std::isfinite(scale)) || scale < 1.0f) return FT2_ERR_INVALID_ARG;
+    if (dtype != FT2_BF16) return FT2_ERR_UNSUPPORTED;
+    int nl = 0;
+    cudaError_t e = launch_finalize(keys, num_seqs, scale, static_cast<uint16_t*>(bounds_out),
+                                    static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* bounds, int32_t num_seqs,
+                       uint32_t* corrected_count, void* stream) {
+    ft2_status s = check_tensor(y);
+    if (s != FT2_OK) return s;
+    if (num_seqs < 1 || bounds == nullptr) return FT2_ERR_INVALID_ARG;
+    if (row_to_seq == nullptr && num_seqs != 1 && (int64_t)num_seqs != y.rows) return FT2_ERR_INVALID_ARG;
+    if (((uintptr_t)bounds & 3u) != 0) return FT2_ERR_MISALIGNED;
+    if ((y.rows * (y.n / 8)) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
+    if (y.rows == 0 || y.n == 0) return FT2_OK;
+    ProtectArgs a;
+    a.y = static_cast<uint16_t*>(y.data);
+    a.ld = y.ld;
+    a.rows = y.rows;
+    a.n = y.n;
+    a.row_to_seq = row_to_seq;
+    a.S = num_seqs;
+    a.bounds = static_cast<const uint16_t*>(bounds);
+    a.counts = corrected_count;
+    int nl = 0;
+    cudaError_t e = launch_protect(a, static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+size_t ft2_gemm_workspace_bytes(int32_t M, int32_t N, int32_t K) { return gemm_ws_bytes(M, N, K); }
+
+ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, const void* bias,
+                                  void* y, int64_t ldy, int32_t M, int32_t N, int32_t K, ft2_gemm_mode mode,
+                                  int32_t col_begin, int32_t col_end, const int32_t* row_to_seq,
+                                  const void* bounds, int32_t num_seqs, uint32_t* corrected_count,
+                                  const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
+                                  int32_t cur_step, const int32_t* base_row, void* workspace, size_t ws_bytes,
+                                  void* stream) {
+    if (M < 0 || N < 0 || K < 0) return FT2_ERR_INVALID_ARG;
+    if (M == 0 || N == 0) return FT2_OK;
+    if (K == 0) return FT2_ERR_UNSUPPORTED;
+    if (x == nullptr || w == nullptr || y == nullptr) return FT2_ERR_INVALID_ARG;
+    if (ldx < K || ldw < K || ldy < N) return FT2_ERR_INVALID_ARG;
+    if (mode != FT2_GEMM_PLAIN && mode != FT2_GEMM_CHECK) return FT2_ERR_INVALID_ARG;
+    if (!al16(x) || !al16(w) || !al16(y) || (bias && ((uintptr_t)bias & 1u)) || (K % 8) || (ldx % 8) ||
+        (ldw % 8) || (ldy % 8))
+        return FT2_ERR_MISALIGNED;
+    if (mode == FT2_GEMM_CHECK) {
+        if (bounds == nullptr || num_seqs < 1) return FT2_ERR_INVALID_ARG;
+        if (row_to_seq == nullptr && num_seqs != 1 && num_seqs != M) return FT2_ERR_INVALID_ARG;
+        if (col_begin < 0 || col_end > N || col_begin > col_end) return FT2_ERR_INVALID_ARG;
+    }
+    if (n_sites < 0 || (n_sites > 0 && sites == nullptr)) return FT2_ERR_INVALID_ARG;
+    if (ws_bytes < gemm_ws_bytes(M, N, K)) return FT2_ERR_INVALID_ARG;
+    GemmArgs a;
+    a.x = static_cast<const uint16_t*>(x);
+    a.ldx = ldx;
+    a.w = static_cast<const uint16_t*>(w);
+    a.ldw = ldw;
+    a.bias = static_cast<const uint16_t*>(bias);
+    a.y = static_cast<uint16_t*>(y);
+    a.ldy = ldy;
+    a.M = M;
+    a.N = N;
+    a.K = K;
+    a.mode = mode;
+    a.col_begin = (mode == FT2_GEMM_CHECK) ? col_begin : 0;
+    a.col_end = (mode == FT2_GEMM_CHECK) ? col_end : N;
+    a.row_to_seq = row_to_seq;
+    a.bounds = static_cast<const uint16_t*>(bounds);
+    a.S = num_seqs;
+    a.counts = corrected_count;
+    a.sites = n_sites > 0 ? sites : nullptr;
+    a.n_sites = n_sites;
+    a.cur_layer = cur_layer;
+    a.cur_step = cur_step;
+    a.base_row = base_row;
+    a.ws = workspace;
+    a.ws_bytes = ws_bytes;
+    int nl = 0;
+    cudaError_t e = launch_gemm(a, static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+ft2_status ft2_make_fault_sites(uint64_t seed, uint64_t trial0, int32_t n_trials, ft2_fault_model model,
+                                ft2_dtype dtype, const ft2_site_geometry* geom, ft2_fault_site* sites_out,
+                                void* stream) {
+    if (geom == nullptr || n_trials < 0) return FT2_ERR_INVALID_ARG;
+    if (n_trials == 0) return FT2_OK;
+    if (sites_out == nullptr || geom->layer_width == nullptr) return FT2_ERR_INVALID_ARG;
+    if (model < FT2_FAULT_1BIT || model > FT2_FAULT_EXP) return FT2_ERR_INVALID_ARG;
+    if (dtype < FT2_BF16 || dtype > FT2_FP32) return FT2_ERR_INVALID_ARG;
+    if (geom->n_layers < 1 || geom->n_steps < 0 || geom->prompt_len < 1) return FT2_ERR_INVALID_ARG;
+    if (geom->step_policy == 1 && geom->n_steps < 1) return FT2_ERR_INVALID_ARG;
+    if (geom->n_layers > FT2_MAX_SITE_LAYERS) return FT2_ERR_UNSUPPORTED;
+    for (int l = 0; l < geom->n_layers; ++l)
+        if (geom->layer_width[l] < 1) return FT2_ERR_INVALID_ARG;
+    int nl = 0;
+    cudaError_t e = launch_make_sites(seed, trial0, n_trials, (int32_t)model, (int32_t)dtype, *geom, sites_out,
+                                      static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
+                             int32_t cur_step, const int32_t* base_row, void* stream) {
+    if (y.rows < 0 || y.n < 0 || y.ld < y.n) return FT2_ERR_INVALID_ARG;
+    if (y.dtype != FT2_BF16) return FT2_ERR_UNSUPPORTED;
+    if (n_sites < 0) return FT2_ERR_INVALID_ARG;
+    if (n_sites == 0 || y.rows == 0 || y.n == 0) return FT2_OK;
+    if (sites == nullptr || y.data == nullptr) return FT2_ERR_INVALID_ARG;
+    int nl = 0;
+    cudaError_t e = launch_inject(static_cast<uint16_t*>(y.data), y.rows, y.n, y.ld, sites, n_sites, cur_layer,
+                                  cur_step, base_row, static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+const char* ft2_status_string(ft2_status s) {
+    switch (s) {
+        case FT2_OK: return "FT2_OK";
+        case FT2_ERR_INVALID_ARG: return "FT2_ERR_INVALID_ARG";
+        case FT2_ERR_MISALIGNED: return "FT2_ERR_MISALIGNED";
+        case FT2_ERR_UNSUPPORTED: return "FT2_ERR_UNSUPPORTED";
+        case FT2_ERR_CUDA: return "FT2_ERR_CUDA";
+    }
+    return "FT2_ERR_UNKNOWN";
+}
+
+uint64_t ft2_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
+
+const char* ft2_version(void) { return "ft2-b200 0.1.0 sm_100a"; }
+
+}  // extern "C"

@@ -1,0 +1,312 @@
+// bounds.cu -- first-token bound profiling as
+// one HBM sweep on sm_100a.
+//
+// Each CTA owns a contiguous range of 16-byte vectors (8 bf16) of the prefill
+// output and splits it at sequence boundaries.  Per segment every thread keeps
+// a packed-u16x2 min and max of order keys over its 128-bit coalesced loads
+// (4 loads in flight per thread: PRMT+LOP3 for the keys, VIMNMX.U16x2 for the
+// min/max -- 2 ALU ops per element), the warp combines with redux.sync
+// (CREDUX), the CTA through shared memory, and the grid through u32 atomicMax
+// on a self-cleaning workspace.  The last CTA to finish (threadfence
+// reduction) scales the bounds (R3), writes them, patches the few non-finite
+// elements it was told about (R4), and zeroes the workspace.
+//
+// Non-finite values (NaN/Inf) are excluded from the bounds (readings A3/A4).
+// The fast loop does not test for them: any non-finite key lies below 0x0080
+// or above 0xFF7F, so a thread whose min/max leave [0x0080, 0xFF7F] re-sweeps
+// its own vectors in a slow exact path.  In the common all-finite case the
+// kernel moves 2 bytes/element and does no extra work.
+#include <cuda_runtime.h>
+
+#include "ft2_device.cuh"
+#include "ft2_internal.h"
+
+namespace ft2impl {
+using namespace ft2dev;
+
+constexpr int kThreads = 256;
+constexpr int kUnroll = 4;
+
+size_t bounds_ws_bytes(int32_t S) {
+    size_t head = (size_t)(3 * S + 4) * 4;
+    head = (head + 7) & ~(size_t)7;
+    return head + (size_t)kPatchCap * 8;
+}
+
+struct BoundsK {
+    uint16_t* y;
+    int64_t ld;
+    uint32_t n8;          // vectors per row
+    uint32_t total_vec;   // rows * n8
+    uint32_t chunk;       // vectors per CTA
+    FastDiv div_n8;
+    int contiguous;       // ld == n
+    const int32_t* seq_offsets;
+    int32_t S;
+    float scale;
+    int32_t finalize, correct;
+    uint16_t* bounds_out;
+    int32_t* keys_out;
+    uint32_t* nonfinite_out;
+    uint32_t* ws;
+};
+
+__device__ __forceinline__ const uint4* vec_ptr(const BoundsK& p, uint32_t v) {
+    if (p.contiguous) return reinterpret_cast<const uint4*>(p.y) + v;
+    uint32_t row = fdiv(v, p.div_n8);
+    uint32_t col = v - row * p.n8;
+    return reinterpret_cast<const uint4*>(p.y + (int64_t)row * p.ld) + col;
+}
+
+// largest s in [0, S] with so[s] <= row  (so non-decreasing); -1 if row < so[0]
+__device__ __forceinline__ int seq_of_row(const int32_t* so, int S, uint32_t row) {
+    if ((int64_t)row < (int64_t)so[0]) return -1;
+    int lo = 0, hi = S;  // invariant so[lo] <= row
+    while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if ((int64_t)so[mid] <= (int64_t)row) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+__device__ __forceinline__ void record_patch(const BoundsK& p, uint32_t* list_count, uint32_t* overflow,
+                                             unsigned long long* list, int s, uint64_t off) {
+    uint32_t i = atomicAdd(list_count, 1u);
+    if (i < (uint32_t)kPatchCap) list[i] = (unsigned long long)(off | ((uint64_t)s << 48));
+    else atomicExch(overflow, 1u);
+}
+
+// Slow exact path for one vector: min/max over finite keys, count the rest.
+__device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, uint32_t& kmin, uint32_t& kmax,
+                                         uint32_t& nf, uint32_t* lc, uint32_t* ov, unsigned long long* list) {
+    const uint4* q = vec_ptr(p, v);
+    uint4 d = *q;
+    uint32_t w[4] = {d.x, d.y, d.z, d.w};
+    uint64_t base = (uint64_t)(reinterpret_cast<const uint16_t*>(q) - p.y);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        uint16_t b = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
+        if ((b & 0x7F80) == 0x7F80) {
+            nf++;
+            if (p.correct) record_patch(p, lc, ov, list, s, base + j);
+        } else {
+            uint32_t k = key1(b);
+            kmin = min(kmin, k);
+            kmax = max(kmax, k);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
+    __shared__ uint32_t sh_min[kThreads / 32], sh_max[kThreads / 32], sh_nf[kThreads / 32];
+    __shared__ int sh_last;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int S = p.S;
+    uint32_t* ws_done = p.ws + 3 * S;
+    uint32_t* ws_lc = p.ws + 3 * S + 1;
+    uint32_t* ws_ov = p.ws + 3 * S + 2;
+    unsigned long long* list = reinterpret_cast<unsigned long long*>(
+        reinterpret_cast<char*>(p.ws) + (((size_t)(3 * S + 4) * 4 + 7) & ~(size_t)7));
+
+    uint32_t v = blockIdx.x * p.chunk;
+    uint32_t v_end = min(v + p.chunk, p.total_vec);
+    while (v < v_end) {
+        int s;
+        uint32_t seg_end;
+        if (p.seq_offsets == nullptr) {
+            s = 0;
+            seg_end = v_end;
+        } else {
+            uint32_t row = fdiv(v, p.div_n8);
+            s = seq_of_row(p.seq_offsets, S, row);
+            if (s < 0) {  // padding rows before the first sequence
+                v = min(v_end, (uint32_t)p.seq_offsets[0] * p.n8);
+                continue;
+            }
+            if (s >= S) break;  // padding rows after the last sequence
+            seg_end = min(v_end, (uint32_t)p.seq_offsets[s + 1] * p.n8);
+        }
+        // ---- fast sweep of [v, seg_end): packed key min/max, 4 x 16 B in flight
+        uint32_t mn2 = 0xFFFFFFFFu, mx2 = 0u;
+        for (uint32_t base = v + tid; base < seg_end; base += kThreads * kUnroll) {
+            uint4 d[kUnroll];
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) {
+                uint32_t vi = base + u * kThreads;
+                d[u] = vi < seg_end ? ld_stream(vec_ptr(p, vi)) : make_uint4(0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu);
+            }
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) {
+                uint32_t vi = base + u * kThreads;
+                uint32_t k0 = key2(d[u].x), k1 = key2(d[u].y), k2 = key2(d[u].z), k3 = key2(d[u].w);
+                uint32_t a = vmin_u16x2(vmin_u16x2(k0, k1), vmin_u16x2(k2, k3));
+                uint32_t b = vmax_u16x2(vmax_u16x2(k0, k1), vmax_u16x2(k2, k3));
+                if (vi < seg_end) { mn2 = vmin_u16x2(mn2, a); mx2 = vmax_u16x2(mx2, b); }
+            }
+        }
+        uint32_t kmin = min(mn2 & 0xFFFFu, mn2 >> 16);
+        uint32_t kmax = max(mx2 & 0xFFFFu, mx2 >> 16);
+        uint32_t nf = 0;
+        if (kmin < 0x0080u || kmax > 0xFF7Fu) {
+            // this thread saw a non-finite value: redo its vectors exactly
+            kmin = 0xFFFFu;
+            kmax = 0u;
+            for (uint32_t vi = v + tid; vi < seg_end; vi += kThreads)
+                slow_vec(p, vi, s, kmin, kmax, nf, ws_lc, ws_ov, list);
+        }
+        kmin = __reduce_min_sync(0xFFFFFFFFu, kmin);
+        kmax = __reduce_max_sync(0xFFFFFFFFu, kmax);
+        nf = __reduce_add_sync(0xFFFFFFFFu, nf);
+        if (lane == 0) { sh_min[warp] = kmin; sh_max[warp] = kmax; sh_nf[warp] = nf; }
+        __syncthreads();
+        if (tid == 0) {
+            uint32_t a = sh_min[0], b = sh_max[0], c = sh_nf[0];
+#pragma unroll
+            for (int i = 1; i < kThreads / 32; ++i) { a = min(a, sh_min[i]); b = max(b, sh_max[i]); c += sh_nf[i]; }
+            if (a <= b) {  // at least one finite value in this segment
+                atomicMax(&p.ws[3 * s + 0], 0x10000u - a);
+                atomicMax(&p.ws[3 * s + 1], b + 1u);
+            }
+            if (c) atomicAdd(&p.ws[3 * s + 2], c);
+        }
+        __syncthreads();
+        v = seg_end;
+    }
+
+    // ---- grid combine: the last CTA finalises
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) sh_last = (atomicAdd(ws_done, 1u) == gridDim.x - 1);
+    __syncthreads();
+    if (!sh_last) return;
+    __threadfence();
+
+    for (int s = tid; s < S; s += kThreads) {
+        uint32_t los = atomicAdd(&p.ws[3 * s + 0], 0u);
+        uint32_t his = atomicAdd(&p.ws[3 * s + 1], 0u);
+        uint32_t nfc = atomicAdd(&p.ws[3 * s + 2], 0u);
+        bool have = los != 0u && his != 0u;
+        uint32_t kmin = 0x10000u - los, kmax = his - 1u;
+        if (p.finalize) {
+            uint16_t lo = 0, hi = 0;  // reading A9
+            if (have) {
+                lo = scale_bound(unkey1((uint16_t)kmin), p.scale, false);
+                hi = scale_bound(unkey1((uint16_t)kmax), p.scale, true);
+            }
+            p.bounds_out[2 * s] = lo;
+            p.bounds_out[2 * s + 1] = hi;
+        }
+        if (p.keys_out) {
+            p.keys_out[2 * s] = have ? (int32_t)(0xFFFFu - kmin) : -1;
+            p.keys_out[2 * s + 1] = have ? (int32_t)kmax : -1;
+        }
+        if (p.nonfinite_out) p.nonfinite_out[s] = nfc;
+        p.ws[3 * s + 0] = 0u;
+        p.ws[3 * s + 1] = 0u;
+        p.ws[3 * s + 2] = 0u;
+    }
+    __syncthreads();
+    if (p.correct) {
+        __threadfence_block();
+        uint32_t cnt = atomicAdd(ws_lc, 0u);
+        uint32_t ov = atomicAdd(ws_ov, 0u);
+        if (!ov) {
+            for (uint32_t i = tid; i < cnt; i += kThreads) {
+                unsigned long long e = list[i];
+                int s = (int)(e >> 48);
+                uint64_t off = e & 0xFFFFFFFFFFFFull;
+                uint16_t b = p.y[off];
+                uint16_t lo = p.bounds_out[2 * s], hi = p.bounds_out[2 * s + 1];
+                // R5 on a non-finite value: NaN -> clamp(+0), +Inf -> hi, -Inf -> lo
+                uint16_t x = ((b & 0x7FFF) > 0x7F80) ? (uint16_t)0 : b;
+                uint16_t k = key1(x);
+                p.y[off] = k < key1(lo) ? lo : (k > key1(hi) ? hi : x);
+            }
+        } else {
+            // more non-finite values than the patch list holds: this CTA sweeps
+            // the whole tensor (only reachable with pathological inputs)
+            for (uint32_t vi = tid; vi < p.total_vec; vi += kThreads) {
+                uint32_t row = fdiv(vi, p.div_n8);
+                int s = 0;
+                if (p.seq_offsets) {
+                    s = seq_of_row(p.seq_offsets, S, row);
+                    if (s < 0 || s >= S) continue;
+                }
+                uint16_t* q = const_cast<uint16_t*>(reinterpret_cast<const uint16_t*>(vec_ptr(p, vi)));
+                uint16_t lo = p.bounds_out[2 * s], hi = p.bounds_out[2 * s + 1];
+                for (int j = 0; j < 8; ++j) {
+                    uint16_t b = q[j];
+                    if ((b & 0x7F80) != 0x7F80) continue;
+                    uint16_t x = ((b & 0x7FFF) > 0x7F80) ? (uint16_t)0 : b;
+                    uint16_t k = key1(x);
+                    q[j] = k < key1(lo) ? lo : (k > key1(hi) ? hi : x);
+                }
+            }
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        *ws_lc = 0u;
+        *ws_ov = 0u;
+        *ws_done = 0u;
+    }
+}
+
+__global__ void finalize_kernel(const int32_t* keys, int32_t S, float scale, uint16_t* out) {
+    int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= S) return;
+    int32_t a = keys[2 * s], b = keys[2 * s + 1];
+    uint16_t lo = 0, hi = 0;
+    if (a >= 0 && b >= 0) {
+        lo = scale_bound(unkey1((uint16_t)(0xFFFF - a)), scale, false);
+        hi = scale_bound(unkey1((uint16_t)b), scale, true);
+    }
+    out[2 * s] = lo;
+    out[2 * s + 1] = hi;
+}
+
+static int g_blocks_per_sm = 0;
+
+cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
+    BoundsK p;
+    p.y = a.y;
+    p.ld = a.ld;
+    p.n8 = (uint32_t)(a.n / 8);
+    p.total_vec = (uint32_t)(a.rows * (a.n / 8));
+    p.div_n8 = make_fastdiv(p.n8);
+    p.contiguous = (a.ld == a.n);
+    p.seq_offsets = a.seq_offsets;
+    p.S = a.S;
+    p.scale = a.scale;
+    p.finalize = a.finalize;
+    p.correct = a.correct;
+    p.bounds_out = a.bounds_out;
+    p.keys_out = a.keys_out;
+    p.nonfinite_out = a.nonfinite_out;
+    p.ws = a.ws;
+    if (g_blocks_per_sm == 0) {
+        int b = 0;
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel, kThreads, 0);
+        if (e != cudaSuccess) return e;
+        g_blocks_per_sm = b > 0 ? b : 1;
+    }
+    const uint32_t per_iter = kThreads * kUnroll;
+    uint32_t max_grid = (uint32_t)(num_sms() * g_blocks_per_sm);
+    uint32_t want = (p.total_vec + 2 * per_iter - 1) / (2 * per_iter);  // >= 2 sweeps per CTA
+    uint32_t grid = want < 1 ? 1 : (want > max_grid ? max_grid : want);
+    p.chunk = (p.total_vec + grid - 1) / grid;
+    grid = (p.total_vec + p.chunk - 1) / p.chunk;
+    if (grid < 1) grid = 1;
+    bounds_kernel<<<grid, kThreads, 0, st>>>(p);
+    ++*n_launch;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out, cudaStream_t st,
+                            int* n_launch) {
+    finalize_kernel<<<(S + 127) / 128, 128, 0, st>>>(keys, S, scale, out);
+    ++*n_launch;
+    return cudaGetLastError();
+}
+
+}  // namespace ft2impl

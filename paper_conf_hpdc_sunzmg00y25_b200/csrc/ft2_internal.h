@@ -1,0 +1,75 @@
+// ft2_internal.h -- launchers shared between the kernel files and abi.cu.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/ft2.h"
+
+namespace ft2impl {
+
+// Workspace of the bounds reduction (u32 words unless noted):
+//   [3s+0] lo slot  = 0x10000 - min key  (0 = no finite value yet)
+//   [3s+1] hi slot  = max key + 1        (0 = none)
+//   [3s+2] non-finite count
+//   [3S+0] CTA completion counter, [3S+1] patch-list count, [3S+2] overflow flag
+//   then (8-byte aligned) u64 patch list [kPatchCap]: offset | seq << 48
+constexpr int kPatchCap = 4096;
+size_t bounds_ws_bytes(int32_t S);
+
+struct BoundsArgs {
+    uint16_t* y;
+    int64_t ld;
+    int64_t rows, n;
+    const int32_t* seq_offsets;
+    int32_t S;
+    float scale;
+    int32_t finalize, correct;
+    uint16_t* bounds_out;
+    int32_t* keys_out;
+    uint32_t* nonfinite_out;
+    uint32_t* ws;
+};
+cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch);
+cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out,
+                            cudaStream_t st, int* n_launch);
+
+struct ProtectArgs {
+    uint16_t* y;
+    int64_t ld, rows, n;
+    const int32_t* row_to_seq;  // or NULL
+    int32_t S;
+    const uint16_t* bounds;
+    uint32_t* counts;
+};
+cudaError_t launch_protect(const ProtectArgs& a, cudaStream_t st, int* n_launch);
+
+cudaError_t launch_make_sites(uint64_t seed, uint64_t trial0, int32_t n, int32_t model,
+                              int32_t dtype, const ft2_site_geometry& g, ft2_fault_site* out,
+                              cudaStream_t st, int* n_launch);
+cudaError_t launch_inject(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
+                          const ft2_fault_site* sites, int32_t n_sites, int32_t layer,
+                          int32_t step, const int32_t* base_row, cudaStream_t st, int* n_launch);
+
+struct GemmArgs {
+    const uint16_t* x; int64_t ldx;
+    const uint16_t* w; int64_t ldw;
+    const uint16_t* bias;
+    uint16_t* y; int64_t ldy;
+    int32_t M, N, K;
+    int32_t mode;
+    int32_t col_begin, col_end;
+    const int32_t* row_to_seq;
+    const uint16_t* bounds;
+    int32_t S;
+    uint32_t* counts;
+    const ft2_fault_site* sites;
+    int32_t n_sites, cur_layer, cur_step;
+    const int32_t* base_row;
+    void* ws; size_t ws_bytes;
+};
+size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K);
+cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch);
+
+int num_sms();
+
+}  // namespace ft2impl

@@ -1,0 +1,124 @@
+"""torch-facing binding of libft2.so: same names as include/ft2.h, arguments
+marshalled from torch tensors (data_ptr, shape, stride) and the current CUDA
+stream.  No computation happens here -- every step runs in the library's
+kernels.  PAPER.md citations are in include/ft2.h.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import _lib
+from ._lib import (FT2_BF16, FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FaultSite, SiteGeometry, Tensor, check,
+                   load)
+
+SITE_BYTES = ctypes.sizeof(FaultSite)
+
+
+def _stream(stream=None):
+    s = torch.cuda.current_stream() if stream is None else stream
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _as_ft2_tensor(y: torch.Tensor) -> Tensor:
+    if y.dtype != torch.bfloat16:
+        raise TypeError("ft2: only bfloat16 activations are implemented")
+    if not y.is_cuda:
+        raise ValueError("ft2: tensor must live on a CUDA device (no CPU fallback)")
+    if y.dim() == 1:
+        y = y.view(1, -1)
+    if y.dim() != 2:
+        y2 = y.reshape(-1, y.shape[-1])
+        if y2.data_ptr() != y.data_ptr():
+            raise ValueError("ft2: tensor must be viewable as 2-D without a copy")
+        y = y2
+    if y.stride(1) != 1:
+        raise ValueError("ft2: rows must be contiguous (stride(-1) == 1)")
+    return Tensor(y.data_ptr(), y.shape[0], y.shape[1], y.stride(0), FT2_BF16)
+
+
+def workspace_bytes(num_seqs: int) -> int:
+    return int(load().ft2_workspace_bytes(num_seqs))
+
+
+def make_workspace(num_seqs: int, device=None) -> torch.Tensor:
+    """Zero-filled workspace for ft2_bounds_from_prefill (self-cleaning afterwards)."""
+    n = workspace_bytes(num_seqs)
+    return torch.zeros((n + 7) // 8, dtype=torch.int64, device=device or "cuda")
+
+
+def bounds_from_prefill(y, bounds_out, workspace, seq_offsets=None, num_seqs=None, scale=2.0,
+                        finalize=True, correct_nonfinite=False, keys_out=None, nonfinite_count=None,
+                        stream=None):
+    """ft2_bounds_from_prefill.  bounds_out: bf16 [S, 2] (or None when finalize=False)."""
+    t = _as_ft2_tensor(y)
+    S = num_seqs if num_seqs is not None else (1 if seq_offsets is None else seq_offsets.numel() - 1)
+    st = load().ft2_bounds_from_prefill(t, _ptr(seq_offsets), S, float(scale), int(finalize),
+                                        int(correct_nonfinite), _ptr(bounds_out), _ptr(keys_out),
+                                        _ptr(nonfinite_count), _ptr(workspace), _stream(stream))
+    check("ft2_bounds_from_prefill", st)
+
+
+def bounds_finalize(keys, bounds_out, scale=2.0, stream=None):
+    S = keys.numel() // 2
+    check("ft2_bounds_finalize", load().ft2_bounds_finalize(_ptr(keys), S, float(scale), FT2_BF16,
+                                                            _ptr(bounds_out), _stream(stream)))
+
+
+def protect(y, bounds, row_to_seq=None, num_seqs=None, corrected_count=None, stream=None):
+    """ft2_protect, in place on y (bf16 [rows, n])."""
+    t = _as_ft2_tensor(y)
+    S = num_seqs if num_seqs is not None else bounds.numel() // 2
+    check("ft2_protect", load().ft2_protect(t, _ptr(row_to_seq), _ptr(bounds), S, _ptr(corrected_count),
+                                            _stream(stream)))
+
+
+def protect_fused_gemm(x, w, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None, row_to_seq=None, num_seqs=None,
+                       corrected_count=None, col_begin=0, col_end=None, sites=None, n_sites=None,
+                       cur_layer=0, cur_step=0, base_row=None, workspace=None, stream=None):
+    """ft2_protect_fused_gemm: y = check(inject(bf16(x @ w.T + bias)))."""
+    M, K = x.shape
+    N = w.shape[0]
+    if col_end is None:
+        col_end = N
+    S = num_seqs if num_seqs is not None else (bounds.numel() // 2 if bounds is not None else 0)
+    ns = 0 if sites is None else (n_sites if n_sites is not None else sites.numel() // SITE_BYTES)
+    ws = 0 if workspace is None else workspace.numel() * workspace.element_size()
+    st = load().ft2_protect_fused_gemm(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y), y.stride(0),
+                                       M, N, K, int(mode), col_begin, col_end, _ptr(row_to_seq), _ptr(bounds), S,
+                                       _ptr(corrected_count), _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),
+                                       _ptr(workspace), ws, _stream(stream))
+    check("ft2_protect_fused_gemm", st)
+
+
+def make_fault_sites(seed, trial0, n_trials, model, layer_width, n_steps, prompt_len, out=None,
+                     layer_uniform=True, step_policy=0, device=None, stream=None):
+    """ft2_make_fault_sites -> uint8 tensor [n_trials * 24] (ft2_fault_site records)."""
+    widths = (ctypes.c_int32 * len(layer_width))(*[int(v) for v in layer_width])
+    g = SiteGeometry(n_steps, prompt_len, len(layer_width), widths, int(layer_uniform), int(step_policy))
+    if out is None:
+        out = torch.empty(n_trials * SITE_BYTES, dtype=torch.uint8, device=device or "cuda")
+    st = load().ft2_make_fault_sites(seed, trial0, n_trials, model, FT2_BF16, ctypes.byref(g), _ptr(out),
+                                     _stream(stream))
+    check("ft2_make_fault_sites", st)
+    return out
+
+
+def inject_faults(y, sites, cur_layer, cur_step, base_row=None, n_sites=None, stream=None):
+    t = _as_ft2_tensor(y)
+    ns = n_sites if n_sites is not None else sites.numel() // SITE_BYTES
+    check("ft2_inject_faults", load().ft2_inject_faults(t, _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),
+                                                        _stream(stream)))
+
+
+def launch_count() -> int:
+    return int(load().ft2_launch_count())
+
+
+def version() -> str:
+    return load().ft2_version().decode()

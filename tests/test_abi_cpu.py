@@ -1,0 +1,85 @@
+"""The C-ABI library loads and exports every symbol include/ft2.h declares;
+argument validation behaves as documented (no GPU needed: every case here
+returns before any CUDA call)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    from paper_conf_hpdc_sunzmg00y25_b200 import build as b
+    b.build()
+    from paper_conf_hpdc_sunzmg00y25_b200 import _lib
+    return _lib.load()
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "ft2.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(ft2_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_every_declared_symbol_is_exported(L):
+    decl = _declared()
+    assert len(decl) >= 10
+    for name in decl:
+        assert hasattr(L, name), name
+    from paper_conf_hpdc_sunzmg00y25_b200 import _lib
+    assert sorted(_lib.EXPORTS) == decl
+
+
+def test_status_strings_and_version(L):
+    assert L.ft2_status_string(0) == b"FT2_OK"
+    assert L.ft2_status_string(4) == b"FT2_ERR_CUDA"
+    assert L.ft2_version().startswith(b"ft2-b200")
+
+
+def test_workspace_bytes(L):
+    assert L.ft2_workspace_bytes(1) >= 4 * 7
+    assert L.ft2_workspace_bytes(1000) > L.ft2_workspace_bytes(1)
+
+
+def test_validation_without_gpu(L):
+    from paper_conf_hpdc_sunzmg00y25_b200._lib import (FT2_ERR_INVALID_ARG, FT2_ERR_MISALIGNED,
+                                                        FT2_ERR_UNSUPPORTED, FT2_OK, Tensor)
+    P = ctypes.c_void_p
+    good = Tensor(0x1000, 4, 16, 16, 0)
+    # NULL bounds / num_seqs < 1
+    assert L.ft2_protect(good, None, None, 1, None, None) == FT2_ERR_INVALID_ARG
+    assert L.ft2_protect(good, None, P(0x2000), 0, None, None) == FT2_ERR_INVALID_ARG
+    # ld < n, negative rows
+    assert L.ft2_protect(Tensor(0x1000, 4, 16, 8, 0), None, P(0x2000), 1, None, None) == FT2_ERR_INVALID_ARG
+    assert L.ft2_protect(Tensor(0x1000, -1, 16, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_INVALID_ARG
+    # misaligned base, n % 8
+    assert L.ft2_protect(Tensor(0x1002, 4, 16, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
+    assert L.ft2_protect(Tensor(0x1000, 4, 12, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
+    # dtype not implemented
+    assert L.ft2_protect(Tensor(0x1000, 4, 16, 16, 1), None, P(0x2000), 1, None, None) == FT2_ERR_UNSUPPORTED
+    # zero-size -> OK with no launch
+    n0 = L.ft2_launch_count()
+    assert L.ft2_protect(Tensor(0x1000, 0, 16, 16, 0), None, P(0x2000), 1, None, None) == FT2_OK
+    assert L.ft2_launch_count() == n0
+    # row_to_seq NULL needs num_seqs in {1, rows}
+    assert L.ft2_protect(good, None, P(0x2000), 3, None, None) == FT2_ERR_INVALID_ARG
+    # bounds: scale < 1, non-finite, missing workspace, correct without finalize
+    args = dict(so=None, S=1, fin=1, cor=0, b=P(0x3000), k=None, nf=None, ws=P(0x4000))
+    def bfp(scale, **kw):
+        a = dict(args, **kw)
+        return L.ft2_bounds_from_prefill(good, a["so"], a["S"], scale, a["fin"], a["cor"], a["b"], a["k"], a["nf"],
+                                         a["ws"], None)
+    assert bfp(0.5) == FT2_ERR_INVALID_ARG
+    assert bfp(float("nan")) == FT2_ERR_INVALID_ARG
+    assert bfp(2.0, ws=None) == FT2_ERR_INVALID_ARG
+    assert bfp(2.0, fin=0, cor=1, k=P(0x5000)) == FT2_ERR_INVALID_ARG
+    assert bfp(2.0, S=2) == FT2_ERR_INVALID_ARG       # several sequences need seq_offsets
+    # fused gemm: misaligned K
+    assert L.ft2_protect_fused_gemm(P(0x1000), 12, P(0x2000), 12, None, P(0x3000), 16, 4, 16, 12, 0, 0, 16,
+                                    None, None, 0, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_MISALIGNED
+    # fused gemm CHECK without bounds
+    assert L.ft2_protect_fused_gemm(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, 4, 16, 16, 1, 0, 16,
+                                    None, None, 1, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_INVALID_ARG
