@@ -1,0 +1,400 @@
+#!/usr/bin/env python
+"""FT2 on B200 -- headline benchmark (BASELINE.json configs[1]).
+
+Workload: OPT-1.3B-shaped decoder (24 blocks, hidden 2048, FFN 8192, 32 heads,
+vocab 50272; seeded synthetic weights, no checkpoint), batch 32, 128-token
+prompts, 60 generated tokens (the paper's QA length), FT2 on the
+72 critical layers (v_proj, out_proj, fc2 x 24; Table 1).
+
+One bench "step" = one whole generation request = the whole hot path once:
+a1 critical-layer selection (static), a2/a3 prefill bounds + non-finite
+correction on all 72 critical layers, a4/a5 59 decode steps with the check
+fused into the tcgen05 GEMM epilogue of every critical layer (CUDA graph),
+a6 (fault sites) is exercised by the campaign / parity tests (no faults are
+injected into the timed serving run).
+
+value = generated tokens/s with FT2 (fused) over all ranks; the unprotected
+run (cuBLAS linears, no FT2 work) is timed in the same process and reported
+as `unprotected` plus the overhead (paper's metric).
+
+Inputs larger than L2: every decode step streams 2.6 GB of weights (> 126 MB
+L2), so no explicit flush is needed; said in `config.l2`.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ft2", choices=["ft2", "reference"])
+    ap.add_argument("--model", default="opt-1.3b")
+    ap.add_argument("--batch", type=int, default=32)
+    ap.add_argument("--prompt", type=int, default=128)
+    ap.add_argument("--gen", type=int, default=60)
+    ap.add_argument("--no-extras", action="store_true", help="skip the kernel roofline / cpu baseline legs")
+    return ap.parse_args()
+
+
+def load_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev_index: int):
+        self.dev = dev_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        self.th.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [x.strip() for x in ln.split(",")]
+            if len(p) < 6:
+                continue
+            try:
+                sm.append(float(p[0]))
+                mx.append(float(p[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, p[2:6]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------ CPU baseline
+def oracle_sample(model_name, B, T, G, seed=1):
+    """Time the CPU oracle on a bounded sample of the same workload: the
+    critical layers (v_proj, out_proj, fc2) of ONE of the 24 blocks, for the
+    prefill bounds (+correction) and ONE decode step at batch B (fp64 linear ->
+    bf16 -> check-and-clip, R8 -> R5).  Extrapolated x n_layers x (G-1) decode
+    steps; attention / non-critical layers are outside the oracle (and outside
+    FT2's hot path) and are not counted.  Single-threaded C."""
+    import numpy as np
+
+    import ft2_synth
+    import oracle
+    from paper_conf_hpdc_sunzmg00y25_b200.runner import CONFIGS
+
+    cfg = CONFIGS[model_name]
+    crit = [(n, o, i) for n, o, i, c in cfg.linears() if c]
+    ws, bs = [], []
+    for j, (n, o, i) in enumerate(crit):
+        ws.append(ft2_synth.gen_bf16((o, i), 1000 + 2 * j, seed, scale_log2=ft2_synth.weight_scale_log2(i)))
+        bs.append(ft2_synth.gen_bf16((o,), 1001 + 2 * j, seed))
+    xs_dec = [ft2_synth.gen_bf16((B, i), 5000 + j, seed) for j, (n, o, i) in enumerate(crit)]
+    so = np.arange(0, (B + 1) * T, T, dtype=np.int32)
+    # prefill part: bounds of the 3 critical outputs of one block (outputs synthesised at prefill size)
+    ys_pre = [ft2_synth.gen_bf16((B * T, o), 6000 + j, seed) for j, (n, o, i) in enumerate(crit)]
+    t0 = time.perf_counter()
+    bounds = []
+    for y in ys_pre:
+        b, _, _ = oracle.bounds(y, seq_offsets=so, correct_nonfinite=True)
+        bounds.append(b)
+    t_pre = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    for j in range(len(crit)):
+        oracle.protected_linear(xs_dec[j], ws[j], bs[j], bounds[j], row_to_seq=np.arange(B, dtype=np.int32))
+    t_dec = time.perf_counter() - t0
+    per_request = cfg.n_layers * (t_pre + (G - 1) * t_dec)
+    return {"tokens_per_s": B * G / per_request, "t_prefill_block_s": t_pre, "t_decode_block_s": t_dec,
+            "sample": (f"critical layers ({', '.join(n for n, _, _ in crit)}) of 1 of {cfg.n_layers} blocks: "
+                       f"prefill bounds on [{B*T}, N] + 1 decode step at B={B} (fp64 linear + check); "
+                       f"extrapolated x{cfg.n_layers} blocks x{G-1} steps"),
+            "cores": 1}
+
+
+# ------------------------------------------------------------------ main
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        if rank != 0:
+            return 0
+        K, W = args.steps, args.warmup
+        for _ in range(min(W, 1)):
+            oracle_sample(args.model, args.batch, args.prompt, args.gen)
+        vals = []
+        t0 = time.perf_counter()
+        for _ in range(K):
+            r = oracle_sample(args.model, args.batch, args.prompt, args.gen)
+            vals.append(r["tokens_per_s"])
+        el = time.perf_counter() - t0
+        v = statistics.median(vals)
+        line = {"impl": "reference", "metric": "protected generated tokens/s (FT2 on critical layers)",
+                "value": v, "unit": "tokens/s", "n_gpus": args.gpus, "steps": K, "warmup": W,
+                "ms_per_step": 1000.0 * el / K, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64-accumulate/bf16", "data": "synthetic",
+                "config": {"workload": f"{args.model} decode, B={args.batch}, prompt {args.prompt}, gen {args.gen}",
+                           "model": args.model, "global_batch": args.batch, "seq_len": args.prompt + args.gen},
+                "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": r["cores"], "kind": "oracle",
+                                 "sample": r["sample"]},
+                "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return 0
+
+    import torch
+    import torch.distributed as dist
+
+    if world > 1:
+        dist.init_process_group("nccl")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+
+    import paper_conf_hpdc_sunzmg00y25_b200 as ft2
+    from paper_conf_hpdc_sunzmg00y25_b200.runner import CONFIGS, Runner
+
+    cfg = CONFIGS[args.model]
+    B, T, G = args.batch, args.prompt, args.gen
+    runner = Runner(cfg, B, T, G, seed=1, device=dev)
+    gen = torch.Generator().manual_seed(1234 + rank)
+    prompt_host = torch.randint(0, cfg.vocab, (B, T), generator=gen).pin_memory()
+    prompt = prompt_host.to(dev)
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def timed(mode, K, e2e=False):
+        out_host = torch.empty((B, G), dtype=torch.int64).pin_memory()
+        barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(K):
+            if e2e:
+                p = prompt_host.to(dev, non_blocking=True)
+                out = runner.generate(p, mode)
+                out_host.copy_(out, non_blocking=True)
+            else:
+                runner.generate(prompt, mode)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ms = e0.elapsed_time(e1) / K
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms
+
+    modes = ["fused", "off", "standalone", "fused_plain"]
+    # warm-up (captures the decode graphs of every mode)
+    for m in modes:
+        for _ in range(max(1, args.warmup if m == "fused" else 1)):
+            runner.generate(prompt, m)
+    torch.cuda.synchronize()
+
+    clk = ClockSampler(local)
+    clk.start()
+    n0 = ft2.launch_count()
+    ms_fused = timed("fused", args.steps)
+    clocks = clk.stop()
+    launches = runner.ft2_launches_per_request("fused") * args.steps
+    ms_off = timed("off", args.steps)
+    ms_stand = timed("standalone", args.steps)
+    ms_plain = timed("fused_plain", args.steps)
+    ms_e2e = timed("fused", args.steps, e2e=True)
+    # phase split and FT2 activity (outside the timed regions)
+    phases = {}
+    runner.time_phases = True
+    for m in modes:
+        runner.generate(prompt, m)
+        pre, dec = runner.phase_times()
+        phases[m] = {"prefill_ms": pre, "decode_ms_per_step": dec}
+    runner.time_phases = False
+    runner.generate(prompt, "fused")
+    torch.cuda.synchronize()
+    corrected = int(runner.state.corrected.sum().item())
+    nonfinite = int(runner.state.nonfinite.sum().item())
+
+    tok = B * G * world
+    value = tok / (ms_fused / 1000.0)
+    res = {
+        "metric": "protected generated tokens/s (FT2 on critical layers; overhead vs unprotected)",
+        "value": value, "unit": "tokens/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms_fused, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "bf16", "data": "synthetic (seeded weights and prompts; no checkpoint or dataset)",
+        "config": {"workload": f"{args.model}-shaped full decode with FT2 (configs[1]), B={B}/GPU, prompt {T}, "
+                               f"gen {G}", "model": args.model, "global_batch": B * world, "seq_len": T + G,
+                   "parallelism": f"dp{world} (independent replicas)", "protected_layers": runner.n_crit,
+                   "l2": "inputs larger than L2 (2.6 GB of weights streamed per decode step)"},
+        "modes_tokens_per_s": {"fused": value, "off": tok / (ms_off / 1e3), "standalone": tok / (ms_stand / 1e3),
+                               "fused_plain": tok / (ms_plain / 1e3)},
+        "overhead_pct_vs_unprotected": {"fused": 100.0 * (1 - ms_off / ms_fused),
+                                        "standalone": 100.0 * (1 - ms_off / ms_stand)},
+        "epilogue_overhead_pct": 100.0 * (1 - ms_plain / ms_fused),
+        "paper_context": "FT2 on A100 FP16, HF generate, B=1: 3.42% average overhead (PAPER.md L330) -- context only",
+        "e2e": {"value": tok / (ms_e2e / 1e3), "unit": "tokens/s", "h2d_bytes_per_step": B * T * 8,
+                "d2h_bytes_per_step": B * G * 8},
+        "gpu_launches": launches,
+        "phases": phases,
+        "ft2_activity_per_request": {"corrected_neurons": corrected, "prefill_nonfinite": nonfinite,
+                                     "checked_neurons": runner.B * (runner.G - 1) * sum(cfg.critical_widths())},
+        "clocks": clocks,
+    }
+
+    if not args.no_extras:
+        res.update(kernel_rooflines(runner, dev, ft2))
+    if rank == 0 and world == 1 and not args.no_extras:
+        cb = oracle_sample(args.model, B, T, G)
+        res["cpu_baseline"] = {"value": cb["tokens_per_s"], "unit": "tokens/s", "cores": cb["cores"],
+                               "kind": "oracle", "sample": cb["sample"]}
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def kernel_rooflines(runner, dev, ft2):
+    """Roofline of the dominant kernel (the fused critical-layer GEMM at its
+    decode shapes, in a CUDA graph of the 72 critical layers of one step) and
+    of the two protection kernels at the 1.44 GB Llama-2-7B prefill size."""
+    import torch
+
+    import ft2_synth
+
+    peaks = load_peaks()
+    hbm_peak = (peaks or {}).get("hbm_gbs", 6650.0)
+    peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if peaks else "fallback 6650 GB/s (B200_PROFILING.md)"
+    B = runner.B
+    stream = torch.cuda.current_stream()
+    # ---- fused GEMM, decode shapes, all critical layers of one step
+    xs = {}
+    launches = []
+    for blk in runner.blocks:
+        for name in runner.crit_names:
+            w, b = blk.w[name], blk.b[name]
+            K = w.shape[1]
+            if K not in xs:
+                xs[K] = ft2_synth.gen_bf16_torch((B, K), 77, K, device=dev)
+            y = torch.empty((B, w.shape[0]), dtype=torch.bfloat16, device=dev)
+            cid = runner._crit_id(blk.idx, name)
+            launches.append((xs[K], w, b, y, cid))
+    st = runner.state
+    big = torch.full((runner.n_crit, B, 2), 0, dtype=torch.bfloat16, device=dev)
+    big[..., 0] = -3.0e38
+    big[..., 1] = 3.0e38
+
+    def run_all():
+        for x, w, b, y, cid in launches:
+            ft2.protect_fused_gemm(x, w, y, bias=b, mode=1 | 16, bounds=big[cid], num_seqs=B,
+                                   corrected_count=st.corrected[cid])
+
+    run_all()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        run_all()
+    for _ in range(3):
+        g.replay()
+    R = 20
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(R):
+        g.replay()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / R
+    nbytes = sum(w.numel() * 2 + x.numel() * 2 + y.numel() * 2 + (b.numel() * 2 if b is not None else 0)
+                 for x, w, b, y, _ in launches)
+    per_launch_us = 1000.0 * ms / len(launches)
+    ach = nbytes / (ms / 1e3) / 1e9
+    gemm = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+            "traffic": None, "kernel": "ft2 gemm_kernel (tcgen05, CHECK epilogue)",
+            "shapes": f"M={B}; (N,K) per block: " + ", ".join(
+                f"{blk_w.shape[0]}x{blk_w.shape[1]}" for blk_w in [runner.blocks[0].w[n] for n in runner.crit_names]),
+            "launches_per_graph": len(launches), "avg_launch_us": per_launch_us,
+            "bytes_per_launch_avg": nbytes / len(launches), "peak_source": peak_src,
+            "algorithmic_bytes": "N*K*2 (W) + M*K*2 (x) + M*N*2 (y) + N*2 (bias) per launch"}
+    # ---- protection kernels at the 1.44 GB size
+    rows, n = 65536, 11008
+    y = ft2_synth.gen_bf16_torch((rows, n), 11, 5, device=dev)
+    ws = ft2.make_workspace(1, device=dev)
+    bnd = torch.zeros((1, 2), dtype=torch.bfloat16, device=dev)
+    wide = torch.tensor([[-3.0e38, 3.0e38]], dtype=torch.bfloat16, device=dev)
+    cnt = torch.zeros(1, dtype=torch.int32, device=dev)
+
+    def time_it(fn, R=20):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(R):
+            fn()
+        b_.record(stream)
+        torch.cuda.synchronize()
+        return a.elapsed_time(b_) / R
+
+    ms_b = time_it(lambda: ft2.bounds_from_prefill(y, bnd, ws))
+    ms_p = time_it(lambda: ft2.protect(y, wide, corrected_count=cnt))
+    nb = rows * n * 2
+    prot = {
+        "bounds": {"bound": "hbm", "achieved": nb / (ms_b / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
+                   "frac": nb / (ms_b / 1e3) / 1e9 / hbm_peak, "traffic": None, "us": 1000 * ms_b,
+                   "shape": [rows, n], "algorithmic_bytes": "2 B read per element"},
+        "protect": {"bound": "hbm", "achieved": nb / (ms_p / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
+                    "frac": nb / (ms_p / 1e3) / 1e9 / hbm_peak, "traffic": None, "us": 1000 * ms_p,
+                    "shape": [rows, n], "algorithmic_bytes": "2 B read per element (no element out of bounds)"},
+        "peak_source": peak_src,
+    }
+    del y
+    torch.cuda.empty_cache()
+    return {"roofline": gemm, "protect_kernels_roofline": prot}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -69,7 +69,11 @@ typedef enum { FT2_FAULT_1BIT = 0, FT2_FAULT_2BIT = 1, FT2_FAULT_EXP = 2 } ft2_f
 /* Epilogue of ft2_protect_fused_gemm. */
 typedef enum {
     FT2_GEMM_PLAIN = 0, /* y = x W^T + b (+ faults), no check: the unprotected baseline */
-    FT2_GEMM_CHECK = 1  /* ... then the check-and-clip of ft2_protect on the bf16 result */
+    FT2_GEMM_CHECK = 1, /* ... then the check-and-clip of ft2_protect on the bf16 result */
+    /* flag, OR-ed into the mode: w is not written by the kernel that precedes
+     * this call in the stream (e.g. model weights), so its first tiles may be
+     * fetched before the programmatic-dependent-launch wait. */
+    FT2_GEMM_W_STATIC = 16
 } ft2_gemm_mode;
 
 typedef struct {
@@ -186,7 +190,16 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
  * sites/n_sites/cur_layer/cur_step/base_row  optional fault injection applied
  *              to the bf16 result before the check (order: GEMM -> bias -> bf16 ->
  *              inject -> check; readings A19, A20), as in ft2_inject_faults.
- * workspace/ws_bytes  scratch of ft2_gemm_workspace_bytes(M, N, K) bytes (may be 0).
+ * workspace/ws_bytes  at least ft2_gemm_workspace_bytes(M, N, K) bytes, 16-byte
+ *              aligned (may be NULL when that is 0): split-K partial tiles and
+ *              per-tile arrival counters.  Zero-filled once before first use; every
+ *              call leaves the counters zero again.  The split-K partial sums are
+ *              combined in a fixed order, so results are deterministic.  At most
+ *              16 MiB for any shape on a 148-SM B200.
+ * The kernel is launched with programmatic stream serialization (PDL): its
+ * prologue and first weight tiles overlap the previous kernel's tail; it reads
+ * x, bias, bounds, sites and writes y, counters, workspace only after the
+ * previous kernel has completed.
  * Limits: K % 8 == 0, ldx/ldw/ldy % 8 == 0, 16-byte aligned bases, M, N >= 1. */
 size_t ft2_gemm_workspace_bytes(int32_t M, int32_t N, int32_t K);
 ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw,

@@ -14,7 +14,7 @@ from .build import LIB
 FT2_OK, FT2_ERR_INVALID_ARG, FT2_ERR_MISALIGNED, FT2_ERR_UNSUPPORTED, FT2_ERR_CUDA = range(5)
 FT2_BF16, FT2_FP16, FT2_FP32 = 0, 1, 2
 FT2_FAULT_1BIT, FT2_FAULT_2BIT, FT2_FAULT_EXP = 0, 1, 2
-FT2_GEMM_PLAIN, FT2_GEMM_CHECK = 0, 1
+FT2_GEMM_PLAIN, FT2_GEMM_CHECK, FT2_GEMM_W_STATIC = 0, 1, 16
 FT2_MAX_SITE_LAYERS = 1024
 FT2_MAX_SEQS = 65535
 

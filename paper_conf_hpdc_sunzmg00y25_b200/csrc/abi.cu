@@ -146,6 +146,8 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
     if (K == 0) return FT2_ERR_UNSUPPORTED;
     if (x == nullptr || w == nullptr || y == nullptr) return FT2_ERR_INVALID_ARG;
     if (ldx < K || ldw < K || ldy < N) return FT2_ERR_INVALID_ARG;
+    const int32_t w_static = (mode & FT2_GEMM_W_STATIC) ? 1 : 0;
+    mode = (ft2_gemm_mode)(mode & ~FT2_GEMM_W_STATIC);
     if (mode != FT2_GEMM_PLAIN && mode != FT2_GEMM_CHECK) return FT2_ERR_INVALID_ARG;
     if (!al16(x) || !al16(w) || !al16(y) || (bias && ((uintptr_t)bias & 1u)) || (K % 8) || (ldx % 8) ||
         (ldw % 8) || (ldy % 8))
@@ -156,7 +158,9 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
         if (col_begin < 0 || col_end > N || col_begin > col_end) return FT2_ERR_INVALID_ARG;
     }
     if (n_sites < 0 || (n_sites > 0 && sites == nullptr)) return FT2_ERR_INVALID_ARG;
-    if (ws_bytes < gemm_ws_bytes(M, N, K)) return FT2_ERR_INVALID_ARG;
+    const size_t need = gemm_ws_bytes(M, N, K);
+    if (need > 0 && (workspace == nullptr || ws_bytes < need)) return FT2_ERR_INVALID_ARG;
+    if (need > 0 && !al16(workspace)) return FT2_ERR_MISALIGNED;
     GemmArgs a;
     a.x = static_cast<const uint16_t*>(x);
     a.ldx = ldx;
@@ -182,6 +186,7 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
     a.base_row = base_row;
     a.ws = workspace;
     a.ws_bytes = ws_bytes;
+    a.w_static = w_static;
     int nl = 0;
     cudaError_t e = launch_gemm(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);

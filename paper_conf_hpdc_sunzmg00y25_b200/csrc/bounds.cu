@@ -245,6 +245,11 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
         }
     }
     __syncthreads();
+    if (p.correct) {  // leave the patch list zero-filled as well
+        uint32_t used = min(atomicAdd(ws_lc, 0u), (uint32_t)kPatchCap);
+        for (uint32_t i = tid; i < used; i += kThreads) list[i] = 0ull;
+    }
+    __syncthreads();
     if (tid == 0) {
         *ws_lc = 0u;
         *ws_ov = 0u;

@@ -66,6 +66,7 @@ struct GemmArgs {
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
     void* ws; size_t ws_bytes;
+    int32_t w_static;
 };
 size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch);

@@ -29,6 +29,7 @@
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
 #include <stdio.h>
+#include <stdlib.h>
 
 #include <mutex>
 
@@ -43,6 +44,11 @@ constexpr int kBlockK = 64;    // one 128-byte swizzle atom of bf16
 constexpr int kUmmaK = 16;
 constexpr int kGemmThreads = 192;
 constexpr int kMaxSitesPerCta = 64;
+// Split-K tile counters live in a fixed region at the start of the workspace
+// (independent of the shape, so one workspace can serve every GEMM); split-K
+// is only used when tiles * splitk fits one co-resident wave, i.e. tiles <= 2 x SMs.
+constexpr int kMaxSplitTiles = 1024;
+constexpr size_t kCounterBytes = (size_t)kMaxSplitTiles * 8;
 
 // ------------------------------------------------------------------ PTX glue
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -148,8 +154,9 @@ __host__ __device__ constexpr uint32_t make_idesc(int m, int n) {
 
 struct GemmK {
     int32_t M, N, K;
-    int32_t swap;         // 1: A = w (features), B = x (tokens)
-    int32_t rowsA, rowsB; // extent of the A / B operands
+    int32_t swap;          // 1: A = w (features), B = x (tokens)
+    int32_t rowsA, rowsB;  // extent of the A / B operands
+    int32_t tilesA, tilesB;
     int32_t splitk, nkb;
     int32_t mode, col_begin, col_end;
     const uint16_t* bias;
@@ -162,6 +169,9 @@ struct GemmK {
     const ft2_fault_site* sites;
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
+    float4* partials;      // [tiles][splitk][BN/4][128] float4 (split-K only)
+    uint32_t* tile_ctr;    // [tiles][2] self-resetting arrival / departure counters
+    int32_t w_static;      // weights not written by the preceding kernel: prefetch before the PDL wait
 };
 
 template <int BN, int STAGES>
@@ -169,11 +179,97 @@ struct GemmSmem {
     static constexpr int kABytes = kBlockA * kBlockK * 2;
     static constexpr int kBBytes = BN * kBlockK * 2;
     static constexpr int kStageBytes = kABytes + kBBytes;
-    static constexpr int kRedStride = BN + 1;  // padded fp32 row (bank-conflict free)
-    static constexpr int kRedBytes = kBlockA * kRedStride * 4;
-    static constexpr int kTileBytes = STAGES * kStageBytes > kRedBytes ? STAGES * kStageBytes : kRedBytes;
-    static constexpr int kBytes = 1024 /*align slack*/ + kTileBytes + 1024 /*barriers etc*/;
+    static constexpr int kTileBytes = STAGES * kStageBytes;
+    static constexpr int kBytes = 1024 /*align slack*/ + kTileBytes + 1024 /*barriers, site list*/ + (BN + 128) * 20;
 };
+
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void griddep_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+// Per-row / per-column epilogue context.  In swap-AB mode rows are output
+// features (bias, protected-slice flag per row) and columns are tokens (bounds
+// per column); otherwise the other way round.  `keys` packs key(lo) | key(hi) << 16;
+// seq < 0 means "do not check".
+struct EpiSide {
+    float bias;
+    uint32_t keys;
+    int32_t seq;
+    int32_t valid;  // index inside [0, M) / [0, N)
+};
+
+__device__ __forceinline__ EpiSide make_side(const GemmK& p, bool is_token, int idx) {
+    EpiSide e{0.f, 0u, -1, 0};
+    if (is_token) {
+        e.valid = idx < p.M;
+        if (e.valid && p.mode == FT2_GEMM_CHECK) {
+            const int s = p.row_mode == 2 ? 0 : (p.row_mode == 1 ? idx : p.row_to_seq[idx]);
+            if (s >= 0 && s < p.S) {
+                const uint32_t lh = (uint32_t)p.bounds[2 * s] | ((uint32_t)p.bounds[2 * s + 1] << 16);
+                e.keys = key2(lh);
+                e.seq = s;
+            }
+        }
+    } else {
+        e.valid = idx < p.N;
+        if (e.valid) {
+            if (p.bias) e.bias = __uint_as_float((uint32_t)p.bias[idx] << 16);
+            e.seq = (p.mode == FT2_GEMM_CHECK && idx >= p.col_begin && idx < p.col_end) ? 0 : -1;  // flag only
+        }
+    }
+    return e;
+}
+
+// Four consecutive columns c..c+3 of one row: all four values are computed
+// before any side effect (stores, counter atomics), so the chains overlap.
+__device__ __forceinline__ void finish4(const GemmK& p, int ga, int gb0, const EpiSide& rs, const EpiSide* cs,
+                                        int la_c0, const float (&acc)[4], const uint32_t* site_e,
+                                        const uint32_t* site_m, uint32_t nsite, uint32_t* row_cnt,
+                                        uint32_t* col_cnt) {
+    uint16_t o[4];
+    bool ok[4];
+    uint32_t changed = 0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const EpiSide& feat = p.swap ? rs : cs[j];
+        const EpiSide& tok = p.swap ? cs[j] : rs;
+        ok[j] = feat.valid && tok.valid;
+        uint16_t x = bf16_rne(acc[j] + feat.bias);
+        for (uint32_t i = 0; i < nsite; ++i)
+            if (site_e[i] == (uint32_t)(la_c0 + j)) x ^= (uint16_t)site_m[i];
+        const bool chk = feat.seq >= 0 && tok.seq >= 0;
+        const uint16_t z = ((x & 0x7FFF) > 0x7F80) ? (uint16_t)0 : x;  // NaN -> +0
+        const uint16_t k = key1(z);
+        const uint16_t kl = (uint16_t)tok.keys, kh = (uint16_t)(tok.keys >> 16);
+        const uint16_t c = k < kl ? unkey1(kl) : (k > kh ? unkey1(kh) : z);
+        o[j] = chk ? c : x;
+        changed |= (ok[j] && o[j] != x) ? (1u << j) : 0u;
+    }
+    if (p.swap) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+            if (ok[j]) p.y[(int64_t)(gb0 + j) * p.ldy + ga] = o[j];
+    } else {
+        uint16_t* dst = p.y + (int64_t)ga * p.ldy + gb0;
+        if (ok[0] && ok[3] && ((reinterpret_cast<uintptr_t>(dst) & 7u) == 0)) {
+            *reinterpret_cast<uint2*>(dst) = make_uint2((uint32_t)o[0] | ((uint32_t)o[1] << 16),
+                                                        (uint32_t)o[2] | ((uint32_t)o[3] << 16));
+        } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                if (ok[j]) dst[j] = o[j];
+        }
+    }
+    if (changed) {  // corrected neurons, aggregated per CTA in shared memory
+        if (p.swap) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                if (changed & (1u << j)) atomicAdd_block(&col_cnt[j], 1u);
+        } else {
+            atomicAdd_block(row_cnt, (uint32_t)__popc(changed));
+        }
+    }
+}
 
 template <int BN, int STAGES>
 __global__ void __launch_bounds__(kGemmThreads, 1)
@@ -187,16 +283,19 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     uint64_t* empty = full + STAGES;
     uint64_t* tmem_full = empty + STAGES;
     uint32_t* tmem_base_sh = reinterpret_cast<uint32_t*>(tmem_full + 1);
-    uint32_t* site_n = tmem_base_sh + 1;
-    uint32_t* site_e = site_n + 1;           // [kMaxSitesPerCta] local element index
-    uint32_t* site_m = site_e + kMaxSitesPerCta;  // [kMaxSitesPerCta] xor mask
-    float* red = reinterpret_cast<float*>(tiles);  // aliases the stage ring after the MMAs
+    uint32_t* flag_sh = tmem_base_sh + 1;
+    uint32_t* site_n = flag_sh + 1;
+    uint32_t* site_e = site_n + 1;                 // [kMaxSitesPerCta] local element index (a * BN + c)
+    uint32_t* site_m = site_e + kMaxSitesPerCta;   // [kMaxSitesPerCta] xor mask
+    EpiSide* col_side = reinterpret_cast<EpiSide*>(site_m + kMaxSitesPerCta);  // [BN] per-column context
+    EpiSide* row_side = col_side + BN;                                        // [128] per-row context
+    uint32_t* col_cnt = reinterpret_cast<uint32_t*>(row_side + 128);          // [BN] corrected per column
+    uint32_t* row_cnt = col_cnt + BN;                                         // [128] corrected per row
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int tileA = blockIdx.x, tileB = blockIdx.z;
-    const uint32_t rank = p.splitk > 1 ? cluster_rank() : 0u;
-    const int kb0 = (int)((int64_t)rank * p.nkb / p.splitk);
-    const int kb1 = (int)((int64_t)(rank + 1) * p.nkb / p.splitk);
+    const int tileA = blockIdx.x, split = blockIdx.y, tileB = blockIdx.z;
+    const int kb0 = (int)((int64_t)split * p.nkb / p.splitk);
+    const int kb1 = (int)((int64_t)(split + 1) * p.nkb / p.splitk);
     const int nk = kb1 - kb0;
     constexpr uint32_t kTmemCols = BN < 32 ? 32 : BN;
 
@@ -217,20 +316,40 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_base_sh;
+    // the next kernel in the stream may start its own prologue now (PDL)
+    griddep_launch();
 
     if (warp == 0) {
         if (lane == 0) {
             // ------------------------------------------------ TMA producer
-            for (int i = 0; i < nk; ++i) {
+            // The weight operand does not depend on the previous kernel: the
+            // first STAGES weight tiles are requested before waiting for it
+            // (programmatic dependent launch), the activations after.
+            const CUtensorMap* mw = p.swap ? &map_a : &map_b;
+            const CUtensorMap* mx = p.swap ? &map_b : &map_a;
+            const int w_row = p.swap ? tileA * kBlockA : tileB * BN;
+            const int x_row = p.swap ? tileB * BN : tileA * kBlockA;
+            const int w_off = p.swap ? 0 : L::kABytes;
+            const int x_off = p.swap ? L::kABytes : 0;
+            const int pre = nk < STAGES ? nk : STAGES;
+            if (!p.w_static) griddep_wait();
+            for (int i = 0; i < pre; ++i) {
+                uint8_t* st = tiles + i * L::kStageBytes;
+                mbar_expect_tx(&full[i], L::kStageBytes);
+                tma_load_2d(mw, &full[i], st + w_off, (kb0 + i) * kBlockK, w_row);
+            }
+            if (p.w_static) griddep_wait();
+            for (int i = 0; i < pre; ++i)
+                tma_load_2d(mx, &full[i], tiles + i * L::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row);
+            for (int i = STAGES; i < nk; ++i) {
                 const int s = i % STAGES;
                 const uint32_t ph = (uint32_t)(i / STAGES) & 1u;
-                if (i >= STAGES) mbar_wait(&empty[s], ph ^ 1u);
-                uint8_t* sa = tiles + s * L::kStageBytes;
-                uint8_t* sb = sa + L::kABytes;
+                mbar_wait(&empty[s], ph ^ 1u);
+                uint8_t* st = tiles + s * L::kStageBytes;
                 mbar_expect_tx(&full[s], L::kStageBytes);
                 const int kc = (kb0 + i) * kBlockK;
-                tma_load_2d(&map_a, &full[s], sa, kc, tileA * kBlockA);
-                tma_load_2d(&map_b, &full[s], sb, kc, tileB * BN);
+                tma_load_2d(mw, &full[s], st + w_off, kc, w_row);
+                tma_load_2d(mx, &full[s], st + x_off, kc, x_row);
             }
         }
     } else if (warp == 1) {
@@ -246,108 +365,147 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 const uint32_t sb = sa + L::kABytes;
                 const uint64_t da = make_sdesc(sa), db = make_sdesc(sb);
 #pragma unroll
-                for (int k = 0; k < kBlockK / kUmmaK; ++k) {
-                    // advance 16 elements (32 B) along K inside the swizzle atom
+                for (int k = 0; k < kBlockK / kUmmaK; ++k)  // 16 elements = 32 B along K per MMA
                     tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc,
                            (i > 0 || k > 0) ? 1u : 0u);
-                }
                 tc_commit(&empty[s]);
             }
             tc_commit(tmem_full);
         }
     } else {
         // ---------------------------------------------------- epilogue warps
-        const int q = warp & 3;  // TMEM lane quarter this warp may access
-        mbar_wait(tmem_full, 0);
-        tc_fence_after();
-        const int row = q * 32 + lane;
+        const int q = warp & 3;               // TMEM lane quarter this warp may access
+        const int a = q * 32 + lane;          // row of the A tile owned by this thread
+        const int et = a;                     // epilogue thread index 0..127
         const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
-        if (BN >= 32) {
-#pragma unroll 1
-            for (int c = 0; c < BN; c += 32) {
-                uint32_t r[32];
-                tmem_ld32(taddr + c, r);
-                tmem_wait_ld();
-#pragma unroll
-                for (int j = 0; j < 32; ++j) red[row * L::kRedStride + c + j] = nk > 0 ? __uint_as_float(r[j]) : 0.f;
-            }
-        } else {
-            uint32_t r[16];
-            tmem_ld16(taddr, r);
-            tmem_wait_ld();
-#pragma unroll
-            for (int j = 0; j < 16; ++j) red[row * L::kRedStride + j] = nk > 0 ? __uint_as_float(r[j]) : 0.f;
+        const int ga = tileA * kBlockA + a;
+        const int tile = tileB * p.tilesA + tileA;
+        griddep_wait();                       // bias/bounds/y/workspace may belong to the previous kernel
+        // rows of the 128-row A tile this CTA finishes: all of them without
+        // split-K, else the split's 1/splitk slice (distributed reduction)
+        const int r0 = (split * kBlockA) / p.splitk, r1 = ((split + 1) * kBlockA) / p.splitk;
+        // epilogue contexts (bias, bound keys) are gathered while the main loop
+        // still runs: columns are tokens in swap-AB mode, features otherwise
+        for (int c = et; c < BN; c += 128) {
+            col_side[c] = make_side(p, p.swap != 0, tileB * BN + c);
+            col_cnt[c] = 0u;
         }
-    }
-    tc_fence_before();
-    __syncthreads();
-
-    // --------------------------------------------- fault sites of this CTA
-    const int rows_per = kBlockA / p.splitk;
-    const int a0 = (int)rank * rows_per;  // my rows of the 128 x BN tile
-    if (p.sites != nullptr) {
-        for (int i = threadIdx.x; i < p.n_sites; i += kGemmThreads) {
-            ft2_fault_site st = p.sites[i];
-            if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
-            int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) + (p.cur_step == 0 ? (int64_t)st.token : 0);
-            int64_t n = st.col;
-            if (m < 0 || m >= p.M || n >= p.N) continue;
-            int64_t ga = p.swap ? n : m, gb = p.swap ? m : n;  // global A / B row
-            int64_t la = ga - (int64_t)tileA * kBlockA - a0, lb = gb - (int64_t)tileB * BN;
-            if (la < 0 || la >= rows_per || lb < 0 || lb >= BN) continue;
-            uint32_t idx = atomicAdd(site_n, 1u);
-            if (idx < (uint32_t)kMaxSitesPerCta) {
-                site_e[idx] = (uint32_t)(la * BN + lb);
-                site_m[idx] = st.xor_mask;
-            }
-        }
-    }
-    if (p.splitk > 1) cluster_sync_all();
-    else __syncthreads();
-    const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
-
-    // ------------------------------------------ split-K combine + epilogue
-    const uint32_t red_base = smem_u32(red);
-    const int elems = rows_per * BN;
-    for (int e = threadIdx.x; e < elems; e += kGemmThreads) {
-        int la, lb;
-        if (p.swap) { la = e % rows_per; lb = e / rows_per; }   // consecutive threads: consecutive features
-        else        { lb = e % BN;       la = e / BN; }
-        const int a = a0 + la;
-        const int ga = tileA * kBlockA + a, gb = tileB * BN + lb;
-        const int m = p.swap ? gb : ga, n = p.swap ? ga : gb;
-        float acc;
-        const uint32_t off = (uint32_t)(a * L::kRedStride + lb) * 4u;
-        if (p.splitk > 1) {
-            acc = 0.f;
-            for (int r = 0; r < p.splitk; ++r) acc += ld_dsmem_f32(mapa(red_base + off, (uint32_t)r));
-        } else {
-            acc = red[a * L::kRedStride + lb];
-        }
-        if (m >= p.M || n >= p.N) continue;
-        if (p.bias) acc += __uint_as_float((uint32_t)p.bias[n] << 16);
-        uint16_t v = bf16_rne(acc);
-        const uint32_t le = (uint32_t)(la * BN + lb);
-        for (uint32_t i = 0; i < nsite; ++i)
-            if (site_e[i] == le) v ^= (uint16_t)site_m[i];
-        if (p.mode == FT2_GEMM_CHECK && n >= p.col_begin && n < p.col_end) {
-            int s = p.row_mode == 2 ? 0 : (p.row_mode == 1 ? m : p.row_to_seq[m]);
-            if (s >= 0 && s < p.S) {
-                uint16_t lo = p.bounds[2 * s], hi = p.bounds[2 * s + 1];
-                uint16_t x = ((v & 0x7FFF) > 0x7F80) ? (uint16_t)0 : v;   // NaN -> +0
-                uint16_t k = key1(x);
-                uint16_t o = k < key1(lo) ? lo : (k > key1(hi) ? hi : x);
-                if (o != v) {
-                    v = o;
-                    if (p.counts) atomicAdd(&p.counts[s], 1u);
+        row_side[et] = make_side(p, p.swap == 0, ga);
+        row_cnt[et] = 0u;
+        // fault sites that land in this CTA's output slice
+        if (p.sites != nullptr) {
+            for (int i = et; i < p.n_sites; i += 128) {
+                ft2_fault_site st = p.sites[i];
+                if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
+                int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
+                            (p.cur_step == 0 ? (int64_t)st.token : 0);
+                int64_t n = st.col;
+                if (m < 0 || m >= p.M || n >= p.N) continue;
+                int64_t la = (p.swap ? n : m) - (int64_t)tileA * kBlockA;
+                int64_t lb = (p.swap ? m : n) - (int64_t)tileB * BN;
+                if (la < r0 || la >= r1 || lb < 0 || lb >= BN) continue;
+                uint32_t idx = atomicAdd(site_n, 1u);
+                if (idx < (uint32_t)kMaxSitesPerCta) {
+                    site_e[idx] = (uint32_t)(la * BN + lb);
+                    site_m[idx] = st.xor_mask;
                 }
             }
         }
-        p.y[(int64_t)m * p.ldy + n] = v;
+        mbar_wait(tmem_full, 0);
+        tc_fence_after();
+        if (p.splitk == 1) {
+            epi_bar();
+            const EpiSide rs = row_side[et];
+            const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
+#pragma unroll 1
+            for (int c0 = 0; c0 < BN; c0 += 16) {
+                uint32_t r[16];
+                tmem_ld16(taddr + c0, r);
+                tmem_wait_ld();
+#pragma unroll
+                for (int j = 0; j < 16; j += 4) {
+                    const float acc[4] = {nk > 0 ? __uint_as_float(r[j]) : 0.f, nk > 0 ? __uint_as_float(r[j + 1]) : 0.f,
+                                          nk > 0 ? __uint_as_float(r[j + 2]) : 0.f, nk > 0 ? __uint_as_float(r[j + 3]) : 0.f};
+                    finish4(p, ga, tileB * BN + c0 + j, rs, col_side + c0 + j, a * BN + c0 + j, acc, site_e, site_m,
+                            nsite, row_cnt + et, col_cnt + c0 + j);
+                }
+            }
+        } else {
+            // 1. publish this split's fp32 partial tile (coalesced float4 columns)
+            float4* tbase = p.partials + (size_t)tile * p.splitk * (BN / 4) * kBlockA;
+            float4* mine = tbase + (size_t)split * (BN / 4) * kBlockA;
+#pragma unroll 1
+            for (int c0 = 0; c0 < BN; c0 += 16) {
+                uint32_t r[16];
+                tmem_ld16(taddr + c0, r);
+                tmem_wait_ld();
+#pragma unroll
+                for (int j = 0; j < 16; j += 4)
+                    __stcg(&mine[((c0 + j) / 4) * kBlockA + a],
+                           make_float4(__uint_as_float(r[j]), __uint_as_float(r[j + 1]), __uint_as_float(r[j + 2]),
+                                       __uint_as_float(r[j + 3])));
+            }
+            epi_bar();
+            // 2. wait until every split of this tile has published.  All split
+            // CTAs are co-resident: the grid never exceeds one wave (<= 1 CTA
+            // per SM), and PDL dependents launch only after all CTAs started.
+            uint32_t* arrive = p.tile_ctr + 2 * tile;
+            uint32_t* depart = arrive + 1;
+            if (et == 0) {
+                // release: the barrier above orders every epilogue thread's partial stores before it
+                asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(arrive) : "memory");
+                uint32_t seen, ns = 32;
+                while (true) {
+                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(seen) : "l"(arrive) : "memory");
+                    if (seen >= (uint32_t)p.splitk) break;
+                    __nanosleep(ns);
+                    if (ns < 256) ns <<= 1;
+                }
+            }
+            epi_bar();  // thread 0's acquire is ordered before everyone's partial loads
+            const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
+            // 3. reduce my row slice over all splits in fixed order 0..splitk-1
+            const int nrow = r1 - r0;
+            const int nvec = nrow * (BN / 4);
+            for (int v = et; v < nvec; v += 128) {
+                const int la = r0 + v % nrow, c4 = v / nrow;
+                float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+                float4 part[16];
+#pragma unroll
+                for (int rr = 0; rr < 16; ++rr)
+                    if (rr < p.splitk) part[rr] = __ldcg(&tbase[((size_t)rr * (BN / 4) + c4) * kBlockA + la]);
+#pragma unroll
+                for (int rr = 0; rr < 16; ++rr)
+                    if (rr < p.splitk) {
+                        acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w;
+                    }
+                const int gla = tileA * kBlockA + la;
+                const EpiSide rs = row_side[la];
+                const float av[4] = {acc.x, acc.y, acc.z, acc.w};
+                finish4(p, gla, tileB * BN + c4 * 4, rs, col_side + c4 * 4, la * BN + c4 * 4, av, site_e, site_m,
+                        nsite, row_cnt + la, col_cnt + c4 * 4);
+            }
+            // 4. the last CTA to leave resets the counters for the next launch
+            epi_bar();
+            if (et == 0) {
+                if (atomicAdd(depart, 1u) == (uint32_t)p.splitk - 1) {
+                    *arrive = 0u;
+                    *depart = 0u;
+                }
+            }
+        }
     }
-    if (p.splitk > 1) cluster_sync_all();  // peers may still read my partial tile
+    if (warp >= 2 && p.counts != nullptr && p.mode == FT2_GEMM_CHECK) {
+        epi_bar();  // every finish4 of this CTA has counted
+        const int et = (warp & 3) * 32 + lane;
+        for (int c = et; c < BN; c += 128)
+            if (col_cnt[c] != 0u && col_side[c].seq >= 0 && p.swap) atomicAdd(&p.counts[col_side[c].seq], col_cnt[c]);
+        if (!p.swap && row_cnt[et] != 0u && row_side[et].seq >= 0) atomicAdd(&p.counts[row_side[et].seq], row_cnt[et]);
+    }
+    tc_fence_before();
+    __syncthreads();
     if (warp == 1) {
-        __syncwarp();
+        tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(kTmemCols));
     }
 }
@@ -379,7 +537,59 @@ static bool make_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, 
     return r == CUDA_SUCCESS;
 }
 
-size_t gemm_ws_bytes(int32_t, int32_t, int32_t) { return 0; }
+// Tiling plan shared by the workspace query and the launch.
+struct GemmPlan {
+    int swap, bn, tilesA, tilesB, splitk, nkb;
+};
+
+// Pipeline depth per BN: BN <= 64 keeps a CTA at <= ~110 KB of shared memory so
+// two CTAs fit on an SM (split-K CTAs of one tile must be co-resident).
+template <int BN> struct Stages { static constexpr int value = BN <= 16 ? 6 : (BN <= 32 ? 5 : (BN <= 64 ? 4 : 6)); };
+static int ctas_per_sm(int bn) {
+    static const int deep32 = [] { const char* e = getenv("FT2_GEMM_STAGES32"); return e ? atoi(e) : 0; }();
+    if (bn == 32 && deep32 >= 8) return 1;
+    return bn <= 64 ? 2 : 1;
+}
+
+static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
+    GemmPlan g;
+    g.swap = M <= 128 ? 1 : 0;
+    g.bn = g.swap ? (M <= 16 ? 16 : (M <= 32 ? 32 : (M <= 64 ? 64 : 128))) : 128;
+    const int rowsA = g.swap ? N : M, rowsB = g.swap ? M : N;
+    g.tilesA = (rowsA + kBlockA - 1) / kBlockA;
+    g.tilesB = (rowsB + g.bn - 1) / g.bn;
+    g.nkb = (K + kBlockK - 1) / kBlockK;
+    const int tiles = g.tilesA * g.tilesB;
+    const int sms = num_sms();
+    const int capacity = sms * ctas_per_sm(g.bn);
+    // Split K so the busiest SM streams as little of one tile's weights as
+    // possible: load(sk) = ceil(tiles*sk / sms) / sk, with a small penalty per
+    // split for the partial-tile traffic; all CTAs must be co-resident and keep
+    // >= 2 k-blocks each.
+    int best = 1;
+    double best_cost = 1e30;
+    for (int sk = 1; sk <= 16; ++sk) {
+        if (sk > 1 && (tiles * sk > capacity || sk * 2 > g.nkb || tiles > kMaxSplitTiles)) break;
+        const double load = (double)((tiles * sk + sms - 1) / sms) / sk;
+        const double cost = load * (1.0 + 0.03 * sk);
+        if (cost < best_cost - 1e-9) { best_cost = cost; best = sk; }
+    }
+    static const int sk_env = [] { const char* e = getenv("FT2_GEMM_SPLITK"); return e ? atoi(e) : 0; }();
+    if (sk_env > 0) {
+        best = sk_env < g.nkb ? sk_env : g.nkb;
+        while (best > 1 && tiles * best > capacity) --best;
+    }
+    g.splitk = best;
+    return g;
+}
+
+size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K) {
+    if (M <= 0 || N <= 0 || K <= 0) return 0;
+    GemmPlan g = plan_gemm(M, N, K);
+    if (g.splitk <= 1) return 0;
+    const size_t tiles = (size_t)g.tilesA * g.tilesB;
+    return kCounterBytes + tiles * g.splitk * (size_t)g.bn * kBlockA * 4;
+}
 
 template <int BN, int STAGES>
 static cudaError_t launch_cfg(const GemmArgs& a, GemmK p, cudaStream_t st, int* n_launch) {
@@ -395,22 +605,16 @@ static cudaError_t launch_cfg(const GemmArgs& a, GemmK p, cudaStream_t st, int* 
         cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              L::kBytes);
         if (e != cudaSuccess) return e;
-        e = cudaFuncSetAttribute(gemm_kernel<BN, STAGES>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-        if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    const int tilesA = (p.rowsA + kBlockA - 1) / kBlockA;
-    const int tilesB = (p.rowsB + BN - 1) / BN;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)tilesA, (unsigned)p.splitk, (unsigned)tilesB);
+    cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);
     cfg.blockDim = dim3(kGemmThreads);
     cfg.dynamicSmemBytes = L::kBytes;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 1;
-    attr[0].val.clusterDim.y = (unsigned)p.splitk;
-    attr[0].val.clusterDim.z = 1;
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, STAGES>, ma, mb, p);
@@ -419,14 +623,18 @@ static cudaError_t launch_cfg(const GemmArgs& a, GemmK p, cudaStream_t st, int* 
 }
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
+    GemmPlan g = plan_gemm(a.M, a.N, a.K);
     GemmK p = {};
     p.M = a.M;
     p.N = a.N;
     p.K = a.K;
-    p.swap = a.M <= 128 ? 1 : 0;
-    p.rowsA = p.swap ? a.N : a.M;
-    p.rowsB = p.swap ? a.M : a.N;
-    p.nkb = (a.K + kBlockK - 1) / kBlockK;
+    p.swap = g.swap;
+    p.rowsA = g.swap ? a.N : a.M;
+    p.rowsB = g.swap ? a.M : a.N;
+    p.tilesA = g.tilesA;
+    p.tilesB = g.tilesB;
+    p.splitk = g.splitk;
+    p.nkb = g.nkb;
     p.mode = a.mode;
     p.col_begin = a.col_begin;
     p.col_end = a.col_end;
@@ -443,21 +651,23 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cur_layer = a.cur_layer;
     p.cur_step = a.cur_step;
     p.base_row = a.base_row;
-
-    int bn;
-    if (p.swap) bn = a.M <= 16 ? 16 : (a.M <= 32 ? 32 : (a.M <= 64 ? 64 : 128));
-    else bn = 128;
-    const int tiles = ((p.rowsA + kBlockA - 1) / kBlockA) * ((p.rowsB + bn - 1) / bn);
-    const int sms = num_sms();
-    int sk = 1;
-    while (sk < 8 && tiles * sk * 2 <= sms && p.nkb >= sk * 2 * 2) sk *= 2;
-    p.splitk = sk;
-
-    switch (bn) {
-        case 16: return launch_cfg<16, 8>(a, p, st, n_launch);
-        case 32: return launch_cfg<32, 8>(a, p, st, n_launch);
-        case 64: return launch_cfg<64, 8>(a, p, st, n_launch);
-        default: return launch_cfg<128, 6>(a, p, st, n_launch);
+    p.w_static = a.w_static;
+    if (g.splitk > 1) {
+        uintptr_t base = reinterpret_cast<uintptr_t>(a.ws);
+        p.tile_ctr = reinterpret_cast<uint32_t*>(base);
+        uintptr_t part = base + kCounterBytes;
+        p.partials = reinterpret_cast<float4*>(part);
+    }
+    switch (g.bn) {
+        case 16: return launch_cfg<16, Stages<16>::value>(a, p, st, n_launch);
+        case 32: {
+            static const int st_env = [] { const char* e = getenv("FT2_GEMM_STAGES32"); return e ? atoi(e) : 0; }();
+            if (st_env == 8) return launch_cfg<32, 8>(a, p, st, n_launch);
+            if (st_env == 10) return launch_cfg<32, 10>(a, p, st, n_launch);
+            return launch_cfg<32, Stages<32>::value>(a, p, st, n_launch);
+        }
+        case 64: return launch_cfg<64, Stages<64>::value>(a, p, st, n_launch);
+        default: return launch_cfg<128, Stages<128>::value>(a, p, st, n_launch);
     }
 }
 

@@ -88,12 +88,34 @@ def protect_fused_gemm(x, w, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None, row
         col_end = N
     S = num_seqs if num_seqs is not None else (bounds.numel() // 2 if bounds is not None else 0)
     ns = 0 if sites is None else (n_sites if n_sites is not None else sites.numel() // SITE_BYTES)
-    ws = 0 if workspace is None else workspace.numel() * workspace.element_size()
+    if workspace is None:
+        workspace = default_gemm_workspace(x.device)
+    ws = workspace.numel() * workspace.element_size()
     st = load().ft2_protect_fused_gemm(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y), y.stride(0),
                                        M, N, K, int(mode), col_begin, col_end, _ptr(row_to_seq), _ptr(bounds), S,
                                        _ptr(corrected_count), _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),
                                        _ptr(workspace), ws, _stream(stream))
     check("ft2_protect_fused_gemm", st)
+
+
+_GEMM_WS = {}
+GEMM_WS_BYTES = 16 << 20
+
+
+def default_gemm_workspace(device) -> torch.Tensor:
+    """Per-device zero-filled split-K workspace shared by calls that pass none.
+    Created on first use (call once outside CUDA-graph capture); not safe for
+    GEMMs running concurrently on different streams -- pass your own then."""
+    key = torch.device(device).index if torch.device(device).index is not None else torch.cuda.current_device()
+    ws = _GEMM_WS.get(key)
+    if ws is None:
+        ws = torch.zeros(GEMM_WS_BYTES // 8, dtype=torch.int64, device=torch.device("cuda", key))
+        _GEMM_WS[key] = ws
+    return ws
+
+
+def gemm_workspace_bytes(M, N, K) -> int:
+    return int(load().ft2_gemm_workspace_bytes(M, N, K))
 
 
 def make_fault_sites(seed, trial0, n_trials, model, layer_width, n_steps, prompt_len, out=None,

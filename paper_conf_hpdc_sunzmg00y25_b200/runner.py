@@ -1,0 +1,367 @@
+"""Synthetic decoder-only LLM runner with FT2 protection on its critical layers.
+
+This is the *host model* around FT2's hot path (attention,
+norms, activations, embeddings and sampling run as plain torch ops -- they
+are not part of the method).  The method itself runs in libft2.so:
+
+* critical layers (Table 1): OPT/GPT-J
+  v_proj, out_proj, fc2; Llama/Qwen2 v_proj, o_proj, up_proj, down_proj;
+* prefill (first token): each critical layer's output is reduced to per-
+  sequence bounds x2 and its non-finite values are corrected
+  (ft2_bounds_from_prefill);
+* every decode step: each critical layer's output is checked and clipped
+  (PAPER.md L259-L272), either
+    - "standalone": cuBLAS linear + ft2_protect (the paper's own structure:
+      a fused clamp/nan_to_num op called after the layer, L272), or
+    - "fused": ft2_protect_fused_gemm with the check in the tcgen05 GEMM
+      epilogue (no extra kernel, no extra HBM pass);
+* "off" is the unprotected baseline (cuBLAS linears, no FT2 work), and
+  "fused_plain" runs the same tcgen05 GEMM without the check (isolates the
+  epilogue's cost).
+
+Weights are seeded synthetic (ft2_synth recipe, scaled 2^-ceil(log2 sqrt K));
+no checkpoint is loaded.  Decode steps are captured once into a CUDA graph and
+replayed per token.
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+
+import torch
+import torch.nn.functional as F
+
+import ft2_synth
+
+from . import ft2 as F2
+from ._lib import FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FT2_GEMM_W_STATIC
+
+MODES = ("off", "standalone", "fused", "fused_plain")
+
+
+@dataclasses.dataclass(frozen=True)
+class ModelConfig:
+    arch: str              # "opt" | "llama"
+    hidden: int
+    ffn: int
+    n_layers: int
+    n_heads: int
+    vocab: int
+    max_pos: int = 2048
+    bias: bool = True
+
+    @property
+    def head_dim(self):
+        return self.hidden // self.n_heads
+
+    def linears(self):
+        """Block linear layers in order: (name, out_features, in_features, critical)."""
+        h, f = self.hidden, self.ffn
+        if self.arch == "opt":
+            return [("q_proj", h, h, False), ("k_proj", h, h, False), ("v_proj", h, h, True),
+                    ("out_proj", h, h, True), ("fc1", f, h, False), ("fc2", h, f, True)]
+        return [("q_proj", h, h, False), ("k_proj", h, h, False), ("v_proj", h, h, True),
+                ("o_proj", h, h, True), ("gate_proj", f, h, False), ("up_proj", f, h, True),
+                ("down_proj", h, f, True)]
+
+    def critical_names(self):
+        return [n for n, _, _, c in self.linears() if c]
+
+    def critical_widths(self):
+        """Output width of every protected layer, block-major (the bounds/site layer ids)."""
+        per = [o for _, o, _, c in self.linears() if c]
+        return per * self.n_layers
+
+    def linear_widths(self):
+        per = [o for _, o, _, _ in self.linears()]
+        return per * self.n_layers
+
+
+# Shapes (SURVEY.md §0 external facts: HF config defaults / public model cards).
+CONFIGS = {
+    "opt-125m": ModelConfig("opt", 768, 3072, 12, 12, 50272),
+    "opt-1.3b": ModelConfig("opt", 2048, 8192, 24, 32, 50272),
+    "opt-2.7b": ModelConfig("opt", 2560, 10240, 32, 32, 50272),
+    "opt-6.7b": ModelConfig("opt", 4096, 16384, 32, 32, 50272),
+    "llama-2-7b": ModelConfig("llama", 4096, 11008, 32, 32, 32000, 4096, False),
+    "llama-2-13b": ModelConfig("llama", 5120, 13824, 40, 40, 32000, 4096, False),
+}
+
+
+def _w(shape, tau, seed, device, K=None):
+    sl = ft2_synth.weight_scale_log2(K) if K else 0
+    return ft2_synth.gen_bf16_torch(shape, tau, seed, scale_log2=sl, device=device)
+
+
+class Block:
+    def __init__(self, cfg: ModelConfig, idx: int, seed: int, device):
+        self.cfg = cfg
+        self.idx = idx
+        tau0 = 1000 + 64 * idx
+        self.w = {}
+        self.b = {}
+        for j, (name, o, i, _) in enumerate(cfg.linears()):
+            self.w[name] = _w((o, i), tau0 + 2 * j, seed, device, K=i)
+            self.b[name] = _w((o,), tau0 + 2 * j + 1, seed, device) if cfg.bias else None
+        h = cfg.hidden
+        self.ln1_w = torch.ones(h, dtype=torch.bfloat16, device=device)
+        self.ln2_w = torch.ones(h, dtype=torch.bfloat16, device=device)
+        self.ln1_b = torch.zeros(h, dtype=torch.bfloat16, device=device) if cfg.arch == "opt" else None
+        self.ln2_b = torch.zeros(h, dtype=torch.bfloat16, device=device) if cfg.arch == "opt" else None
+
+
+class FT2State:
+    """Per-request FT2 state: bounds [L_crit, B, 2], counters, workspace."""
+
+    def __init__(self, n_crit: int, B: int, device):
+        self.bounds = torch.zeros((n_crit, B, 2), dtype=torch.bfloat16, device=device)
+        self.keys = torch.zeros((n_crit, B, 2), dtype=torch.int32, device=device)
+        self.corrected = torch.zeros((n_crit, B), dtype=torch.int32, device=device)
+        self.nonfinite = torch.zeros((n_crit, B), dtype=torch.int32, device=device)
+        self.ws = F2.make_workspace(B, device=device)
+
+    def reset_counters(self):
+        self.corrected.zero_()
+        self.nonfinite.zero_()
+
+
+class Runner:
+    """Batched greedy generation with FT2 on the critical layers."""
+
+    def __init__(self, cfg: ModelConfig, batch: int, prompt_len: int, gen_len: int, seed: int = 1,
+                 device="cuda", scale: float = 2.0):
+        self.cfg = cfg
+        self.B = batch
+        self.T = prompt_len
+        self.G = gen_len
+        self.Tmax = prompt_len + gen_len
+        self.scale = scale
+        self.device = torch.device(device)
+        dv = self.device
+        h = cfg.hidden
+        self.embed = _w((cfg.vocab, h), 1, seed, dv)
+        self.pos_embed = _w((cfg.max_pos + 2, h), 2, seed, dv) if cfg.arch == "opt" else None
+        self.blocks = [Block(cfg, i, seed, dv) for i in range(cfg.n_layers)]
+        self.lnf_w = torch.ones(h, dtype=torch.bfloat16, device=dv)
+        self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
+        self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h)
+        self.crit_names = cfg.critical_names()
+        self.n_crit = len(self.crit_names) * cfg.n_layers
+        self.state = FT2State(self.n_crit, batch, dv)
+        H, D = cfg.n_heads, cfg.head_dim
+        self.k_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
+                        for _ in range(cfg.n_layers)]
+        self.v_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
+                        for _ in range(cfg.n_layers)]
+        self.seq_offsets = torch.arange(0, (batch + 1) * prompt_len, prompt_len, dtype=torch.int32, device=dv)
+        # decode-step static buffers (CUDA-graph inputs/outputs)
+        self.tok = torch.zeros(batch, dtype=torch.int64, device=dv)
+        self.pos = torch.zeros(1, dtype=torch.int64, device=dv)
+        self.out_tokens = torch.zeros((batch, gen_len), dtype=torch.int64, device=dv)
+        self.sites = None        # optional fault sites (uint8 [B*24]); site i = sequence i
+        self.cur_step = torch.zeros(1, dtype=torch.int32, device=dv)
+        self.graphs = {}
+        self.time_phases = False
+        self._phase_events = []
+        self.mode = "fused"
+        if cfg.arch == "llama":
+            inv = 1.0 / (10000 ** (torch.arange(0, D, 2, device=dv, dtype=torch.float32) / D))
+            t = torch.arange(self.Tmax, device=dv, dtype=torch.float32)
+            fr = torch.outer(t, inv)
+            self.rope_cos = torch.cat([fr.cos(), fr.cos()], -1).to(torch.bfloat16)
+            self.rope_sin = torch.cat([fr.sin(), fr.sin()], -1).to(torch.bfloat16)
+
+    # ------------------------------------------------------------ helpers
+    def _norm(self, x, w, b):
+        if self.cfg.arch == "opt":
+            return F.layer_norm(x, (x.shape[-1],), w, b, 1e-5)
+        xf = x.float()
+        return (xf * torch.rsqrt(xf.pow(2).mean(-1, keepdim=True) + 1e-6)).to(x.dtype) * w
+
+    def _rope(self, x, pos_idx):
+        cos = self.rope_cos[pos_idx].unsqueeze(1)
+        sin = self.rope_sin[pos_idx].unsqueeze(1)
+        d = x.shape[-1] // 2
+        rot = torch.cat([-x[..., d:], x[..., :d]], -1)
+        return x * cos + rot * sin
+
+    def _crit_id(self, blk, name):
+        return blk * len(self.crit_names) + self.crit_names.index(name)
+
+    def _linear(self, x2, blk: Block, name: str, phase: str, step_for_sites=None):
+        """One linear layer of the block; FT2 work on critical ones.
+
+        phase "prefill": bounds from the first-token output (+ NaN/Inf correction).
+        phase "decode":  check-and-clip according to self.mode.
+        """
+        w, b = blk.w[name], blk.b[name]
+        crit = name in self.crit_names
+        if phase == "prefill":
+            if crit and self.mode != "off":
+                # prefill GEMMs are compute-bound (M = B*T); they run on cuBLAS in
+                # every mode and FT2's first-token work is the bounds sweep below
+                y = F.linear(x2, w, b)
+                cid = self._crit_id(blk.idx, name)
+                st = self.state
+                F2.bounds_from_prefill(y, st.bounds[cid], st.ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
+                                       scale=self.scale, correct_nonfinite=True, nonfinite_count=st.nonfinite[cid])
+                return y
+            return F.linear(x2, w, b)
+        # decode
+        if not crit or self.mode == "off":
+            return F.linear(x2, w, b)
+        cid = self._crit_id(blk.idx, name)
+        st = self.state
+        if self.mode == "standalone":
+            y = F.linear(x2, w, b)
+            F2.protect(y, st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid])
+            return y
+        y = torch.empty((x2.shape[0], w.shape[0]), dtype=torch.bfloat16, device=x2.device)
+        mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
+        F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, bounds=st.bounds[cid], num_seqs=self.B,
+                              corrected_count=st.corrected[cid], sites=self.sites,
+                              cur_layer=cid, cur_step=step_for_sites if step_for_sites is not None else 0)
+        return y
+
+    # ------------------------------------------------------------ forward
+    def _block(self, blk: Block, x, phase, pos_idx=None, step=None):
+        cfg = self.cfg
+        B = self.B
+        H, D = cfg.n_heads, cfg.head_dim
+        T = x.shape[1]
+        h = self._norm(x, blk.ln1_w, blk.ln1_b)
+        h2 = h.reshape(-1, cfg.hidden)
+        q = self._linear(h2, blk, "q_proj", phase, step)
+        k = self._linear(h2, blk, "k_proj", phase, step)
+        v = self._linear(h2, blk, "v_proj", phase, step)
+        q = q.view(B, T, H, D).transpose(1, 2)
+        k = k.view(B, T, H, D).transpose(1, 2)
+        v = v.view(B, T, H, D).transpose(1, 2)
+        if cfg.arch == "llama":
+            q = self._rope(q, pos_idx)
+            k = self._rope(k, pos_idx)
+        kc, vc = self.k_cache[blk.idx], self.v_cache[blk.idx]
+        if phase == "prefill":
+            kc[:, :, :T] = k
+            vc[:, :, :T] = v
+            a = F.scaled_dot_product_attention(q, k, v, is_causal=True)
+        else:
+            kc.index_copy_(2, self.pos, k)
+            vc.index_copy_(2, self.pos, v)
+            s = torch.matmul(q, kc.transpose(2, 3)) * (1.0 / math.sqrt(D))
+            s = s + self._mask
+            a = torch.matmul(torch.softmax(s.float(), -1).to(q.dtype), vc)
+        a = a.transpose(1, 2).reshape(-1, cfg.hidden)
+        o_name = "out_proj" if cfg.arch == "opt" else "o_proj"
+        x = x + self._linear(a, blk, o_name, phase, step).view(B, T, -1)
+        h = self._norm(x, blk.ln2_w, blk.ln2_b).reshape(-1, cfg.hidden)
+        if cfg.arch == "opt":
+            f = torch.relu(self._linear(h, blk, "fc1", phase, step))
+            y = self._linear(f, blk, "fc2", phase, step)
+        else:
+            g = self._linear(h, blk, "gate_proj", phase, step)
+            u = self._linear(h, blk, "up_proj", phase, step)
+            y = self._linear(F.silu(g) * u, blk, "down_proj", phase, step)
+        return x + y.view(B, T, -1)
+
+    def _embed(self, ids, pos_idx):
+        x = self.embed[ids]
+        if self.cfg.arch == "opt":
+            x = x + self.pos_embed[pos_idx + 2]
+        return x
+
+    def _logits_next(self, x_last):
+        h = self._norm(x_last, self.lnf_w, self.lnf_b)
+        return torch.argmax(F.linear(h, self.lm_head).float(), dim=-1)
+
+    def prefill(self, prompt_ids):
+        """First-token generation: FT2 bounds for every critical layer."""
+        B, T = prompt_ids.shape
+        pos = torch.arange(T, device=self.device)
+        x = self._embed(prompt_ids, pos.unsqueeze(0).expand(B, T))
+        pidx = pos.unsqueeze(0).expand(B, T)
+        for blk in self.blocks:
+            x = self._block(blk, x, "prefill", pos_idx=pidx, step=0)
+        nxt = self._logits_next(x[:, -1])
+        return nxt
+
+    def _decode_step(self):
+        """One decode step on static buffers (graph-capturable)."""
+        pidx = self.pos.view(1, 1).expand(self.B, 1)
+        ar = torch.arange(self.Tmax, device=self.device)
+        self._mask = torch.where(ar <= self.pos, 0.0, float("-inf")).to(torch.bfloat16).view(1, 1, 1, -1)
+        x = self._embed(self.tok.view(self.B, 1), pidx)
+        for blk in self.blocks:
+            x = self._block(blk, x, "decode", pos_idx=pidx, step=self._site_step)
+        nxt = self._logits_next(x[:, -1])
+        gi = (self.pos - self.T + 1).clamp_(0, self.G - 1)
+        self.out_tokens.index_copy_(1, gi, nxt.view(self.B, 1))
+        self.tok.copy_(nxt)
+        self.pos.add_(1)
+
+    def _graph(self, mode, step_for_sites):
+        key = (mode, step_for_sites)
+        if key not in self.graphs:
+            self.mode = mode
+            self._site_step = step_for_sites
+            s = torch.cuda.Stream()
+            s.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(s):
+                save = (self.tok.clone(), self.pos.clone(), self.out_tokens.clone())
+                for _ in range(2):   # warm-up (allocations, cuBLAS handles)
+                    self._decode_step()
+                self.tok.copy_(save[0]); self.pos.copy_(save[1]); self.out_tokens.copy_(save[2])
+            torch.cuda.current_stream().wait_stream(s)
+            g = torch.cuda.CUDAGraph()
+            n0 = F2.launch_count()
+            with torch.cuda.graph(g):
+                self._decode_step()
+            self.graphs[key] = (g, F2.launch_count() - n0)
+            self.tok.copy_(save[0]); self.pos.copy_(save[1]); self.out_tokens.copy_(save[2])
+        return self.graphs[key]
+
+    def ft2_launches_per_request(self, mode):
+        """Library kernels launched by one generate() in `mode` (prefill + decode replays)."""
+        if mode == "off":
+            return 0
+        per_prefill = self.n_crit
+        g, per_step = self._graph(mode, None)
+        return per_prefill + per_step * (self.G - 1)
+
+    def generate(self, prompt_ids, mode="fused", use_graph=True):
+        """Greedy generation of G tokens (1 first token + G-1 decode steps)."""
+        self.mode = mode
+        self._site_step = None
+        self.state.reset_counters()
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)] if self.time_phases else None
+        if ev:
+            ev[0].record()
+        first = self.prefill(prompt_ids)
+        self.out_tokens[:, 0] = first
+        self.tok.copy_(first)
+        self.pos.fill_(self.T)
+        if ev:
+            ev[1].record()
+        if use_graph:
+            g, _ = self._graph(mode, None)
+            self.mode = mode
+            for _ in range(self.G - 1):
+                g.replay()
+        else:
+            for _ in range(self.G - 1):
+                self._decode_step()
+        if ev:
+            ev[2].record()
+            self._phase_events.append(ev)
+        return self.out_tokens
+
+    def phase_times(self):
+        """(prefill ms, decode ms per step) averaged over the generate() calls
+        since the last call (requires time_phases = True)."""
+        torch.cuda.synchronize()
+        if not self._phase_events:
+            return None
+        pre = sum(e[0].elapsed_time(e[1]) for e in self._phase_events) / len(self._phase_events)
+        dec = sum(e[1].elapsed_time(e[2]) for e in self._phase_events) / len(self._phase_events) / max(1, self.G - 1)
+        self._phase_events = []
+        return pre, dec

@@ -164,3 +164,15 @@ def test_gemm_protected_column_slice(ft2):
     rc = oracle.protect(sl, bnds)
     ref[:, 512:] = sl
     assert np.array_equal(host(y), ref) and int(cnt.item()) == int(rc[0])
+
+
+def test_gemm_shared_workspace_across_shapes(ft2):
+    """Regression: one workspace serves GEMMs with different tile counts and
+    split factors back to back (counters must not be clobbered by partials)."""
+    shapes = [(1, 768, 768), (32, 256, 4096), (1, 2048, 2048), (32, 2048, 2048), (8, 4096, 1024), (32, 2048, 2048)]
+    for M, N, K in shapes * 2:
+        x, w, b = _operands(M, N, K, seed=M * 3 + N)
+        y, _ = _run(ft2, x, w, b, 0)
+        yr, _ = oracle.linear_f64(x, w, b)
+        nbad, worst = _tol_ok(y, yr)
+        assert nbad == 0, (M, N, K, nbad, worst)
