@@ -16,7 +16,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIBDIR = os.path.join(PKG, "lib")
-LIB = os.path.join(LIBDIR, "libft2.so")
+LIB = os.environ.get("FT2_LIB") or os.path.join(LIBDIR, "libft2.so")
+TRACE_LIB = os.path.join(LIBDIR, "libft2_trace.so")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
@@ -35,25 +36,29 @@ def sources():
 
 
 def needs_build() -> bool:
-    if not os.path.exists(LIB):
+    lib = os.path.join(LIBDIR, "libft2.so")
+    if not os.path.exists(lib):
         return True
-    t = os.path.getmtime(LIB)
+    t = os.path.getmtime(lib)
     deps = sources() + glob.glob(os.path.join(CSRC, "*.cuh")) + glob.glob(os.path.join(CSRC, "*.h")) + \
         [os.path.join(ROOT, "include", "ft2.h")]
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, trace: bool = False) -> str:
+    """Compile every csrc/*.cu for sm_100a and link lib/libft2.so.  trace=True
+    builds lib/libft2_trace.so with per-CTA timestamps in the GEMM (debug)."""
+    out_lib = TRACE_LIB if trace else os.path.join(LIBDIR, "libft2.so")
+    if not force and not trace and not needs_build():
         return LIB
     os.makedirs(LIBDIR, exist_ok=True)
-    objdir = os.path.join(LIBDIR, "obj")
+    objdir = os.path.join(LIBDIR, "obj_trace" if trace else "obj")
     os.makedirs(objdir, exist_ok=True)
     objs = []
     procs = []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
-        cmd = [_nvcc(), *ARCH, *FLAGS, "-c", src, "-o", obj]
+        cmd = [_nvcc(), *ARCH, *FLAGS, *(["-DFT2_GEMM_TRACE"] + (["-DFT2_TRACE_CLOCK"] if os.environ.get("FT2_TRACE_CLOCK") else []) if trace else []), "-c", src, "-o", obj]
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)))
         objs.append(obj)
     for cmd, p in procs:
@@ -62,12 +67,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
             print(out)
         if p.returncode != 0:
             raise RuntimeError("nvcc failed:\n" + " ".join(cmd) + "\n" + out)
-    tmp = LIB + ".tmp"
+    tmp = out_lib + ".tmp"
     cmd = [_nvcc(), *ARCH, "-shared", "-o", tmp, *objs]
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, out_lib)
+    return out_lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, trace="--trace" in sys.argv))

@@ -4,157 +4,74 @@
 //   y[m, j] = check(inject(bf16_rne(sum_k x[m, k] * w[j, k] + bias[j])))
 //
 // PAPER.md L259 ("Protection is applied after the execution of each critical
-// layer"), L272 (clamp + nan_to_num applied right after the layer).  The
-// check operates on the bf16-rounded value after bias (reading A19); a fault
-// site is applied before the check (A20).
+// layer"), L272 (clamp + nan_to_num applied right after the layer).  The check
+// operates on the bf16-rounded value after bias (reading A19); a fault site is
+// applied before the check (A20).
 //
-// Structure (one CTA = one 128 x BN output tile x one K slice):
-//   warp 0      TMA producer: 128B-swizzled K-major tiles of A and B into a
-//               kStages-deep shared-memory ring (mbarrier full/empty).
-//   warp 1      TMEM allocator + single-thread tcgen05.mma.cta_group::1.kind::f16
-//               issuer (BF16 x BF16 -> FP32 in TMEM); tcgen05.commit frees a
-//               stage and finally signals the epilogue.
-//   warps 2-5   epilogue: tcgen05.ld (32x32b) TMEM -> registers -> shared memory.
-// Split-K runs as a thread-block cluster along K (cluster dims (1, splitk, 1)):
-// each CTA's fp32 partial tile is combined through distributed shared memory
-// in fixed rank order (deterministic), each CTA then finishes 128/splitk rows:
-// bias, RNE to bf16, fault XOR, key-space clamp, corrected count, store.  The
-// clip is therefore applied to the complete K reduction (it is non-linear).
+// One CTA = one 128 x BN output tile x one K slice, 192 threads:
+//   warp 0     TMA producer: 128B-swizzled K-major tiles of A and B into a
+//              STAGES-deep shared-memory ring (mbarrier full/empty).  With
+//              programmatic dependent launch the first weight tiles are
+//              requested before waiting for the previous kernel (opt-in).
+//   warp 1     TMEM allocator + single-thread tcgen05.mma.cta_group::1.kind::f16
+//              issuer (BF16 x BF16 -> FP32 in TMEM); tcgen05.commit frees a
+//              stage and finally signals the epilogue.
+//   warps 2-5  tcgen05.ld the accumulator (32x32b, one TMEM lane per thread)
+//              and stage it as fp32 rows in shared memory.
+//   all warps  finish the CTA's rows: bias -> RNE bf16 -> fault XOR ->
+//              key-space check-and-clip (two values per 32-bit word, the same
+//              order-key machinery as ft2_protect) -> store -> count.
+// Split-K is a thread-block cluster (1, splitk, 1): CTA r owns rows
+// [r0(r), r0(r+1)) of the tile; every CTA pushes each accumulator row into the
+// owner's receive slot with st.async over DSMEM (completion counted on the
+// owner's mbarrier): no global workspace, no fences, no spinning.  The owner
+// sums the slots in fixed order 0..splitk-1 (deterministic) and clips only the
+// complete K reduction (clipping is non-linear).
 //
-// Orientation: for decode (M <= 128 tokens) the kernel runs "swap-AB": the
-// UMMA M = 128 dimension walks output features (rows of W) and UMMA N = BN
-// walks tokens, so skinny activations still fill the tensor core; for prefill
-// (M > 128) A = x and B = w.
+// Orientation: decode (M <= 128 tokens) runs "swap-AB": UMMA M = 128 walks
+// output features (rows of W), UMMA N = BN walks tokens, so skinny activations
+// still fill the tensor core; prefill (M > 128) uses A = x, B = w.
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
-#include <stdio.h>
 #include <stdlib.h>
 
 #include <mutex>
 
 #include "ft2_device.cuh"
 #include "ft2_internal.h"
+#include "sm100_ptx.cuh"
 
 namespace ft2impl {
 using namespace ft2dev;
 
-constexpr int kBlockA = 128;   // UMMA M
-constexpr int kBlockK = 64;    // one 128-byte swizzle atom of bf16
+constexpr int kBlockA = 128;  // UMMA M
+constexpr int kBlockK = 64;   // one 128-byte swizzle atom of bf16
 constexpr int kUmmaK = 16;
 constexpr int kGemmThreads = 192;
 constexpr int kMaxSitesPerCta = 64;
-// Split-K tile counters live in a fixed region at the start of the workspace
-// (independent of the shape, so one workspace can serve every GEMM); split-K
-// is only used when tiles * splitk fits one co-resident wave, i.e. tiles <= 2 x SMs.
-constexpr int kMaxSplitTiles = 1024;
-constexpr size_t kCounterBytes = (size_t)kMaxSplitTiles * 8;
+constexpr int kMaxSplitK = 16;  // cluster size along K (non-portable above 8)
 
-// ------------------------------------------------------------------ PTX glue
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-    return (uint32_t)__cvta_generic_to_shared(p);
+#ifdef FT2_GEMM_TRACE
+// Debug builds only (lib/libft2_trace.so): per-CTA timestamps.
+__device__ unsigned long long g_trace[4096 * 16];
+__device__ __forceinline__ void trace(int slot) {
+    unsigned long long t;
+#ifdef FT2_TRACE_CLOCK
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
+#else
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+#endif
+    const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+    if (cta < 4096) g_trace[cta * 16 + slot] = t;
 }
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    uint32_t a = smem_u32(bar);
-    asm volatile(
-        "{\n\t.reg .pred P1;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-        "@!P1 bra WAIT_%=;\n}" ::"r"(a),
-        "r"(parity)
-        : "memory");
-}
-__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
-            smem_u32(dst)),
-        "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
-        : "memory");
-}
-__device__ __forceinline__ void prefetch_tmap(const CUtensorMap* map) {
-    asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
-}
-__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_commit(uint64_t* bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
-                 : "memory");
-}
-__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-        "l"(da), "l"(db), "r"(idesc), "r"(acc)
-        : "memory");
-}
-// 32 lanes x 32 consecutive 32-bit columns -> 32 registers per thread
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
-        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
-          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
-          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-        : "r"(taddr));
-}
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
-        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-        : "r"(taddr));
-}
-__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
-
-__device__ __forceinline__ uint32_t cluster_rank() {
-    uint32_t r;
-    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-    return r;
-}
-__device__ __forceinline__ void cluster_sync_all() {
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
-    uint32_t r;
-    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
-    return r;
-}
-__device__ __forceinline__ float ld_dsmem_f32(uint32_t addr) {
-    float v;
-    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr));
-    return v;
-}
-
-// UMMA shared-memory descriptor: K-major, 128-byte swizzle, 8-row core
-// matrix groups 1024 B apart (SBO), sm100 descriptor version 1.
-__device__ __forceinline__ uint64_t make_sdesc(uint32_t saddr) {
-    uint64_t d = 0;
-    d |= (uint64_t)((saddr >> 4) & 0x3FFF);
-    d |= (uint64_t)(1024 >> 4) << 32;
-    d |= (uint64_t)1 << 46;
-    d |= (uint64_t)2 << 61;
-    return d;
-}
-
-// Instruction descriptor, kind::f16: D fp32, A/B bf16, both K-major.
-__host__ __device__ constexpr uint32_t make_idesc(int m, int n) {
-    return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
-}
+#define FT2_TRACE(slot) trace(slot)
+#else
+#define FT2_TRACE(slot) ((void)0)
+#endif
 
 struct GemmK {
     int32_t M, N, K;
-    int32_t swap;          // 1: A = w (features), B = x (tokens)
     int32_t rowsA, rowsB;  // extent of the A / B operands
     int32_t tilesA, tilesB;
     int32_t splitk, nkb;
@@ -163,193 +80,230 @@ struct GemmK {
     uint16_t* y;
     int64_t ldy;
     const int32_t* row_to_seq;
-    int32_t S, row_mode;
+    int32_t S, row_mode;  // row_mode 0: row_to_seq[], 1: token m -> seq m, 2: all -> seq 0
     const uint16_t* bounds;
     uint32_t* counts;
     const ft2_fault_site* sites;
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
-    float4* partials;      // [tiles][splitk][BN/4][128] float4 (split-K only)
-    uint32_t* tile_ctr;    // [tiles][2] self-resetting arrival / departure counters
-    int32_t w_static;      // weights not written by the preceding kernel: prefetch before the PDL wait
+    int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
 };
 
-template <int BN, int STAGES>
-struct GemmSmem {
-    static constexpr int kABytes = kBlockA * kBlockK * 2;
-    static constexpr int kBBytes = BN * kBlockK * 2;
-    static constexpr int kStageBytes = kABytes + kBBytes;
-    static constexpr int kTileBytes = STAGES * kStageBytes;
-    static constexpr int kBytes = 1024 /*align slack*/ + kTileBytes + 1024 /*barriers, site list*/ + (BN + 128) * 20;
-};
-
-__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
-__device__ __forceinline__ void griddep_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
-__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
-
-// Per-row / per-column epilogue context.  In swap-AB mode rows are output
-// features (bias, protected-slice flag per row) and columns are tokens (bounds
-// per column); otherwise the other way round.  `keys` packs key(lo) | key(hi) << 16;
-// seq < 0 means "do not check".
-struct EpiSide {
+// Per-row / per-column epilogue table entry.  Feature side: bias, flags
+// bit0 = in range, bit1 = protected column (CHECK and inside [col_begin,
+// col_end)).  Token side: keys = key(lo) | key(hi) << 16, seq, flags bit0 =
+// in range, bit1 = has bounds (CHECK and a valid sequence).
+struct TabE {
     float bias;
     uint32_t keys;
     int32_t seq;
-    int32_t valid;  // index inside [0, M) / [0, N)
+    uint32_t flags;
 };
 
-__device__ __forceinline__ EpiSide make_side(const GemmK& p, bool is_token, int idx) {
-    EpiSide e{0.f, 0u, -1, 0};
-    if (is_token) {
-        e.valid = idx < p.M;
-        if (e.valid && p.mode == FT2_GEMM_CHECK) {
-            const int s = p.row_mode == 2 ? 0 : (p.row_mode == 1 ? idx : p.row_to_seq[idx]);
+__device__ __forceinline__ TabE feature_entry(const GemmK& p, int n) {
+    TabE e{0.f, 0u, -1, 0u};
+    if (n < p.N) {
+        e.flags = 1u;
+        if (p.bias) e.bias = __uint_as_float((uint32_t)p.bias[n] << 16);
+        if (p.mode == FT2_GEMM_CHECK && n >= p.col_begin && n < p.col_end) e.flags |= 2u;
+    }
+    return e;
+}
+__device__ __forceinline__ TabE token_entry(const GemmK& p, int m) {
+    TabE e{0.f, 0u, -1, 0u};
+    if (m < p.M) {
+        e.flags = 1u;
+        if (p.mode == FT2_GEMM_CHECK) {
+            const int s = p.row_mode == 2 ? 0 : (p.row_mode == 1 ? m : p.row_to_seq[m]);
             if (s >= 0 && s < p.S) {
-                const uint32_t lh = (uint32_t)p.bounds[2 * s] | ((uint32_t)p.bounds[2 * s + 1] << 16);
-                e.keys = key2(lh);
+                e.keys = key2((uint32_t)p.bounds[2 * s] | ((uint32_t)p.bounds[2 * s + 1] << 16));
                 e.seq = s;
+                e.flags |= 2u;
             }
-        }
-    } else {
-        e.valid = idx < p.N;
-        if (e.valid) {
-            if (p.bias) e.bias = __uint_as_float((uint32_t)p.bias[idx] << 16);
-            e.seq = (p.mode == FT2_GEMM_CHECK && idx >= p.col_begin && idx < p.col_end) ? 0 : -1;  // flag only
         }
     }
     return e;
 }
 
-// Four consecutive columns c..c+3 of one row: all four values are computed
-// before any side effect (stores, counter atomics), so the chains overlap.
-__device__ __forceinline__ void finish4(const GemmK& p, int ga, int gb0, const EpiSide& rs, const EpiSide* cs,
-                                        int la_c0, const float (&acc)[4], const uint32_t* site_e,
-                                        const uint32_t* site_m, uint32_t nsite, uint32_t* row_cnt,
-                                        uint32_t* col_cnt) {
-    uint16_t o[4];
-    bool ok[4];
-    uint32_t changed = 0;
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const EpiSide& feat = p.swap ? rs : cs[j];
-        const EpiSide& tok = p.swap ? cs[j] : rs;
-        ok[j] = feat.valid && tok.valid;
-        uint16_t x = bf16_rne(acc[j] + feat.bias);
-        for (uint32_t i = 0; i < nsite; ++i)
-            if (site_e[i] == (uint32_t)(la_c0 + j)) x ^= (uint16_t)site_m[i];
-        const bool chk = feat.seq >= 0 && tok.seq >= 0;
-        const uint16_t z = ((x & 0x7FFF) > 0x7F80) ? (uint16_t)0 : x;  // NaN -> +0
-        const uint16_t k = key1(z);
-        const uint16_t kl = (uint16_t)tok.keys, kh = (uint16_t)(tok.keys >> 16);
-        const uint16_t c = k < kl ? unkey1(kl) : (k > kh ? unkey1(kh) : z);
-        o[j] = chk ? c : x;
-        changed |= (ok[j] && o[j] != x) ? (1u << j) : 0u;
+template <int BN>
+struct Cfg {
+    static constexpr int STAGES = BN <= 16 ? 5 : (BN <= 32 ? 4 : (BN <= 64 ? 3 : 4));
+    static constexpr int kABytes = kBlockA * kBlockK * 2;
+    static constexpr int kBBytes = BN * kBlockK * 2;
+    static constexpr int kStageBytes = kABytes + kBBytes;
+    static constexpr int kTileBytes = STAGES * kStageBytes;
+    // fp32 tile staging / split-K receive buffer: splitk slots x ceil(128/splitk)
+    // rows (<= 143 in total) x (BN + 4) fp32; the pad keeps float4 row reads
+    // bank-conflict free
+    static constexpr int kRecvStride = BN + 4;
+    static constexpr int kRecvBytes = 144 * kRecvStride * 4;
+    static constexpr int kMiscBytes = 1024;  // mbarriers, TMEM base, site list
+    static constexpr int kTabBytes = (kBlockA + BN) * (int)sizeof(TabE) + (kBlockA + BN) * 4;
+    static constexpr int kBytes = 1024 /*align slack*/ + kTileBytes + kRecvBytes + kMiscBytes + kTabBytes;
+    static constexpr uint32_t kTmemCols = BN < 32 ? 32 : BN;
+};
+
+// XOR the fault masks of the sites that hit elements le0..le0+3 (rare: only
+// fault-injection runs have sites).  Out of line to keep the epilogue small.
+__device__ __noinline__ uint2 xor_sites(uint2 w, uint32_t le0, const uint32_t* site_e, const uint32_t* site_m,
+                                        uint32_t nsite) {
+    for (uint32_t i = 0; i < nsite; ++i) {
+        const uint32_t d = site_e[i] - le0;
+        if (d < 4u) {
+            const uint32_t m = site_m[i] & 0xFFFFu;
+            if (d == 0) w.x ^= m;
+            else if (d == 1) w.x ^= m << 16;
+            else if (d == 2) w.y ^= m;
+            else w.y ^= m << 16;
+        }
     }
-    if (p.swap) {
+    return w;
+}
+
+// Check-and-clip of two packed bf16 (R5): NaN -> key(+0), clamp in key space.
+__device__ __forceinline__ uint32_t clip2_nocount(uint32_t w, uint32_t kL2, uint32_t kH2) {
+    const uint32_t k = key2(w);
+    const uint32_t nm = half_sign_mask(nan_bits2(w));
+    const uint32_t kz = (k & ~nm) | (0x80008000u & nm);
+    return unkey2(vmax_u16x2(vmin_u16x2(kz, kH2), kL2));
+}
+
+// Finish four consecutive columns c0..c0+3 of tile row la.
+template <bool SWAP>
+__device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, int ga, int gb0, const TabE& re,
+                                        const TabE* __restrict__ ce, uint32_t le0, float4 acc,
+                                        const uint32_t* site_e, const uint32_t* site_m, uint32_t nsite,
+                                        uint32_t* row_cnt, uint32_t* col_cnt) {
+    // feature side: SWAP ? the row : the column; token side: the other one
+    const float b0 = SWAP ? re.bias : ce[0].bias, b1 = SWAP ? re.bias : ce[1].bias;
+    const float b2 = SWAP ? re.bias : ce[2].bias, b3 = SWAP ? re.bias : ce[3].bias;
+    uint2 w = make_uint2((uint32_t)bf16_rne(acc.x + b0) | ((uint32_t)bf16_rne(acc.y + b1) << 16),
+                         (uint32_t)bf16_rne(acc.z + b2) | ((uint32_t)bf16_rne(acc.w + b3) << 16));
+    if (nsite) w = xor_sites(w, le0, site_e, site_m, nsite);
+    uint32_t f[4], kL01, kH01, kL23, kH23;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) f[j] = re.flags & ce[j].flags;  // bit0 valid, bit1 checked
+    if (SWAP) {
+        kL01 = (ce[0].keys & 0xFFFFu) | (ce[1].keys << 16);
+        kH01 = (ce[0].keys >> 16) | (ce[1].keys & 0xFFFF0000u);
+        kL23 = (ce[2].keys & 0xFFFFu) | (ce[3].keys << 16);
+        kH23 = (ce[2].keys >> 16) | (ce[3].keys & 0xFFFF0000u);
+    } else {
+        kL01 = kL23 = (re.keys & 0xFFFFu) * 0x10001u;
+        kH01 = kH23 = (re.keys >> 16) * 0x10001u;
+    }
+    const uint32_t m01 = ((f[0] & 2u) ? 0x0000FFFFu : 0u) | ((f[1] & 2u) ? 0xFFFF0000u : 0u);
+    const uint32_t m23 = ((f[2] & 2u) ? 0x0000FFFFu : 0u) | ((f[3] & 2u) ? 0xFFFF0000u : 0u);
+    const uint32_t o01 = (clip2_nocount(w.x, kL01, kH01) & m01) | (w.x & ~m01);
+    const uint32_t o23 = (clip2_nocount(w.y, kL23, kH23) & m23) | (w.y & ~m23);
+    const uint32_t d01 = o01 ^ w.x, d23 = o23 ^ w.y;
+    const uint16_t o[4] = {(uint16_t)o01, (uint16_t)(o01 >> 16), (uint16_t)o23, (uint16_t)(o23 >> 16)};
+    if (SWAP) {
+        uint16_t* dst = y + (int64_t)gb0 * ldy + ga;
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-            if (ok[j]) p.y[(int64_t)(gb0 + j) * p.ldy + ga] = o[j];
+            if (f[j] & 1u) dst[(int64_t)j * ldy] = o[j];
     } else {
-        uint16_t* dst = p.y + (int64_t)ga * p.ldy + gb0;
-        if (ok[0] && ok[3] && ((reinterpret_cast<uintptr_t>(dst) & 7u) == 0)) {
-            *reinterpret_cast<uint2*>(dst) = make_uint2((uint32_t)o[0] | ((uint32_t)o[1] << 16),
-                                                        (uint32_t)o[2] | ((uint32_t)o[3] << 16));
+        uint16_t* dst = y + (int64_t)ga * ldy + gb0;
+        if ((f[0] & f[1] & f[2] & f[3] & 1u) && ((reinterpret_cast<uintptr_t>(dst) & 7u) == 0)) {
+            *reinterpret_cast<uint2*>(dst) = make_uint2(o01, o23);
         } else {
 #pragma unroll
             for (int j = 0; j < 4; ++j)
-                if (ok[j]) dst[j] = o[j];
+                if (f[j] & 1u) dst[j] = o[j];
         }
     }
-    if (changed) {  // corrected neurons, aggregated per CTA in shared memory
-        if (p.swap) {
+    if (d01 | d23) {  // corrected neurons, aggregated per CTA in shared memory
+        const uint32_t ch[4] = {d01 & 0xFFFFu, d01 >> 16, d23 & 0xFFFFu, d23 >> 16};
 #pragma unroll
-            for (int j = 0; j < 4; ++j)
-                if (changed & (1u << j)) atomicAdd_block(&col_cnt[j], 1u);
-        } else {
-            atomicAdd_block(row_cnt, (uint32_t)__popc(changed));
-        }
+        for (int j = 0; j < 4; ++j)
+            if (ch[j] && (f[j] & 1u)) atomicAdd_block(SWAP ? &col_cnt[j] : row_cnt, 1u);
     }
 }
 
-template <int BN, int STAGES>
+template <int BN, bool SWAP>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
                 const __grid_constant__ GemmK p) {
-    using L = GemmSmem<BN, STAGES>;
+    using C = Cfg<BN>;
+    constexpr int STAGES = C::STAGES;
     extern __shared__ uint8_t smem_raw[];
-    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+    // 1024-byte alignment (128B swizzle) by offset arithmetic on the shared
+    // array, so the compiler keeps the shared address space (LDS/STS)
+    uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     uint8_t* tiles = smem;
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + L::kTileBytes);
+    float* recv = reinterpret_cast<float*>(smem + C::kTileBytes);
+    uint8_t* misc = smem + C::kTileBytes + C::kRecvBytes;
+    uint64_t* full = reinterpret_cast<uint64_t*>(misc);
     uint64_t* empty = full + STAGES;
     uint64_t* tmem_full = empty + STAGES;
-    uint32_t* tmem_base_sh = reinterpret_cast<uint32_t*>(tmem_full + 1);
-    uint32_t* flag_sh = tmem_base_sh + 1;
-    uint32_t* site_n = flag_sh + 1;
-    uint32_t* site_e = site_n + 1;                 // [kMaxSitesPerCta] local element index (a * BN + c)
-    uint32_t* site_m = site_e + kMaxSitesPerCta;   // [kMaxSitesPerCta] xor mask
-    EpiSide* col_side = reinterpret_cast<EpiSide*>(site_m + kMaxSitesPerCta);  // [BN] per-column context
-    EpiSide* row_side = col_side + BN;                                        // [128] per-row context
-    uint32_t* col_cnt = reinterpret_cast<uint32_t*>(row_side + 128);          // [BN] corrected per column
-    uint32_t* row_cnt = col_cnt + BN;                                         // [128] corrected per row
+    uint64_t* recv_bar = tmem_full + 1;
+    uint32_t* tmem_base_sh = reinterpret_cast<uint32_t*>(recv_bar + 1);
+    uint32_t* site_n = tmem_base_sh + 1;
+    uint32_t* site_e = site_n + 1;                // [kMaxSitesPerCta] local element a * BN + b
+    uint32_t* site_m = site_e + kMaxSitesPerCta;  // [kMaxSitesPerCta] xor mask
+    TabE* row_tab = reinterpret_cast<TabE*>(misc + C::kMiscBytes);  // [128]
+    TabE* col_tab = row_tab + kBlockA;                                // [BN]
+    uint32_t* row_cnt = reinterpret_cast<uint32_t*>(col_tab + BN);    // [128]
+    uint32_t* col_cnt = row_cnt + kBlockA;                            // [BN]
 
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int tileA = blockIdx.x, split = blockIdx.y, tileB = blockIdx.z;
-    const int kb0 = (int)((int64_t)split * p.nkb / p.splitk);
-    const int kb1 = (int)((int64_t)(split + 1) * p.nkb / p.splitk);
+    const int splitk = p.splitk;
+    const int kb0 = (int)((int64_t)split * p.nkb / splitk);
+    const int kb1 = (int)((int64_t)(split + 1) * p.nkb / splitk);
     const int nk = kb1 - kb0;
-    constexpr uint32_t kTmemCols = BN < 32 ? 32 : BN;
+    // rows of the tile this CTA finishes: all of them, or its split-K slice
+    const int r0 = (split * kBlockA) / splitk, r1 = ((split + 1) * kBlockA) / splitk;
 
     if (warp == 0 && lane == 0) {
+        FT2_TRACE(0);
         prefetch_tmap(&map_a);
         prefetch_tmap(&map_b);
         for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
         mbar_init(tmem_full, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        mbar_init(recv_bar, 1);
+        if (splitk > 1)  // bytes the other splits will push into my slice
+            mbar_expect_tx(recv_bar, (uint32_t)((splitk - 1) * (r1 - r0) * BN * 4));
+        fence_mbar_init();
         *site_n = 0;
     }
-    if (warp == 1) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_base_sh)),
-                     "r"(kTmemCols));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
+    if (warp == 1) tmem_alloc(tmem_base_sh, C::kTmemCols);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
+    // peers may push into my receive buffer once my barrier is initialised
+    if (splitk > 1) cluster_arrive_relaxed();
     const uint32_t tmem_base = *tmem_base_sh;
-    // the next kernel in the stream may start its own prologue now (PDL)
-    griddep_launch();
+    griddep_launch();  // the next kernel in the stream may start its prologue (PDL)
 
     if (warp == 0) {
         if (lane == 0) {
             // ------------------------------------------------ TMA producer
-            // The weight operand does not depend on the previous kernel: the
-            // first STAGES weight tiles are requested before waiting for it
-            // (programmatic dependent launch), the activations after.
-            const CUtensorMap* mw = p.swap ? &map_a : &map_b;
-            const CUtensorMap* mx = p.swap ? &map_b : &map_a;
-            const int w_row = p.swap ? tileA * kBlockA : tileB * BN;
-            const int x_row = p.swap ? tileB * BN : tileA * kBlockA;
-            const int w_off = p.swap ? 0 : L::kABytes;
-            const int x_off = p.swap ? L::kABytes : 0;
+            const CUtensorMap* mw = SWAP ? &map_a : &map_b;
+            const CUtensorMap* mx = SWAP ? &map_b : &map_a;
+            const int w_row = SWAP ? tileA * kBlockA : tileB * BN;
+            const int x_row = SWAP ? tileB * BN : tileA * kBlockA;
+            const int w_off = SWAP ? 0 : C::kABytes;
+            const int x_off = SWAP ? C::kABytes : 0;
+            FT2_TRACE(1);
             const int pre = nk < STAGES ? nk : STAGES;
             if (!p.w_static) griddep_wait();
             for (int i = 0; i < pre; ++i) {
-                uint8_t* st = tiles + i * L::kStageBytes;
-                mbar_expect_tx(&full[i], L::kStageBytes);
-                tma_load_2d(mw, &full[i], st + w_off, (kb0 + i) * kBlockK, w_row);
+                mbar_expect_tx(&full[i], C::kStageBytes);
+                tma_load_2d(mw, &full[i], tiles + i * C::kStageBytes + w_off, (kb0 + i) * kBlockK, w_row);
             }
             if (p.w_static) griddep_wait();
+            FT2_TRACE(2);
             for (int i = 0; i < pre; ++i)
-                tma_load_2d(mx, &full[i], tiles + i * L::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row);
+                tma_load_2d(mx, &full[i], tiles + i * C::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row);
             for (int i = STAGES; i < nk; ++i) {
                 const int s = i % STAGES;
-                const uint32_t ph = (uint32_t)(i / STAGES) & 1u;
-                mbar_wait(&empty[s], ph ^ 1u);
-                uint8_t* st = tiles + s * L::kStageBytes;
-                mbar_expect_tx(&full[s], L::kStageBytes);
-                const int kc = (kb0 + i) * kBlockK;
-                tma_load_2d(mw, &full[s], st + w_off, kc, w_row);
-                tma_load_2d(mx, &full[s], st + x_off, kc, x_row);
+                mbar_wait(&empty[s], ((uint32_t)(i / STAGES) & 1u) ^ 1u);
+                uint8_t* st = tiles + s * C::kStageBytes;
+                mbar_expect_tx(&full[s], C::kStageBytes);
+                tma_load_2d(mw, &full[s], st + w_off, (kb0 + i) * kBlockK, w_row);
+                tma_load_2d(mx, &full[s], st + x_off, (kb0 + i) * kBlockK, x_row);
             }
         }
     } else if (warp == 1) {
@@ -358,12 +312,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             constexpr uint32_t idesc = make_idesc(kBlockA, BN);
             for (int i = 0; i < nk; ++i) {
                 const int s = i % STAGES;
-                const uint32_t ph = (uint32_t)(i / STAGES) & 1u;
-                mbar_wait(&full[s], ph);
+                mbar_wait(&full[s], (uint32_t)(i / STAGES) & 1u);
+                if (i == 0) FT2_TRACE(3);
                 tc_fence_after();
-                const uint32_t sa = smem_u32(tiles + s * L::kStageBytes);
-                const uint32_t sb = sa + L::kABytes;
-                const uint64_t da = make_sdesc(sa), db = make_sdesc(sb);
+                const uint32_t sa = smem_u32(tiles + s * C::kStageBytes);
+                const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + C::kABytes);
 #pragma unroll
                 for (int k = 0; k < kBlockK / kUmmaK; ++k)  // 16 elements = 32 B along K per MMA
                     tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc,
@@ -371,40 +324,32 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 tc_commit(&empty[s]);
             }
             tc_commit(tmem_full);
+            FT2_TRACE(4);
         }
     } else {
         // ---------------------------------------------------- epilogue warps
-        const int q = warp & 3;               // TMEM lane quarter this warp may access
-        const int a = q * 32 + lane;          // row of the A tile owned by this thread
-        const int et = a;                     // epilogue thread index 0..127
-        const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
-        const int ga = tileA * kBlockA + a;
-        const int tile = tileB * p.tilesA + tileA;
-        griddep_wait();                       // bias/bounds/y/workspace may belong to the previous kernel
-        // rows of the 128-row A tile this CTA finishes: all of them without
-        // split-K, else the split's 1/splitk slice (distributed reduction)
-        const int r0 = (split * kBlockA) / p.splitk, r1 = ((split + 1) * kBlockA) / p.splitk;
-        // epilogue contexts (bias, bound keys) are gathered while the main loop
-        // still runs: columns are tokens in swap-AB mode, features otherwise
-        for (int c = et; c < BN; c += 128) {
-            col_side[c] = make_side(p, p.swap != 0, tileB * BN + c);
+        const int q = warp & 3;  // TMEM lane quarter this warp may access
+        const int a = q * 32 + lane;
+        griddep_wait();  // bias/bounds/sites/y may belong to the previous kernel
+        // epilogue tables, gathered while the main loop still streams
+        row_tab[a] = SWAP ? feature_entry(p, tileA * kBlockA + a) : token_entry(p, tileA * kBlockA + a);
+        row_cnt[a] = 0u;
+        for (int c = a; c < BN; c += 128) {
+            col_tab[c] = SWAP ? token_entry(p, tileB * BN + c) : feature_entry(p, tileB * BN + c);
             col_cnt[c] = 0u;
         }
-        row_side[et] = make_side(p, p.swap == 0, ga);
-        row_cnt[et] = 0u;
-        // fault sites that land in this CTA's output slice
-        if (p.sites != nullptr) {
-            for (int i = et; i < p.n_sites; i += 128) {
-                ft2_fault_site st = p.sites[i];
+        if (p.sites != nullptr) {  // fault sites landing in my slice
+            for (int i = a; i < p.n_sites; i += 128) {
+                const ft2_fault_site st = p.sites[i];
                 if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
-                int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
-                            (p.cur_step == 0 ? (int64_t)st.token : 0);
-                int64_t n = st.col;
+                const int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
+                                  (p.cur_step == 0 ? (int64_t)st.token : 0);
+                const int64_t n = st.col;
                 if (m < 0 || m >= p.M || n >= p.N) continue;
-                int64_t la = (p.swap ? n : m) - (int64_t)tileA * kBlockA;
-                int64_t lb = (p.swap ? m : n) - (int64_t)tileB * BN;
+                const int64_t la = (SWAP ? n : m) - (int64_t)tileA * kBlockA;
+                const int64_t lb = (SWAP ? m : n) - (int64_t)tileB * BN;
                 if (la < r0 || la >= r1 || lb < 0 || lb >= BN) continue;
-                uint32_t idx = atomicAdd(site_n, 1u);
+                const uint32_t idx = atomicAdd(site_n, 1u);
                 if (idx < (uint32_t)kMaxSitesPerCta) {
                     site_e[idx] = (uint32_t)(la * BN + lb);
                     site_m[idx] = st.xor_mask;
@@ -412,101 +357,79 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             }
         }
         mbar_wait(tmem_full, 0);
+        if (a == 0) FT2_TRACE(5);
         tc_fence_after();
-        if (p.splitk == 1) {
-            epi_bar();
-            const EpiSide rs = row_side[et];
-            const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
+        // Stage accumulator row a as fp32 in the receive slot of its owner
+        // (this CTA without split-K; a cluster peer with it).
+        const int RS = (kBlockA + splitk - 1) / splitk;  // rows per receive slot
+        int owner = 0;
+        while (owner + 1 < splitk && a >= ((owner + 1) * kBlockA) / splitk) ++owner;
+        const uint32_t slot_off =
+            (uint32_t)(((split * RS + (a - (owner * kBlockA) / splitk)) * C::kRecvStride) * 4);
+        if (splitk > 1) cluster_wait();  // every peer's receive barrier is initialised
+        const bool local = owner == split;
+        const uint32_t dst = local ? smem_u32(recv) + slot_off : mapa(smem_u32(recv) + slot_off, (uint32_t)owner);
+        const uint32_t dbar = local ? 0u : mapa(smem_u32(recv_bar), (uint32_t)owner);
+        const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
-            for (int c0 = 0; c0 < BN; c0 += 16) {
-                uint32_t r[16];
-                tmem_ld16(taddr + c0, r);
-                tmem_wait_ld();
+        for (int c0 = 0; c0 < BN; c0 += 16) {
+            uint32_t r[16];
+            tmem_ld16(taddr + c0, r);
+            tmem_wait_ld();
+            if (nk == 0) {
 #pragma unroll
-                for (int j = 0; j < 16; j += 4) {
-                    const float acc[4] = {nk > 0 ? __uint_as_float(r[j]) : 0.f, nk > 0 ? __uint_as_float(r[j + 1]) : 0.f,
-                                          nk > 0 ? __uint_as_float(r[j + 2]) : 0.f, nk > 0 ? __uint_as_float(r[j + 3]) : 0.f};
-                    finish4(p, ga, tileB * BN + c0 + j, rs, col_side + c0 + j, a * BN + c0 + j, acc, site_e, site_m,
-                            nsite, row_cnt + et, col_cnt + c0 + j);
-                }
+                for (int j = 0; j < 16; ++j) r[j] = 0u;
             }
-        } else {
-            // 1. publish this split's fp32 partial tile (coalesced float4 columns)
-            float4* tbase = p.partials + (size_t)tile * p.splitk * (BN / 4) * kBlockA;
-            float4* mine = tbase + (size_t)split * (BN / 4) * kBlockA;
-#pragma unroll 1
-            for (int c0 = 0; c0 < BN; c0 += 16) {
-                uint32_t r[16];
-                tmem_ld16(taddr + c0, r);
-                tmem_wait_ld();
 #pragma unroll
-                for (int j = 0; j < 16; j += 4)
-                    __stcg(&mine[((c0 + j) / 4) * kBlockA + a],
-                           make_float4(__uint_as_float(r[j]), __uint_as_float(r[j + 1]), __uint_as_float(r[j + 2]),
-                                       __uint_as_float(r[j + 3])));
-            }
-            epi_bar();
-            // 2. wait until every split of this tile has published.  All split
-            // CTAs are co-resident: the grid never exceeds one wave (<= 1 CTA
-            // per SM), and PDL dependents launch only after all CTAs started.
-            uint32_t* arrive = p.tile_ctr + 2 * tile;
-            uint32_t* depart = arrive + 1;
-            if (et == 0) {
-                // release: the barrier above orders every epilogue thread's partial stores before it
-                asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(arrive) : "memory");
-                uint32_t seen, ns = 32;
-                while (true) {
-                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(seen) : "l"(arrive) : "memory");
-                    if (seen >= (uint32_t)p.splitk) break;
-                    __nanosleep(ns);
-                    if (ns < 256) ns <<= 1;
-                }
-            }
-            epi_bar();  // thread 0's acquire is ordered before everyone's partial loads
-            const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
-            // 3. reduce my row slice over all splits in fixed order 0..splitk-1
-            const int nrow = r1 - r0;
-            const int nvec = nrow * (BN / 4);
-            for (int v = et; v < nvec; v += 128) {
-                const int la = r0 + v % nrow, c4 = v / nrow;
-                float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-                float4 part[16];
-#pragma unroll
-                for (int rr = 0; rr < 16; ++rr)
-                    if (rr < p.splitk) part[rr] = __ldcg(&tbase[((size_t)rr * (BN / 4) + c4) * kBlockA + la]);
-#pragma unroll
-                for (int rr = 0; rr < 16; ++rr)
-                    if (rr < p.splitk) {
-                        acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w;
-                    }
-                const int gla = tileA * kBlockA + la;
-                const EpiSide rs = row_side[la];
-                const float av[4] = {acc.x, acc.y, acc.z, acc.w};
-                finish4(p, gla, tileB * BN + c4 * 4, rs, col_side + c4 * 4, la * BN + c4 * 4, av, site_e, site_m,
-                        nsite, row_cnt + la, col_cnt + c4 * 4);
-            }
-            // 4. the last CTA to leave resets the counters for the next launch
-            epi_bar();
-            if (et == 0) {
-                if (atomicAdd(depart, 1u) == (uint32_t)p.splitk - 1) {
-                    *arrive = 0u;
-                    *depart = 0u;
-                }
+            for (int j = 0; j < 16; j += 4) {
+                if (local) st_shared_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
+                else st_async_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
             }
         }
     }
-    if (warp >= 2 && p.counts != nullptr && p.mode == FT2_GEMM_CHECK) {
-        epi_bar();  // every finish4 of this CTA has counted
-        const int et = (warp & 3) * 32 + lane;
-        for (int c = et; c < BN; c += 128)
-            if (col_cnt[c] != 0u && col_side[c].seq >= 0 && p.swap) atomicAdd(&p.counts[col_side[c].seq], col_cnt[c]);
-        if (!p.swap && row_cnt[et] != 0u && row_side[et].seq >= 0) atomicAdd(&p.counts[row_side[et].seq], row_cnt[et]);
+    // ---------------------------------------------- finish the slice (all warps)
+    named_bar(2, kGemmThreads);  // tables, site list and my own rows are in shared memory
+    griddep_wait();              // (no-op for threads that already waited)
+    if (splitk > 1) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
+    if (tid == 64) FT2_TRACE(6);
+    {
+        const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
+        const int RS = (kBlockA + splitk - 1) / splitk;
+        const int nrow = r1 - r0;
+        const int nvec = nrow * (BN / 4);
+        const uint32_t inv = (uint32_t)((1u << 20) + nrow - 1) / (uint32_t)nrow;  // v / nrow == (v * inv) >> 20
+        uint16_t* const y = p.y;
+        const int64_t ldy = p.ldy;
+#pragma unroll 1
+        for (int v = tid; v < nvec; v += kGemmThreads) {
+            // item v -> (row lr, column quad c4); consecutive threads take
+            // consecutive rows (coalesced stores in swap-AB mode)
+            const int c4 = (int)(((uint32_t)v * inv) >> 20), lr = v - c4 * nrow, la = r0 + lr;
+            const float* src = recv + lr * C::kRecvStride + c4 * 4;
+            float4 part[kMaxSplitK];
+#pragma unroll
+            for (int rr = 0; rr < kMaxSplitK; ++rr)
+                if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
+            float4 acc = part[0];
+#pragma unroll
+            for (int rr = 1; rr < kMaxSplitK; ++rr)
+                if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
+            finish4<SWAP>(y, ldy, tileA * kBlockA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
+                          (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4);
+        }
+    }
+    if (tid == 64) FT2_TRACE(7);
+    if (p.counts != nullptr && p.mode == FT2_GEMM_CHECK) {
+        named_bar(2, kGemmThreads);  // every finish4 of this CTA has counted
+        if (!SWAP && tid < kBlockA && row_cnt[tid] != 0u) atomicAdd(&p.counts[row_tab[tid].seq], row_cnt[tid]);
+        for (int c = tid; SWAP && c < BN; c += kGemmThreads)
+            if (col_cnt[c] != 0u) atomicAdd(&p.counts[col_tab[c].seq], col_cnt[c]);
     }
     tc_fence_before();
     __syncthreads();
     if (warp == 1) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(kTmemCols));
+        tmem_dealloc(tmem_base, C::kTmemCols);
     }
 }
 
@@ -537,19 +460,57 @@ static bool make_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, 
     return r == CUDA_SUCCESS;
 }
 
-// Tiling plan shared by the workspace query and the launch.
+template <int BN, bool SWAP>
+static cudaError_t set_attrs() {
+    static cudaError_t res = [] {
+        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg<BN>::kBytes);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        return e;
+    }();
+    return res;
+}
+
+// How many (1, sk, 1) clusters of this instantiation can be resident at once.
+template <int BN, bool SWAP>
+static int max_clusters(int sk) {
+    static int cache[kMaxSplitK + 1] = {0};
+    if (sk < 1 || sk > kMaxSplitK) return -1;
+    if (cache[sk] != 0) return cache[sk];
+    if (set_attrs<BN, SWAP>() != cudaSuccess) return cache[sk] = -1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(1, (unsigned)sk, 1);
+    cfg.blockDim = dim3(kGemmThreads);
+    cfg.dynamicSmemBytes = Cfg<BN>::kBytes;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 1;
+    attr[0].val.clusterDim.y = (unsigned)sk;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int n = 0;
+    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BN, SWAP>, &cfg) != cudaSuccess) {
+        cudaGetLastError();
+        n = -1;
+    }
+    return cache[sk] = (n > 0 ? n : -1);
+}
+
+static int max_clusters_bn(int bn, int sk) {
+    switch (bn) {
+        case 16: return max_clusters<16, true>(sk);
+        case 32: return max_clusters<32, true>(sk);
+        case 64: return max_clusters<64, true>(sk);
+        default: return max_clusters<128, true>(sk);
+    }
+}
+
+// Tiling plan: orientation, tile width, split-K factor.
 struct GemmPlan {
     int swap, bn, tilesA, tilesB, splitk, nkb;
 };
-
-// Pipeline depth per BN: BN <= 64 keeps a CTA at <= ~110 KB of shared memory so
-// two CTAs fit on an SM (split-K CTAs of one tile must be co-resident).
-template <int BN> struct Stages { static constexpr int value = BN <= 16 ? 6 : (BN <= 32 ? 5 : (BN <= 64 ? 4 : 6)); };
-static int ctas_per_sm(int bn) {
-    static const int deep32 = [] { const char* e = getenv("FT2_GEMM_STAGES32"); return e ? atoi(e) : 0; }();
-    if (bn == 32 && deep32 >= 8) return 1;
-    return bn <= 64 ? 2 : 1;
-}
 
 static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     GemmPlan g;
@@ -561,74 +522,69 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     g.nkb = (K + kBlockK - 1) / kBlockK;
     const int tiles = g.tilesA * g.tilesB;
     const int sms = num_sms();
-    const int capacity = sms * ctas_per_sm(g.bn);
-    // Split K so the busiest SM streams as little of one tile's weights as
-    // possible: load(sk) = ceil(tiles*sk / sms) / sk, with a small penalty per
-    // split for the partial-tile traffic; all CTAs must be co-resident and keep
-    // >= 2 k-blocks each.
+    // Decode (swap-AB) shapes have few tiles: split K so the busiest SM
+    // streams as little of one tile's weights as possible, load(sk) =
+    // ceil(tiles*sk / sms) / sk, with a small per-split penalty (DSMEM partial
+    // traffic).  A split keeps >= 2 k-blocks per CTA and all clusters of the
+    // grid must be resident in one wave.
     int best = 1;
     double best_cost = 1e30;
-    for (int sk = 1; sk <= 16; ++sk) {
-        if (sk > 1 && (tiles * sk > capacity || sk * 2 > g.nkb || tiles > kMaxSplitTiles)) break;
+    for (int sk = 1; sk <= kMaxSplitK && g.swap; ++sk) {
+        if (sk > 1 && sk * 2 > g.nkb) break;
+        if (sk > 1 && max_clusters_bn(g.bn, sk) < tiles) continue;
         const double load = (double)((tiles * sk + sms - 1) / sms) / sk;
         const double cost = load * (1.0 + 0.03 * sk);
         if (cost < best_cost - 1e-9) { best_cost = cost; best = sk; }
     }
     static const int sk_env = [] { const char* e = getenv("FT2_GEMM_SPLITK"); return e ? atoi(e) : 0; }();
-    if (sk_env > 0) {
-        best = sk_env < g.nkb ? sk_env : g.nkb;
-        while (best > 1 && tiles * best > capacity) --best;
+    if (sk_env > 0 && g.swap) {
+        int sk = sk_env < g.nkb ? sk_env : g.nkb;
+        if (sk > kMaxSplitK) sk = kMaxSplitK;
+        while (sk > 1 && max_clusters_bn(g.bn, sk) < 1) --sk;
+        best = sk;
     }
     g.splitk = best;
     return g;
 }
 
-size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K) {
-    if (M <= 0 || N <= 0 || K <= 0) return 0;
-    GemmPlan g = plan_gemm(M, N, K);
-    if (g.splitk <= 1) return 0;
-    const size_t tiles = (size_t)g.tilesA * g.tilesB;
-    return kCounterBytes + tiles * g.splitk * (size_t)g.bn * kBlockA * 4;
-}
+// The cluster split-K needs no global workspace.
+size_t gemm_ws_bytes(int32_t, int32_t, int32_t) { return 0; }
 
-template <int BN, int STAGES>
-static cudaError_t launch_cfg(const GemmArgs& a, GemmK p, cudaStream_t st, int* n_launch) {
-    using L = GemmSmem<BN, STAGES>;
+template <int BN, bool SWAP>
+static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st, int* n_launch) {
     CUtensorMap ma, mb;
-    const void* pa = p.swap ? (const void*)a.w : (const void*)a.x;
-    const void* pb = p.swap ? (const void*)a.x : (const void*)a.w;
-    int64_t lda = p.swap ? a.ldw : a.ldx, ldb = p.swap ? a.ldx : a.ldw;
+    const void* pa = SWAP ? (const void*)a.w : (const void*)a.x;
+    const void* pb = SWAP ? (const void*)a.x : (const void*)a.w;
+    const int64_t lda = SWAP ? a.ldw : a.ldx, ldb = SWAP ? a.ldx : a.ldw;
     if (!make_map(&ma, pa, p.rowsA, a.K, lda, kBlockA)) return cudaErrorInvalidValue;
     if (!make_map(&mb, pb, p.rowsB, a.K, ldb, BN)) return cudaErrorInvalidValue;
-    static bool attr_set = false;  // per template instance
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, STAGES>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             L::kBytes);
-        if (e != cudaSuccess) return e;
-        attr_set = true;
-    }
+    cudaError_t e = set_attrs<BN, SWAP>();
+    if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);
     cfg.blockDim = dim3(kGemmThreads);
-    cfg.dynamicSmemBytes = L::kBytes;
+    cfg.dynamicSmemBytes = Cfg<BN>::kBytes;
     cfg.stream = st;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = 1;
+    attr[1].id = cudaLaunchAttributeClusterDimension;
+    attr[1].val.clusterDim.x = 1;
+    attr[1].val.clusterDim.y = (unsigned)p.splitk;
+    attr[1].val.clusterDim.z = 1;
     cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, STAGES>, ma, mb, p);
+    cfg.numAttrs = p.splitk > 1 ? 2 : 1;
+    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
-    GemmPlan g = plan_gemm(a.M, a.N, a.K);
+    const GemmPlan g = plan_gemm(a.M, a.N, a.K);
     GemmK p = {};
     p.M = a.M;
     p.N = a.N;
     p.K = a.K;
-    p.swap = g.swap;
     p.rowsA = g.swap ? a.N : a.M;
     p.rowsB = g.swap ? a.M : a.N;
     p.tilesA = g.tilesA;
@@ -652,23 +608,20 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cur_step = a.cur_step;
     p.base_row = a.base_row;
     p.w_static = a.w_static;
-    if (g.splitk > 1) {
-        uintptr_t base = reinterpret_cast<uintptr_t>(a.ws);
-        p.tile_ctr = reinterpret_cast<uint32_t*>(base);
-        uintptr_t part = base + kCounterBytes;
-        p.partials = reinterpret_cast<float4*>(part);
-    }
+    if (!g.swap) return launch_cfg<128, false>(a, p, st, n_launch);
     switch (g.bn) {
-        case 16: return launch_cfg<16, Stages<16>::value>(a, p, st, n_launch);
-        case 32: {
-            static const int st_env = [] { const char* e = getenv("FT2_GEMM_STAGES32"); return e ? atoi(e) : 0; }();
-            if (st_env == 8) return launch_cfg<32, 8>(a, p, st, n_launch);
-            if (st_env == 10) return launch_cfg<32, 10>(a, p, st, n_launch);
-            return launch_cfg<32, Stages<32>::value>(a, p, st, n_launch);
-        }
-        case 64: return launch_cfg<64, Stages<64>::value>(a, p, st, n_launch);
-        default: return launch_cfg<128, Stages<128>::value>(a, p, st, n_launch);
+        case 16: return launch_cfg<16, true>(a, p, st, n_launch);
+        case 32: return launch_cfg<32, true>(a, p, st, n_launch);
+        case 64: return launch_cfg<64, true>(a, p, st, n_launch);
+        default: return launch_cfg<128, true>(a, p, st, n_launch);
     }
 }
 
 }  // namespace ft2impl
+
+#ifdef FT2_GEMM_TRACE
+extern "C" int ft2_debug_trace_read(void* dst, size_t bytes) {
+    if (bytes > sizeof(ft2impl::g_trace)) bytes = sizeof(ft2impl::g_trace);
+    return (int)cudaMemcpyFromSymbol(dst, ft2impl::g_trace, bytes);
+}
+#endif
