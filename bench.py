@@ -46,6 +46,8 @@ def parse():
     ap.add_argument("--prompt", type=int, default=128)
     ap.add_argument("--gen", type=int, default=60)
     ap.add_argument("--no-extras", action="store_true", help="skip the kernel roofline / cpu baseline legs")
+    ap.add_argument("--profile", action="store_true",
+                    help="warm up, then run exactly one fused request (for ncu launch lists) and exit")
     return ap.parse_args()
 
 
@@ -227,6 +229,16 @@ def main():
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms = float(t.item())
         return ms
+
+    if args.profile:
+        for _ in range(2):
+            runner.generate(prompt, "fused")
+        torch.cuda.synchronize()
+        torch.cuda.nvtx.range_push("ft2_profiled_request")
+        runner.generate(prompt, "fused")
+        torch.cuda.synchronize()
+        torch.cuda.nvtx.range_pop()
+        return 0
 
     modes = ["fused", "off", "standalone", "fused_plain"]
     # warm-up (captures the decode graphs of every mode)

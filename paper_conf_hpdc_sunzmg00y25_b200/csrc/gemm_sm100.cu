@@ -34,6 +34,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
+#include <stdio.h>
 #include <stdlib.h>
 
 #include <mutex>
@@ -50,7 +51,8 @@ constexpr int kBlockK = 64;   // one 128-byte swizzle atom of bf16
 constexpr int kUmmaK = 16;
 constexpr int kGemmThreads = 192;
 constexpr int kMaxSitesPerCta = 64;
-constexpr int kMaxSplitK = 16;  // cluster size along K (non-portable above 8)
+constexpr int kMaxSplitK = 16;        // cluster size along K (non-portable above 8)
+constexpr int kMaxSplitPlanned = 12;  // largest split the planner picks (16-CTA clusters schedule slowly)
 
 #ifdef FT2_GEMM_TRACE
 // Debug builds only (lib/libft2_trace.so): per-CTA timestamps.
@@ -467,6 +469,10 @@ static cudaError_t set_attrs() {
                                              Cfg<BN>::kBytes);
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        // full shared-memory carveout so two ~105 KB decode CTAs share an SM
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                     (int)cudaSharedmemCarveoutMaxShared);
         return e;
     }();
     return res;
@@ -522,19 +528,18 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     g.nkb = (K + kBlockK - 1) / kBlockK;
     const int tiles = g.tilesA * g.tilesB;
     const int sms = num_sms();
-    // Decode (swap-AB) shapes have few tiles: split K so the busiest SM
-    // streams as little of one tile's weights as possible, load(sk) =
-    // ceil(tiles*sk / sms) / sk, with a small per-split penalty (DSMEM partial
-    // traffic).  A split keeps >= 2 k-blocks per CTA and all clusters of the
-    // grid must be resident in one wave.
+    // Decode (swap-AB) shapes have few tiles (N/128): split K across a cluster
+    // so that every SM streams weights.  Measured on B200 (tools/
+    // sweep_splitk.sh, profiles/): the best split is the largest one with
+    // tiles * splitk <= 2 * SMs (two ~105 KB CTAs fit an SM), >= 4 k-blocks of
+    // 64 per CTA, and a cluster of at most 12 CTAs.
     int best = 1;
-    double best_cost = 1e30;
-    for (int sk = 1; sk <= kMaxSplitK && g.swap; ++sk) {
-        if (sk > 1 && sk * 2 > g.nkb) break;
-        if (sk > 1 && max_clusters_bn(g.bn, sk) < tiles) continue;
-        const double load = (double)((tiles * sk + sms - 1) / sms) / sk;
-        const double cost = load * (1.0 + 0.03 * sk);
-        if (cost < best_cost - 1e-9) { best_cost = cost; best = sk; }
+    if (g.swap) {
+        for (int sk = 2; sk <= kMaxSplitPlanned; ++sk) {
+            if (tiles * sk > 2 * sms || g.nkb < 4 * sk) break;
+            if (max_clusters_bn(g.bn, sk) < 1) break;
+            best = sk;
+        }
     }
     static const int sk_env = [] { const char* e = getenv("FT2_GEMM_SPLITK"); return e ? atoi(e) : 0; }();
     if (sk_env > 0 && g.swap) {
@@ -544,6 +549,13 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
         best = sk;
     }
     g.splitk = best;
+    static const bool dbg = getenv("FT2_GEMM_DEBUG") != nullptr;
+    if (dbg) {
+        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d bn=%d tiles=%dx%d nkb=%d splitk=%d clusters(sk)=", M, N, K,
+                g.swap, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk);
+        for (int sk = 2; sk <= 8 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
+        fprintf(stderr, "\n");
+    }
     return g;
 }
 

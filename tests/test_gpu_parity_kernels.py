@@ -244,3 +244,38 @@ def test_inject_bit_exact(ft2):
         yd = dev(y2)
         ft2.inject_faults(yd, sd, layer, 0, base_row=dev_i32(base))
         assert np.array_equal(host(yd), ref)
+
+
+def test_tp_sharded_bounds_equal_unsharded(ft2):
+    """Column shards -> keys (finalize=0) -> MAX combine -> finalize == unsharded bounds (bit-exact)."""
+    rows, n, world = 256, 4096, 4
+    y = _tensor(rows, n, seed=21)
+    so = [0, 64, 64, 200, 256]
+    rb, rk, _ = oracle.bounds(y.copy(), seq_offsets=so)
+    keys = []
+    for r in range(world):
+        shard = np.ascontiguousarray(y[:, r * n // world:(r + 1) * n // world])
+        _, _, k, _ = _gpu_bounds(ft2, shard, so, finalize=False)
+        keys.append(torch.as_tensor(k))
+    comb = torch.stack(keys).amax(0).contiguous()
+    assert np.array_equal(comb.numpy(), _oracle_keys_encoded(rk))
+    b = torch.zeros((4, 2), dtype=torch.bfloat16, device="cuda")
+    ft2.bounds_finalize(comb.cuda(), b)
+    assert np.array_equal(host(b), rb)
+
+
+def test_tp_bounds_nccl_world1(ft2):
+    """The product TP path (kernel keys -> NCCL MAX all-reduce -> finalize) on a 1-rank NCCL group."""
+    import socket
+    import torch.distributed as dist
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+    if not dist.is_initialized():
+        s = socket.socket(); s.bind(("127.0.0.1", 0)); port = s.getsockname()[1]; s.close()
+        dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+    y = _tensor(128, 1024, seed=22)
+    so = [0, 32, 128]
+    rb, _, _ = oracle.bounds(y.copy(), seq_offsets=so)
+    b = torch.zeros((2, 2), dtype=torch.bfloat16, device="cuda")
+    tp.tp_bounds_from_prefill(dev(y), b, ft2.make_workspace(2), seq_offsets=dev_i32(so), num_seqs=2)
+    assert np.array_equal(host(b), rb)
+    dist.destroy_process_group()
