@@ -146,6 +146,7 @@ class Runner:
         self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
         self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h)
         self.crit_names = cfg.critical_names()
+        self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
         self.state = FT2State(self.n_crit, batch, dv)
         H, D = cfg.n_heads, cfg.head_dim
@@ -188,39 +189,53 @@ class Runner:
     def _crit_id(self, blk, name):
         return blk * len(self.crit_names) + self.crit_names.index(name)
 
+    def _lin_id(self, blk, name):
+        """Linear-layer id for fault sites: block-major over all linear layers."""
+        return blk * len(self.lin_names) + self.lin_names.index(name)
+
     def _linear(self, x2, blk: Block, name: str, phase: str, step_for_sites=None):
         """One linear layer of the block; FT2 work on critical ones.
 
         phase "prefill": bounds from the first-token output (+ NaN/Inf correction).
         phase "decode":  check-and-clip according to self.mode.
+        With self.sites set (fault-injection campaign, eager mode only), the
+        site of each trial row is applied to the layer's bf16 output before the
+        check (order GEMM -> bias -> bf16 -> inject -> check, readings A19/A20).
         """
         w, b = blk.w[name], blk.b[name]
         crit = name in self.crit_names
+        sites = self.sites
+        step = 0 if phase == "prefill" else (step_for_sites if step_for_sites is not None else 0)
+        lid = self._lin_id(blk.idx, name) if sites is not None else 0
         if phase == "prefill":
+            # prefill GEMMs are compute-bound (M = B*T); they run on cuBLAS in
+            # every mode and FT2's first-token work is the bounds sweep below
+            y = F.linear(x2, w, b)
+            if sites is not None:
+                F2.inject_faults(y, sites, lid, 0, base_row=self.seq_offsets, n_sites=self.B)
             if crit and self.mode != "off":
-                # prefill GEMMs are compute-bound (M = B*T); they run on cuBLAS in
-                # every mode and FT2's first-token work is the bounds sweep below
-                y = F.linear(x2, w, b)
                 cid = self._crit_id(blk.idx, name)
                 st = self.state
                 F2.bounds_from_prefill(y, st.bounds[cid], st.ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
                                        scale=self.scale, correct_nonfinite=True, nonfinite_count=st.nonfinite[cid])
-                return y
-            return F.linear(x2, w, b)
+            return y
         # decode
-        if not crit or self.mode == "off":
-            return F.linear(x2, w, b)
+        if not crit or self.mode in ("off", "standalone"):
+            y = F.linear(x2, w, b)
+            if sites is not None:
+                F2.inject_faults(y, sites, lid, step, n_sites=self.B)
+            if crit and self.mode == "standalone":
+                cid = self._crit_id(blk.idx, name)
+                st = self.state
+                F2.protect(y, st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid])
+            return y
         cid = self._crit_id(blk.idx, name)
         st = self.state
-        if self.mode == "standalone":
-            y = F.linear(x2, w, b)
-            F2.protect(y, st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid])
-            return y
         y = torch.empty((x2.shape[0], w.shape[0]), dtype=torch.bfloat16, device=x2.device)
         mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
         F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, bounds=st.bounds[cid], num_seqs=self.B,
-                              corrected_count=st.corrected[cid], sites=self.sites,
-                              cur_layer=cid, cur_step=step_for_sites if step_for_sites is not None else 0)
+                              corrected_count=st.corrected[cid], sites=sites, n_sites=self.B if sites is not None else None,
+                              cur_layer=lid, cur_step=step)
         return y
 
     # ------------------------------------------------------------ forward
@@ -330,6 +345,8 @@ class Runner:
 
     def generate(self, prompt_ids, mode="fused", use_graph=True):
         """Greedy generation of G tokens (1 first token + G-1 decode steps)."""
+        if self.sites is not None and use_graph:
+            raise ValueError("fault sites need eager decode (use_graph=False): the step index changes per token")
         self.mode = mode
         self._site_step = None
         self.state.reset_counters()
@@ -348,8 +365,10 @@ class Runner:
             for _ in range(self.G - 1):
                 g.replay()
         else:
-            for _ in range(self.G - 1):
+            for t in range(1, self.G):
+                self._site_step = t   # decode step t (0 = prefill / first token)
                 self._decode_step()
+            self._site_step = None
         if ev:
             ev[2].record()
             self._phase_events.append(ev)
