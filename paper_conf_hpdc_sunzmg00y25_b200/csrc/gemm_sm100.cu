@@ -554,7 +554,22 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
         fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d bn=%d tiles=%dx%d nkb=%d splitk=%d clusters(sk)=", M, N, K,
                 g.swap, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk);
         for (int sk = 2; sk <= 8 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
-        fprintf(stderr, "\n");
+        int occ = -1;
+        if (g.bn == 32) {
+            set_attrs<32, true>();
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gemm_kernel<32, true>, kGemmThreads, Cfg<32>::kBytes);
+        }
+        size_t avail2 = 0, avail1 = 0;
+        cudaOccupancyAvailableDynamicSMemPerBlock(&avail2, gemm_kernel<32, true>, 2, kGemmThreads);
+        cudaOccupancyAvailableDynamicSMemPerBlock(&avail1, gemm_kernel<32, true>, 1, kGemmThreads);
+        cudaFuncAttributes fa;
+        cudaFuncGetAttributes(&fa, gemm_kernel<32, true>);
+        int smem_sm = 0, dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
+        fprintf(stderr, " occ(bn32)=%d smem=%d avail@2=%zu avail@1=%zu regs=%d static=%zu maxdyn=%d carve=%d smem/SM=%d\n",
+                occ, Cfg<32>::kBytes, avail2, avail1, fa.numRegs, fa.sharedSizeBytes, fa.maxDynamicSharedSizeBytes,
+                fa.preferredShmemCarveout, smem_sm);
     }
     return g;
 }

@@ -51,6 +51,8 @@ for M, N, K in shapes:
     buf[:] = 0
     L.ft2_debug_trace_write_zero() if hasattr(L, "ft2_debug_trace_write_zero") else None
     print(f"== M={M} N={N} K={K}: {t.shape[0]} CTAs; kernel span {(t[:, 7].max() - t0) / 1000:.2f} us")
+    st = (t[:, 0] - t0) / 1000.0
+    print(f"   start-time histogram (us): {np.histogram(st, bins=8)[0].tolist()} edges {np.round(np.histogram(st, bins=8)[1], 2).tolist()}")
     for j, n in enumerate(names):
         v = (t[:, j] - t0) / 1000.0
         v = v[t[:, j] > 0]
