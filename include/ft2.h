@@ -57,9 +57,9 @@ typedef enum {
     FT2_ERR_CUDA = 4
 } ft2_status;
 
-/* Activation dtype.  BF16 is implemented; FP16/FP32 (the paper's FP16 main
- * precision L282 and its FP32 study L334) return FT2_ERR_UNSUPPORTED in this
- * release. */
+/* Activation dtype.  BF16 and FP16 (the paper's main precision, L282) are
+ * implemented by every entry point; FP32 (the paper's FP32 study, L334)
+ * returns FT2_ERR_UNSUPPORTED in this release. */
 typedef enum { FT2_BF16 = 0, FT2_FP16 = 1, FT2_FP32 = 2 } ft2_dtype;
 
 /* Fault models, PAPER.md L84 (Sec. 2.2): single-bit flip, double-bit flip,
@@ -159,7 +159,7 @@ ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int
 /* Bounds from (all-reduced) keys in the ft2_bounds_from_prefill keys_out
  * encoding: the second half of the tensor-parallel path. */
 ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scale,
-                               ft2_dtype dtype, void* bounds_out, void* stream);
+                               ft2_dtype dtype, void* bounds_out, void* stream);  /* dtype: BF16 / FP16 */
 
 /* Online range restriction of one protected layer's output: PAPER.md L151,
  * L259-L261 (Sec. 4.3: check every neuron after each critical layer), L261/L270
@@ -181,7 +181,7 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
  * MMA, TMEM accumulators, TMA-fed shared-memory pipeline on sm_100a):
  *   y[m, j] = check(inject(bf16_rne(sum_k x[m, k] * w[j, k] + bias[j])))
  * x [M x K] (ldx), w [N x K] (ldw, nn.Linear layout), bias [N] or NULL, y [M x N]
- * (ldy), all bf16, fp32 accumulation.  The K reduction is complete before the
+ * (ldy), all of type dtype (FT2_BF16 or FT2_FP16), fp32 accumulation.  The K reduction is complete before the
  * epilogue (split-K partial sums are combined first: clipping is non-linear).
  * mode         FT2_GEMM_PLAIN or FT2_GEMM_CHECK.
  * col_begin/col_end  the protected column slice [col_begin, col_end) (e.g. V of
@@ -204,7 +204,7 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
 size_t ft2_gemm_workspace_bytes(int32_t M, int32_t N, int32_t K);
 ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw,
                                   const void* bias, void* y, int64_t ldy, int32_t M, int32_t N,
-                                  int32_t K, ft2_gemm_mode mode, int32_t col_begin, int32_t col_end,
+                                  int32_t K, ft2_gemm_mode mode, ft2_dtype dtype, int32_t col_begin, int32_t col_end,
                                   const int32_t* row_to_seq, const void* bounds, int32_t num_seqs,
                                   uint32_t* corrected_count, const ft2_fault_site* sites,
                                   int32_t n_sites, int32_t cur_layer, int32_t cur_step,

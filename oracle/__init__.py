@@ -74,6 +74,19 @@ def lib():
             ("ft2o_protected_linear", None, [P, i64, P, i64, P, i32, i32, i32, P, i64, P, P, i32, P,
                                              P, i32, i32, i32, P]),
             ("ft2o_site_size", i32, []),
+            ("ft2o_isnan_dt", ctypes.c_int, [u16, ctypes.c_int]), ("ft2o_isinf_dt", ctypes.c_int, [u16, ctypes.c_int]),
+            ("ft2o_isfinite_dt", ctypes.c_int, [u16, ctypes.c_int]),
+            ("ft2o_to_f64_dt", ctypes.c_double, [u16, ctypes.c_int]),
+            ("ft2o_f64_to_dt_rne", u16, [ctypes.c_double, ctypes.c_int]),
+            ("ft2o_f64_to_dt_dir", u16, [ctypes.c_double, ctypes.c_int, ctypes.c_int]),
+            ("ft2o_scale_bound_dt", u16, [u16, ctypes.c_float, ctypes.c_int, ctypes.c_int]),
+            ("ft2o_clip_value_dt", u16, [u16, u16, u16, ctypes.c_int]),
+            ("ft2o_protect_dt", None, [P, i64, i64, i64, P, P, i32, P, ctypes.c_int]),
+            ("ft2o_bounds_dt", None, [P, i64, i64, i64, P, i32, ctypes.c_float, i32, P, P, P, ctypes.c_int]),
+            ("ft2o_bounds_from_keys_dt", None, [P, i32, ctypes.c_float, P, ctypes.c_int]),
+            ("ft2o_linear_f64_dt", None, [P, i64, P, i64, P, i32, i32, i32, P, P, i64, ctypes.c_int]),
+            ("ft2o_protected_linear_dt", None, [P, i64, P, i64, P, i32, i32, i32, P, i64, P, P, i32, P,
+                                                P, i32, i32, i32, P, ctypes.c_int]),
         ]:
             f = getattr(L, name)
             f.restype = res
@@ -94,6 +107,11 @@ def _u16(a):
 
 
 # ----------------------------------------------------------------- scalars --
+def isnan_dt(b: int, dtype: int) -> bool: return bool(lib().ft2o_isnan_dt(b, dtype))
+def isinf_dt(b: int, dtype: int) -> bool: return bool(lib().ft2o_isinf_dt(b, dtype))
+def to_f64(b: int, dtype: int = DT_BF16) -> float: return lib().ft2o_to_f64_dt(b, dtype)
+def f64_to(d: float, dtype: int = DT_BF16) -> int: return lib().ft2o_f64_to_dt_rne(d, dtype)
+def f64_to_dir(d: float, direction: int, dtype: int = DT_BF16) -> int: return lib().ft2o_f64_to_dt_dir(d, direction, dtype)
 def key(b: int) -> int: return lib().ft2o_key(b)
 def unkey(k: int) -> int: return lib().ft2o_unkey(k)
 def isnan(b: int) -> bool: return bool(lib().ft2o_isnan(b))
@@ -101,8 +119,9 @@ def isinf(b: int) -> bool: return bool(lib().ft2o_isinf(b))
 def bf16_to_f64(b: int) -> float: return lib().ft2o_bf16_to_f64(b)
 def f64_to_bf16(d: float) -> int: return lib().ft2o_f64_to_bf16_rne(d)
 def f64_to_bf16_dir(d: float, direction: int) -> int: return lib().ft2o_f64_to_bf16_dir(d, direction)
-def scale_bound(raw: int, c: float, is_hi: bool) -> int: return lib().ft2o_scale_bound(raw, c, int(is_hi))
-def clip_value(y: int, lo: int, hi: int) -> int: return lib().ft2o_clip_value(y, lo, hi)
+def scale_bound(raw: int, c: float, is_hi: bool, dtype: int = DT_BF16) -> int:
+    return lib().ft2o_scale_bound_dt(raw, c, int(is_hi), dtype)
+def clip_value(y: int, lo: int, hi: int, dtype: int = DT_BF16) -> int: return lib().ft2o_clip_value_dt(y, lo, hi, dtype)
 
 
 def philox4x32_10(ctr, key_):
@@ -114,7 +133,7 @@ def philox4x32_10(ctr, key_):
 
 
 # ------------------------------------------------------------------ tensors --
-def bounds(y, seq_offsets=None, scale: float = 2.0, correct_nonfinite: bool = False, ld=None):
+def bounds(y, seq_offsets=None, scale: float = 2.0, correct_nonfinite: bool = False, ld=None, dtype=DT_BF16):
     """R2-R4.  y: uint16 [rows, n] (modified in place iff correct_nonfinite).
 
     Returns (bounds uint16 [S,2], raw_keys int32 [S,2], nonfinite uint32 [S]).
@@ -127,19 +146,19 @@ def bounds(y, seq_offsets=None, scale: float = 2.0, correct_nonfinite: bool = Fa
     b = np.zeros((S, 2), np.uint16)
     k = np.zeros((S, 2), np.int32)
     nf = np.zeros(S, np.uint32)
-    lib().ft2o_bounds(_p(y), rows, n, ld, _p(so), S, scale, int(correct_nonfinite), _p(b), _p(k), _p(nf))
+    lib().ft2o_bounds_dt(_p(y), rows, n, ld, _p(so), S, scale, int(correct_nonfinite), _p(b), _p(k), _p(nf), dtype)
     return b, k, nf
 
 
-def bounds_from_keys(raw_keys, scale: float = 2.0):
+def bounds_from_keys(raw_keys, scale: float = 2.0, dtype=DT_BF16):
     k = np.ascontiguousarray(raw_keys, dtype=np.int32)
     S = k.shape[0]
     b = np.zeros((S, 2), np.uint16)
-    lib().ft2o_bounds_from_keys(_p(k), S, scale, _p(b))
+    lib().ft2o_bounds_from_keys_dt(_p(k), S, scale, _p(b), dtype)
     return b
 
 
-def protect(y, bounds_, row_to_seq=None, count=None):
+def protect(y, bounds_, row_to_seq=None, count=None, dtype=DT_BF16):
     """R5 in place.  y: uint16 [rows, n]; bounds_: uint16 [S, 2]. Returns count [S]."""
     assert y.dtype == np.uint16 and y.ndim == 2 and y.flags.c_contiguous
     rows, n = y.shape
@@ -148,7 +167,7 @@ def protect(y, bounds_, row_to_seq=None, count=None):
     r2s = None if row_to_seq is None else np.ascontiguousarray(row_to_seq, dtype=np.int32)
     if count is None:
         count = np.zeros(S, np.uint32)
-    lib().ft2o_protect(_p(y), rows, n, n, _p(r2s), _p(b), S, _p(count))
+    lib().ft2o_protect_dt(_p(y), rows, n, n, _p(r2s), _p(b), S, _p(count), dtype)
     return count
 
 
@@ -169,8 +188,8 @@ def inject(y, sites, cur_layer, cur_step, base_row=None):
     return y
 
 
-def linear_f64(x, w, bias=None):
-    """R8: returns (y_f64 [M,N], y_bf16 [M,N])."""
+def linear_f64(x, w, bias=None, dtype=DT_BF16):
+    """R8: returns (y_f64 [M,N], y rounded to the activation dtype [M,N] as uint16 bits)."""
     x = _u16(x)
     w = _u16(w)
     M, K = x.shape
@@ -178,12 +197,12 @@ def linear_f64(x, w, bias=None):
     b = None if bias is None else _u16(bias)
     yd = np.zeros((M, N), np.float64)
     yb = np.zeros((M, N), np.uint16)
-    lib().ft2o_linear_f64(_p(x), K, _p(w), K, _p(b), M, N, K, _p(yd), _p(yb), N)
+    lib().ft2o_linear_f64_dt(_p(x), K, _p(w), K, _p(b), M, N, K, _p(yd), _p(yb), N, dtype)
     return yd, yb
 
 
 def protected_linear(x, w, bias, bounds_, row_to_seq=None, sites=None, cur_layer=0, cur_step=0,
-                     base_row=None):
+                     base_row=None, dtype=DT_BF16):
     """R8 -> R7 -> R5. Returns (y bf16 [M,N], count [S])."""
     x = _u16(x)
     w = _u16(w)
@@ -198,6 +217,6 @@ def protected_linear(x, w, bias, bounds_, row_to_seq=None, sites=None, cur_layer
     s = None if sites is None else np.ascontiguousarray(sites, dtype=SITE_DTYPE)
     ns = 0 if s is None else s.size
     br = None if base_row is None else np.ascontiguousarray(base_row, dtype=np.int32)
-    lib().ft2o_protected_linear(_p(x), K, _p(w), K, _p(b), M, N, K, _p(y), N, _p(r2s), _p(bd), S,
-                                _p(cnt), _p(s), ns, cur_layer, cur_step, _p(br))
+    lib().ft2o_protected_linear_dt(_p(x), K, _p(w), K, _p(b), M, N, K, _p(y), N, _p(r2s), _p(bd), S,
+                                   _p(cnt), _p(s), ns, cur_layer, cur_step, _p(br), dtype)
     return y, cnt

@@ -26,11 +26,32 @@
 #define EXPORT __attribute__((visibility("default")))
 
 /* ------------------------------------------------------------------ R0 --- */
-/* bf16 layout 1/8/7 (PAPER.md L185 describes the FP16 1/5/10 analogue). */
+/* 16-bit floating formats: bf16 1/8/7 (the build's activation type) and the
+ * paper's FP16 1/5/10 (PAPER.md L185 describes that layout; L282: FP16 models).
+ * dtype 0 = bf16, 1 = fp16.  Both are sign-magnitude, so the order key below
+ * is the same function for both; only the exponent field differs. */
+typedef struct {
+    int mbits;        /* fraction bits */
+    int bias;         /* exponent bias */
+    uint16_t expmask; /* exponent field */
+    uint16_t maxfin;  /* largest finite magnitude */
+    uint16_t qnan;    /* canonical NaN */
+} ft2o_fmt;
+static const ft2o_fmt FMT[2] = {
+    {7, 127, 0x7F80, 0x7F7F, 0x7FC0},  /* bf16 */
+    {10, 15, 0x7C00, 0x7BFF, 0x7E00},  /* fp16 */
+};
+static const ft2o_fmt* fmt_of(int dtype) { return &FMT[dtype == 1 ? 1 : 0]; }
 
-EXPORT int ft2o_isnan(uint16_t b) { return (b & 0x7FFF) > 0x7F80; }
-EXPORT int ft2o_isinf(uint16_t b) { return (b & 0x7FFF) == 0x7F80; }
-EXPORT int ft2o_isfinite(uint16_t b) { return (b & 0x7F80) != 0x7F80; }
+EXPORT int ft2o_isnan_dt(uint16_t b, int dtype) { return (b & 0x7FFF) > fmt_of(dtype)->expmask; }
+EXPORT int ft2o_isinf_dt(uint16_t b, int dtype) { return (b & 0x7FFF) == fmt_of(dtype)->expmask; }
+EXPORT int ft2o_isfinite_dt(uint16_t b, int dtype) {
+    const uint16_t e = fmt_of(dtype)->expmask;
+    return (b & e) != e;
+}
+EXPORT int ft2o_isnan(uint16_t b) { return ft2o_isnan_dt(b, 0); }
+EXPORT int ft2o_isinf(uint16_t b) { return ft2o_isinf_dt(b, 0); }
+EXPORT int ft2o_isfinite(uint16_t b) { return ft2o_isfinite_dt(b, 0); }
 
 EXPORT uint16_t ft2o_key(uint16_t b) {
     return (b & 0x8000) ? (uint16_t)(~b & 0xFFFF) : (uint16_t)(b | 0x8000);
@@ -40,73 +61,78 @@ EXPORT uint16_t ft2o_unkey(uint16_t k) {
     return (k & 0x8000) ? (uint16_t)(k & 0x7FFF) : (uint16_t)(~k & 0xFFFF);
 }
 
-EXPORT double ft2o_bf16_to_f64(uint16_t b) {
-    uint32_t u = (uint32_t)b << 16;
-    float f;
-    memcpy(&f, &u, 4);
-    return (double)f;
+/* Exact value of a 16-bit float (from the definition of the format). */
+EXPORT double ft2o_to_f64_dt(uint16_t b, int dtype) {
+    const ft2o_fmt* f = fmt_of(dtype);
+    const int ebits = (f->expmask >> f->mbits) & 0xFF;  /* all-ones exponent value */
+    int e = (b >> f->mbits) & ebits;
+    int m = b & ((1 << f->mbits) - 1);
+    double s = (b & 0x8000) ? -1.0 : 1.0;
+    if (e == ebits) return m ? NAN : s * INFINITY;
+    if (e == 0) return s * ldexp((double)m, 1 - f->bias - f->mbits);      /* subnormal */
+    return s * ldexp((double)((1 << f->mbits) | m), e - f->bias - f->mbits);
 }
+EXPORT double ft2o_bf16_to_f64(uint16_t b) { return ft2o_to_f64_dt(b, 0); }
 
-/* Round-to-nearest-even of an arbitrary double to bf16 (NaN -> 0x7FC0).
- * Written from the definition: find the representable neighbours' spacing at
- * the value's binade and round the scaled significand with rint() (the
- * default FE_TONEAREST mode is ties-to-even).  Used for R8 (fp64 GEMM -> bf16)
- * and for fp32 inputs (exact promotion to double). */
-EXPORT uint16_t ft2o_f64_to_bf16_rne(double d) {
-    if (isnan(d)) return 0x7FC0;
+/* Round-to-nearest-even of an arbitrary double to the 16-bit format (NaN ->
+ * canonical NaN).  Written from the definition: the representable spacing at
+ * the value's binade is 2^(E - mbits) (2^(emin - mbits) below the normal
+ * range), and rint() in the default FE_TONEAREST mode is ties-to-even.  Used
+ * for R8 (fp64 GEMM -> activation type) and for fp32 inputs (exact promotion
+ * to double). */
+EXPORT uint16_t ft2o_f64_to_dt_rne(double d, int dtype) {
+    const ft2o_fmt* f = fmt_of(dtype);
+    const int emin = 1 - f->bias;
+    if (isnan(d)) return f->qnan;
     uint16_t sign = signbit(d) ? 0x8000 : 0x0000;
     double a = fabs(d);
-    if (isinf(a)) return sign | 0x7F80;
-    if (a < ldexp(1.0, -126)) {
-        /* subnormal range: spacing 2^-133; rint(a * 2^133) in [0, 128] */
-        double q = rint(ldexp(a, 133));
-        return sign | (uint16_t)q; /* q == 128 encodes the smallest normal */
+    if (isinf(a)) return sign | f->expmask;
+    if (a < ldexp(1.0, emin)) {
+        /* subnormal range; q == 2^mbits encodes the smallest normal */
+        double q = rint(ldexp(a, f->mbits - emin));
+        return sign | (uint16_t)q;
     }
     int e;
     double m = frexp(a, &e); /* a = m * 2^e, m in [0.5, 1) */
-    double q = rint(ldexp(m, 8)); /* significand with 7 fraction bits, [128, 256] */
+    double q = rint(ldexp(m, f->mbits + 1)); /* significand, [2^mbits, 2^(mbits+1)] */
     int E = e - 1;
-    if (q == 256.0) { q = 128.0; E += 1; }
-    if (E + 127 >= 255) return sign | 0x7F80; /* overflow -> Inf */
-    return sign | (uint16_t)(((E + 127) << 7) | ((int)q - 128));
+    if (q == ldexp(1.0, f->mbits + 1)) { q = ldexp(1.0, f->mbits); E += 1; }
+    if (E + f->bias >= 2 * f->bias + 1) return sign | f->expmask; /* overflow -> Inf */
+    return sign | (uint16_t)(((E + f->bias) << f->mbits) | ((int)q - (1 << f->mbits)));
 }
+EXPORT uint16_t ft2o_f64_to_bf16_rne(double d) { return ft2o_f64_to_dt_rne(d, 0); }
 
-/* Directed rounding of a double to bf16: dir = -1 toward -Inf, +1 toward +Inf.
- * Used by R3 (bounds are rounded outward, reading A10).  Defined from RNE:
- * take the nearest value, and step one ulp outward if it lies on the wrong
- * side of d. */
-static uint16_t next_up_bf16(uint16_t b) { /* next representable toward +Inf */
-    uint16_t k = ft2o_key(b);
-    return ft2o_unkey((uint16_t)(k + 1));
-}
-static uint16_t next_down_bf16(uint16_t b) {
-    uint16_t k = ft2o_key(b);
-    return ft2o_unkey((uint16_t)(k - 1));
-}
-EXPORT uint16_t ft2o_f64_to_bf16_dir(double d, int dir) {
-    uint16_t r = ft2o_f64_to_bf16_rne(d);
-    double rv = ft2o_bf16_to_f64(r);
-    if (dir < 0 && rv > d) r = next_down_bf16(r);
-    if (dir > 0 && rv < d) r = next_up_bf16(r);
+/* Directed rounding of a double: dir = -1 toward -Inf, +1 toward +Inf.  Used
+ * by R3 (bounds are rounded outward, reading A10).  Defined from RNE: take
+ * the nearest value, and step one ulp outward (in key order) if it lies on
+ * the wrong side of d. */
+EXPORT uint16_t ft2o_f64_to_dt_dir(double d, int dir, int dtype) {
+    uint16_t r = ft2o_f64_to_dt_rne(d, dtype);
+    double rv = ft2o_to_f64_dt(r, dtype);
+    if (dir < 0 && rv > d) r = ft2o_unkey((uint16_t)(ft2o_key(r) - 1));
+    if (dir > 0 && rv < d) r = ft2o_unkey((uint16_t)(ft2o_key(r) + 1));
     return r;
 }
+EXPORT uint16_t ft2o_f64_to_bf16_dir(double d, int dir) { return ft2o_f64_to_dt_dir(d, dir, 0); }
 
 /* ------------------------------------------------------------------ R3 --- */
 /* Bound scaling, PAPER.md L229-L233 (Sec. 4.2.1, TA#6): "the scaling factor is
  * set to 2".  Reading A2: widen away from the interval, i.e. lo <= 0 is
  * multiplied by c and lo > 0 divided by c (and symmetrically for hi).  The
  * product/quotient is formed in fp32 (one IEEE op), then rounded outward to
- * bf16 (A10) and saturated to +-max finite 0x7F7F (A8). */
-EXPORT uint16_t ft2o_scale_bound(uint16_t raw, float c, int is_hi) {
-    float x = (float)ft2o_bf16_to_f64(raw);
+ * the activation type (A10) and saturated to +-max finite (A8). */
+EXPORT uint16_t ft2o_scale_bound_dt(uint16_t raw, float c, int is_hi, int dtype) {
+    const ft2o_fmt* f = fmt_of(dtype);
+    float x = (float)ft2o_to_f64_dt(raw, dtype);
     volatile float s;
     if (is_hi) s = (x >= 0.0f) ? x * c : x / c;
     else       s = (x <= 0.0f) ? x * c : x / c;
-    uint16_t r = ft2o_f64_to_bf16_dir((double)s, is_hi ? +1 : -1);
-    if (r == 0x7F80) r = 0x7F7F; /* +Inf -> +max finite */
-    if (r == 0xFF80) r = 0xFF7F; /* -Inf -> -max finite */
+    uint16_t r = ft2o_f64_to_dt_dir((double)s, is_hi ? +1 : -1, dtype);
+    if (r == f->expmask) r = f->maxfin;                           /* +Inf -> +max finite */
+    if (r == (uint16_t)(0x8000 | f->expmask)) r = 0x8000 | f->maxfin; /* -Inf -> -max finite */
     return r;
 }
+EXPORT uint16_t ft2o_scale_bound(uint16_t raw, float c, int is_hi) { return ft2o_scale_bound_dt(raw, c, is_hi, 0); }
 
 /* ------------------------------------------------------------------ R5 --- */
 /* Check-and-clip of one value, PAPER.md L259-L261 (Sec. 4.3: "FT2 checks all
@@ -115,34 +141,39 @@ EXPORT uint16_t ft2o_scale_bound(uint16_t raw, float c, int is_hi) {
  * (torch.clamp + torch.nan_to_num).  Reading A5: NaN -> clamp(+0, lo, hi);
  * A6: +-Inf -> hi/lo through the clamp; A7: a value equal to a bound is in
  * bounds, order = key order. Returns the corrected bits. */
-EXPORT uint16_t ft2o_clip_value(uint16_t y, uint16_t lo, uint16_t hi) {
-    uint16_t x = ft2o_isnan(y) ? 0x0000 : y; /* nan_to_num(nan=0.0) */
+EXPORT uint16_t ft2o_clip_value_dt(uint16_t y, uint16_t lo, uint16_t hi, int dtype) {
+    uint16_t x = ft2o_isnan_dt(y, dtype) ? 0x0000 : y; /* nan_to_num(nan=0.0) */
     uint16_t k = ft2o_key(x);
     if (k < ft2o_key(lo)) return lo;
     if (k > ft2o_key(hi)) return hi;
     return x;
 }
+EXPORT uint16_t ft2o_clip_value(uint16_t y, uint16_t lo, uint16_t hi) { return ft2o_clip_value_dt(y, lo, hi, 0); }
 
 /* In-place check-and-clip of y[rows][n] (row stride ld).  Row r belongs to
  * sequence row_to_seq[r]; bounds[2*s] = lo_s, bounds[2*s+1] = hi_s.
  * count[s] += number of elements whose bits changed (R5: corrected <=> y' != y).
  * Rows whose sequence is out of [0, num_seqs) are skipped. */
-EXPORT void ft2o_protect(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
-                         const int32_t* row_to_seq, const uint16_t* bounds,
-                         int32_t num_seqs, uint32_t* count) {
+EXPORT void ft2o_protect_dt(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
+                            const int32_t* row_to_seq, const uint16_t* bounds,
+                            int32_t num_seqs, uint32_t* count, int dtype) {
     for (int64_t r = 0; r < rows; ++r) {
         int32_t s = row_to_seq ? row_to_seq[r] : (num_seqs == 1 ? 0 : (int32_t)r);
         if (s < 0 || s >= num_seqs) continue;
         uint16_t lo = bounds[2 * s], hi = bounds[2 * s + 1];
         for (int64_t j = 0; j < n; ++j) {
             uint16_t v = y[r * ld + j];
-            uint16_t w = ft2o_clip_value(v, lo, hi);
+            uint16_t w = ft2o_clip_value_dt(v, lo, hi, dtype);
             if (w != v) {
                 y[r * ld + j] = w;
                 if (count) count[s] += 1;
             }
         }
     }
+}
+EXPORT void ft2o_protect(uint16_t* y, int64_t rows, int64_t n, int64_t ld, const int32_t* row_to_seq,
+                         const uint16_t* bounds, int32_t num_seqs, uint32_t* count) {
+    ft2o_protect_dt(y, rows, n, ld, row_to_seq, bounds, num_seqs, count, 0);
 }
 
 /* ------------------------------------------------------------- R2/R3/R4 --- */
@@ -155,15 +186,15 @@ EXPORT void ft2o_protect(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
  * y: [rows][n] bits, stride ld.  seq_offsets: [S+1] row offsets (NULL = one
  * sequence covering all rows).  Outputs per sequence s:
  *   raw_keys[2s] = key(min finite) or -1, raw_keys[2s+1] = key(max finite) or -1
- *   bounds[2s], bounds[2s+1] = R3-scaled lo, hi (bf16 bits)
+ *   bounds[2s], bounds[2s+1] = R3-scaled lo, hi (bits)
  *   nonfinite[s] = number of non-finite elements
  * If correct_nonfinite, R4 applies R5 to the prefill output with the fresh
  * bounds ("NaN can always be detected and
  * corrected" during the first token). */
-EXPORT void ft2o_bounds(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
-                        const int32_t* seq_offsets, int32_t num_seqs, float scale,
-                        int32_t correct_nonfinite, uint16_t* bounds, int32_t* raw_keys,
-                        uint32_t* nonfinite) {
+EXPORT void ft2o_bounds_dt(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
+                           const int32_t* seq_offsets, int32_t num_seqs, float scale,
+                           int32_t correct_nonfinite, uint16_t* bounds, int32_t* raw_keys,
+                           uint32_t* nonfinite, int dtype) {
     for (int32_t s = 0; s < num_seqs; ++s) {
         int64_t r0 = seq_offsets ? seq_offsets[s] : 0;
         int64_t r1 = seq_offsets ? seq_offsets[s + 1] : rows;
@@ -173,7 +204,7 @@ EXPORT void ft2o_bounds(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
         for (int64_t r = r0; r < r1; ++r) {
             for (int64_t j = 0; j < n; ++j) {
                 uint16_t v = y[r * ld + j];
-                if (!ft2o_isfinite(v)) { nf++; continue; }
+                if (!ft2o_isfinite_dt(v, dtype)) { nf++; continue; }
                 uint16_t k = ft2o_key(v);
                 if (!have || k < kmin) kmin = k;
                 if (!have || k > kmax) kmax = k;
@@ -182,8 +213,8 @@ EXPORT void ft2o_bounds(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
         }
         uint16_t lo, hi;
         if (have) {
-            lo = ft2o_scale_bound(ft2o_unkey(kmin), scale, 0);
-            hi = ft2o_scale_bound(ft2o_unkey(kmax), scale, 1);
+            lo = ft2o_scale_bound_dt(ft2o_unkey(kmin), scale, 0, dtype);
+            hi = ft2o_scale_bound_dt(ft2o_unkey(kmax), scale, 1, dtype);
         } else {
             lo = hi = 0x0000; /* A9 */
         }
@@ -196,21 +227,29 @@ EXPORT void ft2o_bounds(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
         if (correct_nonfinite) {
             for (int64_t r = r0; r < r1; ++r)
                 for (int64_t j = 0; j < n; ++j)
-                    y[r * ld + j] = ft2o_clip_value(y[r * ld + j], lo, hi);
+                    y[r * ld + j] = ft2o_clip_value_dt(y[r * ld + j], lo, hi, dtype);
         }
     }
+}
+EXPORT void ft2o_bounds(uint16_t* y, int64_t rows, int64_t n, int64_t ld, const int32_t* seq_offsets,
+                        int32_t num_seqs, float scale, int32_t correct_nonfinite, uint16_t* bounds,
+                        int32_t* raw_keys, uint32_t* nonfinite) {
+    ft2o_bounds_dt(y, rows, n, ld, seq_offsets, num_seqs, scale, correct_nonfinite, bounds, raw_keys, nonfinite, 0);
 }
 
 /* Bounds from raw keys (the TP path): raw_keys as produced by
  * ft2o_bounds (-1 = no finite value). */
-EXPORT void ft2o_bounds_from_keys(const int32_t* raw_keys, int32_t num_seqs, float scale,
-                                  uint16_t* bounds) {
+EXPORT void ft2o_bounds_from_keys_dt(const int32_t* raw_keys, int32_t num_seqs, float scale,
+                                     uint16_t* bounds, int dtype) {
     for (int32_t s = 0; s < num_seqs; ++s) {
         int32_t a = raw_keys[2 * s], b = raw_keys[2 * s + 1];
         if (a < 0 || b < 0) { bounds[2 * s] = bounds[2 * s + 1] = 0; continue; }
-        bounds[2 * s] = ft2o_scale_bound(ft2o_unkey((uint16_t)a), scale, 0);
-        bounds[2 * s + 1] = ft2o_scale_bound(ft2o_unkey((uint16_t)b), scale, 1);
+        bounds[2 * s] = ft2o_scale_bound_dt(ft2o_unkey((uint16_t)a), scale, 0, dtype);
+        bounds[2 * s + 1] = ft2o_scale_bound_dt(ft2o_unkey((uint16_t)b), scale, 1, dtype);
     }
+}
+EXPORT void ft2o_bounds_from_keys(const int32_t* raw_keys, int32_t num_seqs, float scale, uint16_t* bounds) {
+    ft2o_bounds_from_keys_dt(raw_keys, num_seqs, scale, bounds, 0);
 }
 
 /* --------------------------------------------------------------- Philox --- */
@@ -338,19 +377,24 @@ EXPORT void ft2o_inject(uint16_t* y, int64_t rows, int64_t n, int64_t ld, const 
 /* Reference linear layer for the fused path: y = x W^T + b (nn.Linear),
  * accumulated in fp64 (independent of summation order), rounded once to bf16.
  * x: [M][K] (ldx), w: [N][K] (ldw), bias: [N] or NULL, y: [M][N] (ldy). */
-EXPORT void ft2o_linear_f64(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
-                            const uint16_t* bias, int32_t M, int32_t N, int32_t K,
-                            double* y_f64, uint16_t* y_bf16, int64_t ldy) {
+EXPORT void ft2o_linear_f64_dt(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
+                               const uint16_t* bias, int32_t M, int32_t N, int32_t K,
+                               double* y_f64, uint16_t* y_out, int64_t ldy, int dtype) {
     for (int32_t m = 0; m < M; ++m) {
         for (int32_t j = 0; j < N; ++j) {
             double acc = 0.0;
             for (int32_t k = 0; k < K; ++k)
-                acc += ft2o_bf16_to_f64(x[(int64_t)m * ldx + k]) * ft2o_bf16_to_f64(w[(int64_t)j * ldw + k]);
-            if (bias) acc += ft2o_bf16_to_f64(bias[j]);
+                acc += ft2o_to_f64_dt(x[(int64_t)m * ldx + k], dtype) * ft2o_to_f64_dt(w[(int64_t)j * ldw + k], dtype);
+            if (bias) acc += ft2o_to_f64_dt(bias[j], dtype);
             if (y_f64) y_f64[(int64_t)m * ldy + j] = acc;
-            if (y_bf16) y_bf16[(int64_t)m * ldy + j] = ft2o_f64_to_bf16_rne(acc);
+            if (y_out) y_out[(int64_t)m * ldy + j] = ft2o_f64_to_dt_rne(acc, dtype);
         }
     }
+}
+EXPORT void ft2o_linear_f64(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
+                            const uint16_t* bias, int32_t M, int32_t N, int32_t K,
+                            double* y_f64, uint16_t* y_bf16, int64_t ldy) {
+    ft2o_linear_f64_dt(x, ldx, w, ldw, bias, M, N, K, y_f64, y_bf16, ldy, 0);
 }
 
 /* Full oracle layer (R8 then R7 then R5): linear -> bf16 -> inject -> check. */
@@ -363,6 +407,17 @@ EXPORT void ft2o_protected_linear(const uint16_t* x, int64_t ldx, const uint16_t
     ft2o_linear_f64(x, ldx, w, ldw, bias, M, N, K, 0, y, ldy);
     if (sites && n_sites > 0) ft2o_inject(y, M, N, ldy, sites, n_sites, cur_layer, cur_step, base_row);
     if (bounds) ft2o_protect(y, M, N, ldy, row_to_seq, bounds, num_seqs, count);
+}
+
+EXPORT void ft2o_protected_linear_dt(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
+                                     const uint16_t* bias, int32_t M, int32_t N, int32_t K,
+                                     uint16_t* y, int64_t ldy, const int32_t* row_to_seq,
+                                     const uint16_t* bounds, int32_t num_seqs, uint32_t* count,
+                                     const ft2o_site* sites, int32_t n_sites, int32_t cur_layer,
+                                     int32_t cur_step, const int32_t* base_row, int dtype) {
+    ft2o_linear_f64_dt(x, ldx, w, ldw, bias, M, N, K, 0, y, ldy, dtype);
+    if (sites && n_sites > 0) ft2o_inject(y, M, N, ldy, sites, n_sites, cur_layer, cur_step, base_row);
+    if (bounds) ft2o_protect_dt(y, M, N, ldy, row_to_seq, bounds, num_seqs, count, dtype);
 }
 
 EXPORT int32_t ft2o_site_size(void) { return (int32_t)sizeof(ft2o_site); }

@@ -63,7 +63,7 @@ def load(path: str = LIB):
         "ft2_bounds_finalize": (st, [P, i32, f32, ctypes.c_int, P, P]),
         "ft2_protect": (st, [Tensor, P, P, i32, P, P]),
         "ft2_gemm_workspace_bytes": (ctypes.c_size_t, [i32, i32, i32]),
-        "ft2_protect_fused_gemm": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, i32, i32,
+        "ft2_protect_fused_gemm": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, ctypes.c_int, i32, i32,
                                         P, P, i32, P, P, i32, i32, i32, P, P, ctypes.c_size_t, P]),
         "ft2_make_fault_sites": (st, [u64, u64, i32, ctypes.c_int, ctypes.c_int, ctypes.POINTER(SiteGeometry),
                                       P, P]),

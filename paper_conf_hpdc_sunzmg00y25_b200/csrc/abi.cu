@@ -33,7 +33,7 @@ static inline bool al16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
 static ft2_status check_tensor(const ft2_tensor& t, bool allow_null_if_empty = true) {
     if (t.rows < 0 || t.n < 0 || t.ld < t.n) return FT2_ERR_INVALID_ARG;
-    if (t.dtype != FT2_BF16) return FT2_ERR_UNSUPPORTED;
+    if (t.dtype != FT2_BF16 && t.dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
     if (t.rows == 0 || t.n == 0) return FT2_OK;
     if (t.data == nullptr) return FT2_ERR_INVALID_ARG;
     if (!al16(t.data) || (t.n % 8) != 0 || (t.ld % 8) != 0) return FT2_ERR_MISALIGNED;
@@ -93,6 +93,7 @@ ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int
     a.keys_out = keys_out;
     a.nonfinite_out = nonfinite_count;
     a.ws = static_cast<uint32_t*>(workspace);
+    a.dtype = y.dtype;
     int nl = 0;
     cudaError_t e = launch_bounds(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
@@ -102,9 +103,9 @@ ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scal
                                void* bounds_out, void* stream) {
     if (keys == nullptr || bounds_out == nullptr || num_seqs < 1) return FT2_ERR_INVALID_ARG;
     if (!(std::isfinite(scale)) || scale < 1.0f) return FT2_ERR_INVALID_ARG;
-    if (dtype != FT2_BF16) return FT2_ERR_UNSUPPORTED;
+    if (dtype != FT2_BF16 && dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
     int nl = 0;
-    cudaError_t e = launch_finalize(keys, num_seqs, scale, static_cast<uint16_t*>(bounds_out),
+    cudaError_t e = launch_finalize(keys, num_seqs, scale, static_cast<uint16_t*>(bounds_out), (int)dtype,
                                     static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
 }
@@ -127,6 +128,7 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
     a.S = num_seqs;
     a.bounds = static_cast<const uint16_t*>(bounds);
     a.counts = corrected_count;
+    a.dtype = y.dtype;
     int nl = 0;
     cudaError_t e = launch_protect(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
@@ -136,12 +138,13 @@ size_t ft2_gemm_workspace_bytes(int32_t M, int32_t N, int32_t K) { return gemm_w
 
 ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, const void* bias,
                                   void* y, int64_t ldy, int32_t M, int32_t N, int32_t K, ft2_gemm_mode mode,
-                                  int32_t col_begin, int32_t col_end, const int32_t* row_to_seq,
+                                  ft2_dtype dtype, int32_t col_begin, int32_t col_end, const int32_t* row_to_seq,
                                   const void* bounds, int32_t num_seqs, uint32_t* corrected_count,
                                   const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
                                   int32_t cur_step, const int32_t* base_row, void* workspace, size_t ws_bytes,
                                   void* stream) {
     if (M < 0 || N < 0 || K < 0) return FT2_ERR_INVALID_ARG;
+    if (dtype != FT2_BF16 && dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
     if (M == 0 || N == 0) return FT2_OK;
     if (K == 0) return FT2_ERR_UNSUPPORTED;
     if (x == nullptr || w == nullptr || y == nullptr) return FT2_ERR_INVALID_ARG;
@@ -187,6 +190,7 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
     a.ws = workspace;
     a.ws_bytes = ws_bytes;
     a.w_static = w_static;
+    a.dtype = dtype;
     int nl = 0;
     cudaError_t e = launch_gemm(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
@@ -214,7 +218,7 @@ ft2_status ft2_make_fault_sites(uint64_t seed, uint64_t trial0, int32_t n_trials
 ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
                              int32_t cur_step, const int32_t* base_row, void* stream) {
     if (y.rows < 0 || y.n < 0 || y.ld < y.n) return FT2_ERR_INVALID_ARG;
-    if (y.dtype != FT2_BF16) return FT2_ERR_UNSUPPORTED;
+    if (y.dtype != FT2_BF16 && y.dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
     if (n_sites < 0) return FT2_ERR_INVALID_ARG;
     if (n_sites == 0 || y.rows == 0 || y.n == 0) return FT2_OK;
     if (sites == nullptr || y.data == nullptr) return FT2_ERR_INVALID_ARG;

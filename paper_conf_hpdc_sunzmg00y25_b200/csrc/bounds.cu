@@ -77,6 +77,7 @@ __device__ __forceinline__ void record_patch(const BoundsK& p, uint32_t* list_co
 }
 
 // Slow exact path for one vector: min/max over finite keys, count the rest.
+template <int DT>
 __device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, uint32_t& kmin, uint32_t& kmax,
                                          uint32_t& nf, uint32_t* lc, uint32_t* ov, unsigned long long* list) {
     const uint4* q = vec_ptr(p, v);
@@ -86,7 +87,7 @@ __device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, ui
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
         uint16_t b = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
-        if ((b & 0x7F80) == 0x7F80) {
+        if (nonfinite1<DT>(b)) {
             nf++;
             if (p.correct) record_patch(p, lc, ov, list, s, base + j);
         } else {
@@ -97,6 +98,7 @@ __device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, ui
     }
 }
 
+template <int DT>
 __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
     __shared__ uint32_t sh_min[kThreads / 32], sh_max[kThreads / 32], sh_nf[kThreads / 32];
     __shared__ int sh_last;
@@ -147,12 +149,12 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
         uint32_t kmin = min(mn2 & 0xFFFFu, mn2 >> 16);
         uint32_t kmax = max(mx2 & 0xFFFFu, mx2 >> 16);
         uint32_t nf = 0;
-        if (kmin < 0x0080u || kmax > 0xFF7Fu) {
+        if (kmin < Fmt<DT>::kKeyLo || kmax > Fmt<DT>::kKeyHi) {
             // this thread saw a non-finite value: redo its vectors exactly
             kmin = 0xFFFFu;
             kmax = 0u;
             for (uint32_t vi = v + tid; vi < seg_end; vi += kThreads)
-                slow_vec(p, vi, s, kmin, kmax, nf, ws_lc, ws_ov, list);
+                slow_vec<DT>(p, vi, s, kmin, kmax, nf, ws_lc, ws_ov, list);
         }
         kmin = __reduce_min_sync(0xFFFFFFFFu, kmin);
         kmax = __reduce_max_sync(0xFFFFFFFFu, kmax);
@@ -190,8 +192,8 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
         if (p.finalize) {
             uint16_t lo = 0, hi = 0;  // reading A9
             if (have) {
-                lo = scale_bound(unkey1((uint16_t)kmin), p.scale, false);
-                hi = scale_bound(unkey1((uint16_t)kmax), p.scale, true);
+                lo = scale_bound<DT>(unkey1((uint16_t)kmin), p.scale, false);
+                hi = scale_bound<DT>(unkey1((uint16_t)kmax), p.scale, true);
             }
             p.bounds_out[2 * s] = lo;
             p.bounds_out[2 * s + 1] = hi;
@@ -218,7 +220,7 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
                 uint16_t b = p.y[off];
                 uint16_t lo = p.bounds_out[2 * s], hi = p.bounds_out[2 * s + 1];
                 // R5 on a non-finite value: NaN -> clamp(+0), +Inf -> hi, -Inf -> lo
-                uint16_t x = ((b & 0x7FFF) > 0x7F80) ? (uint16_t)0 : b;
+                uint16_t x = isnan1<DT>(b) ? (uint16_t)0 : b;
                 uint16_t k = key1(x);
                 p.y[off] = k < key1(lo) ? lo : (k > key1(hi) ? hi : x);
             }
@@ -236,8 +238,8 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
                 uint16_t lo = p.bounds_out[2 * s], hi = p.bounds_out[2 * s + 1];
                 for (int j = 0; j < 8; ++j) {
                     uint16_t b = q[j];
-                    if ((b & 0x7F80) != 0x7F80) continue;
-                    uint16_t x = ((b & 0x7FFF) > 0x7F80) ? (uint16_t)0 : b;
+                    if (!nonfinite1<DT>(b)) continue;
+                    uint16_t x = isnan1<DT>(b) ? (uint16_t)0 : b;
                     uint16_t k = key1(x);
                     q[j] = k < key1(lo) ? lo : (k > key1(hi) ? hi : x);
                 }
@@ -257,14 +259,15 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
     }
 }
 
+template <int DT>
 __global__ void finalize_kernel(const int32_t* keys, int32_t S, float scale, uint16_t* out) {
     int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S) return;
     int32_t a = keys[2 * s], b = keys[2 * s + 1];
     uint16_t lo = 0, hi = 0;
     if (a >= 0 && b >= 0) {
-        lo = scale_bound(unkey1((uint16_t)(0xFFFF - a)), scale, false);
-        hi = scale_bound(unkey1((uint16_t)b), scale, true);
+        lo = scale_bound<DT>(unkey1((uint16_t)(0xFFFF - a)), scale, false);
+        hi = scale_bound<DT>(unkey1((uint16_t)b), scale, true);
     }
     out[2 * s] = lo;
     out[2 * s + 1] = hi;
@@ -273,6 +276,7 @@ __global__ void finalize_kernel(const int32_t* keys, int32_t S, float scale, uin
 static int g_blocks_per_sm = 0;
 
 cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
+    auto kern = a.dtype == FT2_FP16 ? bounds_kernel<1> : bounds_kernel<0>;
     BoundsK p;
     p.y = a.y;
     p.ld = a.ld;
@@ -291,7 +295,7 @@ cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
     p.ws = a.ws;
     if (g_blocks_per_sm == 0) {
         int b = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel, kThreads, 0);
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel<0>, kThreads, 0);
         if (e != cudaSuccess) return e;
         g_blocks_per_sm = b > 0 ? b : 1;
     }
@@ -302,14 +306,15 @@ cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
     p.chunk = (p.total_vec + grid - 1) / grid;
     grid = (p.total_vec + p.chunk - 1) / p.chunk;
     if (grid < 1) grid = 1;
-    bounds_kernel<<<grid, kThreads, 0, st>>>(p);
+    kern<<<grid, kThreads, 0, st>>>(p);
     ++*n_launch;
     return cudaGetLastError();
 }
 
-cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out, cudaStream_t st,
+cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out, int dtype, cudaStream_t st,
                             int* n_launch) {
-    finalize_kernel<<<(S + 127) / 128, 128, 0, st>>>(keys, S, scale, out);
+    if (dtype == FT2_FP16) finalize_kernel<1><<<(S + 127) / 128, 128, 0, st>>>(keys, S, scale, out);
+    else finalize_kernel<0><<<(S + 127) / 128, 128, 0, st>>>(keys, S, scale, out);
     ++*n_launch;
     return cudaGetLastError();
 }

@@ -9,6 +9,7 @@
 // min/max), which makes every result bit-exact and independent of reduction
 // order.
 #pragma once
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -42,15 +43,40 @@ __device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
     return d;
 }
 
-// Bit 15 of each half set iff that bf16 half is NaN: (h & 0x7FFF) >= 0x7F81.
+// 16-bit activation formats: DT 0 = bf16 (1/8/7), DT 1 = fp16 (1/5/10, the
+// paper's precision).  Both are sign-magnitude, so the order
+// key is the same; only the exponent field (and so NaN/Inf) differs.
+template <int DT> struct Fmt;
+template <> struct Fmt<0> {
+    static constexpr uint32_t kExp = 0x7F80u;     // exponent field = +Inf pattern
+    static constexpr uint32_t kMaxFin = 0x7F7Fu;  // largest finite magnitude
+    static constexpr uint32_t kKeyLo = 0x0080u;   // key(-max finite)
+    static constexpr uint32_t kKeyHi = 0xFF7Fu;   // key(+max finite)
+};
+template <> struct Fmt<1> {
+    static constexpr uint32_t kExp = 0x7C00u;
+    static constexpr uint32_t kMaxFin = 0x7BFFu;
+    static constexpr uint32_t kKeyLo = 0x0400u;
+    static constexpr uint32_t kKeyHi = 0xFBFFu;
+};
+
+// Bit 15 of each half set iff that half is NaN: (h & 0x7FFF) > kExp.
+template <int DT = 0>
 __device__ __forceinline__ uint32_t nan_bits2(uint32_t w) {
-    return ((w & 0x7FFF7FFFu) + 0x007F007Fu) & 0x80008000u;
+    constexpr uint32_t add = (0x7FFFu - Fmt<DT>::kExp) * 0x10001u;
+    return ((w & 0x7FFF7FFFu) + add) & 0x80008000u;
 }
 
 // Bit 15 of each half set iff that half is non-finite (exponent all ones).
+template <int DT = 0>
 __device__ __forceinline__ uint32_t nonfinite_bits2(uint32_t w) {
-    return ((w & 0x7F807F80u) + 0x00800080u) & 0x80008000u;
+    constexpr uint32_t e = Fmt<DT>::kExp * 0x10001u, one = (0x8000u - Fmt<DT>::kExp) * 0x10001u;
+    return ((w & e) + one) & 0x80008000u;
 }
+template <int DT = 0>
+__device__ __forceinline__ bool isnan1(uint16_t b) { return (b & 0x7FFFu) > Fmt<DT>::kExp; }
+template <int DT = 0>
+__device__ __forceinline__ bool nonfinite1(uint16_t b) { return (b & Fmt<DT>::kExp) == Fmt<DT>::kExp; }
 
 // Number of 16-bit halves of d that are non-zero (0, 1 or 2).
 __device__ __forceinline__ uint32_t nonzero_halves(uint32_t d) {
@@ -67,9 +93,10 @@ __device__ __forceinline__ uint16_t unkey1(uint16_t k) {
 // Check-and-clip of two packed bf16 against packed keys (kL2 = kL|kL<<16 ...).
 // NaN halves are first replaced by +0 (key 0x8000), then clamped in key space.
 // Returns the corrected packed bf16; *changed = number of halves whose bits changed.
+template <int DT = 0>
 __device__ __forceinline__ uint32_t clip2(uint32_t w, uint32_t kL2, uint32_t kH2, uint32_t* changed) {
     uint32_t k = key2(w);
-    uint32_t nm = half_sign_mask(nan_bits2(w));           // 0xFFFF on NaN halves
+    uint32_t nm = half_sign_mask(nan_bits2<DT>(w));       // 0xFFFF on NaN halves
     uint32_t kz = (k & ~nm) | (0x80008000u & nm);          // NaN -> key(+0)
     uint32_t kc = vmax_u16x2(vmin_u16x2(kz, kH2), kL2);
     *changed = nonzero_halves(kc ^ k);
@@ -91,14 +118,23 @@ __device__ __forceinline__ uint16_t bf16_from_f32_dir(float s, bool up) {
     return (uint16_t)t;
 }
 
+template <int DT = 0>
+__device__ __forceinline__ float to_f32(uint16_t b) {
+    if (DT == 0) return __uint_as_float((uint32_t)b << 16);
+    return __half2float(__ushort_as_half(b));
+}
+
+template <int DT = 0>
 __device__ __forceinline__ uint16_t scale_bound(uint16_t raw, float c, bool is_hi) {
-    float x = __uint_as_float((uint32_t)raw << 16);
+    const float x = to_f32<DT>(raw);
     float s;
     if (is_hi) s = (x >= 0.0f) ? __fmul_rn(x, c) : __fdiv_rn(x, c);
     else       s = (x <= 0.0f) ? __fmul_rn(x, c) : __fdiv_rn(x, c);
-    uint16_t r = bf16_from_f32_dir(s, is_hi);
-    if (r == 0x7F80) r = 0x7F7F;
-    if (r == 0xFF80) r = 0xFF7F;
+    uint16_t r;
+    if (DT == 0) r = bf16_from_f32_dir(s, is_hi);
+    else r = __half_as_ushort(is_hi ? __float2half_ru(s) : __float2half_rd(s));
+    if (r == Fmt<DT>::kExp) r = (uint16_t)Fmt<DT>::kMaxFin;
+    if (r == (0x8000u | Fmt<DT>::kExp)) r = (uint16_t)(0x8000u | Fmt<DT>::kMaxFin);
     return r;
 }
 
@@ -108,6 +144,12 @@ __device__ __forceinline__ uint16_t bf16_rne(float f) {
     if ((u & 0x7FFFFFFFu) > 0x7F800000u) return 0x7FC0;
     u += 0x7FFFu + ((u >> 16) & 1u);
     return (uint16_t)(u >> 16);
+}
+// fp32 -> activation format, round-to-nearest-even.
+template <int DT = 0>
+__device__ __forceinline__ uint16_t rne16(float f) {
+    if (DT == 0) return bf16_rne(f);
+    return __half_as_ushort(__float2half_rn(f));
 }
 
 // ------------------------------------------------------------------ Philox

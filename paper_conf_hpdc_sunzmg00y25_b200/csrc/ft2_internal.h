@@ -28,9 +28,10 @@ struct BoundsArgs {
     int32_t* keys_out;
     uint32_t* nonfinite_out;
     uint32_t* ws;
+    int32_t dtype;  // FT2_BF16 or FT2_FP16
 };
 cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch);
-cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out,
+cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out, int dtype,
                             cudaStream_t st, int* n_launch);
 
 struct ProtectArgs {
@@ -40,6 +41,7 @@ struct ProtectArgs {
     int32_t S;
     const uint16_t* bounds;
     uint32_t* counts;
+    int32_t dtype;
 };
 cudaError_t launch_protect(const ProtectArgs& a, cudaStream_t st, int* n_launch);
 
@@ -67,6 +69,7 @@ struct GemmArgs {
     const int32_t* base_row;
     void* ws; size_t ws_bytes;
     int32_t w_static;
+    int32_t dtype;
 };
 size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch);

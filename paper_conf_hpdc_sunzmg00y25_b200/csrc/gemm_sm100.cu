@@ -102,11 +102,12 @@ struct TabE {
     uint32_t flags;
 };
 
+template <int DT>
 __device__ __forceinline__ TabE feature_entry(const GemmK& p, int n) {
     TabE e{0.f, 0u, -1, 0u};
     if (n < p.N) {
         e.flags = 1u;
-        if (p.bias) e.bias = __uint_as_float((uint32_t)p.bias[n] << 16);
+        if (p.bias) e.bias = to_f32<DT>(p.bias[n]);
         if (p.mode == FT2_GEMM_CHECK && n >= p.col_begin && n < p.col_end) e.flags |= 2u;
     }
     return e;
@@ -163,15 +164,16 @@ __device__ __noinline__ uint2 xor_sites(uint2 w, uint32_t le0, const uint32_t* s
 }
 
 // Check-and-clip of two packed bf16 (R5): NaN -> key(+0), clamp in key space.
+template <int DT>
 __device__ __forceinline__ uint32_t clip2_nocount(uint32_t w, uint32_t kL2, uint32_t kH2) {
     const uint32_t k = key2(w);
-    const uint32_t nm = half_sign_mask(nan_bits2(w));
+    const uint32_t nm = half_sign_mask(nan_bits2<DT>(w));
     const uint32_t kz = (k & ~nm) | (0x80008000u & nm);
     return unkey2(vmax_u16x2(vmin_u16x2(kz, kH2), kL2));
 }
 
 // Finish four consecutive columns c0..c0+3 of tile row la.
-template <bool SWAP>
+template <bool SWAP, int DT>
 __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, int ga, int gb0, const TabE& re,
                                         const TabE* __restrict__ ce, uint32_t le0, float4 acc,
                                         const uint32_t* site_e, const uint32_t* site_m, uint32_t nsite,
@@ -179,8 +181,8 @@ __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, i
     // feature side: SWAP ? the row : the column; token side: the other one
     const float b0 = SWAP ? re.bias : ce[0].bias, b1 = SWAP ? re.bias : ce[1].bias;
     const float b2 = SWAP ? re.bias : ce[2].bias, b3 = SWAP ? re.bias : ce[3].bias;
-    uint2 w = make_uint2((uint32_t)bf16_rne(acc.x + b0) | ((uint32_t)bf16_rne(acc.y + b1) << 16),
-                         (uint32_t)bf16_rne(acc.z + b2) | ((uint32_t)bf16_rne(acc.w + b3) << 16));
+    uint2 w = make_uint2((uint32_t)rne16<DT>(acc.x + b0) | ((uint32_t)rne16<DT>(acc.y + b1) << 16),
+                         (uint32_t)rne16<DT>(acc.z + b2) | ((uint32_t)rne16<DT>(acc.w + b3) << 16));
     if (nsite) w = xor_sites(w, le0, site_e, site_m, nsite);
     uint32_t f[4], kL01, kH01, kL23, kH23;
 #pragma unroll
@@ -196,8 +198,8 @@ __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, i
     }
     const uint32_t m01 = ((f[0] & 2u) ? 0x0000FFFFu : 0u) | ((f[1] & 2u) ? 0xFFFF0000u : 0u);
     const uint32_t m23 = ((f[2] & 2u) ? 0x0000FFFFu : 0u) | ((f[3] & 2u) ? 0xFFFF0000u : 0u);
-    const uint32_t o01 = (clip2_nocount(w.x, kL01, kH01) & m01) | (w.x & ~m01);
-    const uint32_t o23 = (clip2_nocount(w.y, kL23, kH23) & m23) | (w.y & ~m23);
+    const uint32_t o01 = (clip2_nocount<DT>(w.x, kL01, kH01) & m01) | (w.x & ~m01);
+    const uint32_t o23 = (clip2_nocount<DT>(w.y, kL23, kH23) & m23) | (w.y & ~m23);
     const uint32_t d01 = o01 ^ w.x, d23 = o23 ^ w.y;
     const uint16_t o[4] = {(uint16_t)o01, (uint16_t)(o01 >> 16), (uint16_t)o23, (uint16_t)(o23 >> 16)};
     if (SWAP) {
@@ -223,7 +225,7 @@ __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, i
     }
 }
 
-template <int BN, bool SWAP>
+template <int BN, bool SWAP, int DT>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
                 const __grid_constant__ GemmK p) {
@@ -311,7 +313,9 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     } else if (warp == 1) {
         if (lane == 0) {
             // ------------------------------------------------ MMA issuer
-            constexpr uint32_t idesc = make_idesc(kBlockA, BN);
+            // kind::f16 operand format: 0 = F16, 1 = BF16 (bits 7-9 A, 10-12 B)
+            constexpr uint32_t idesc =
+                (make_idesc(kBlockA, BN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
             for (int i = 0; i < nk; ++i) {
                 const int s = i % STAGES;
                 mbar_wait(&full[s], (uint32_t)(i / STAGES) & 1u);
@@ -334,10 +338,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const int a = q * 32 + lane;
         griddep_wait();  // bias/bounds/sites/y may belong to the previous kernel
         // epilogue tables, gathered while the main loop still streams
-        row_tab[a] = SWAP ? feature_entry(p, tileA * kBlockA + a) : token_entry(p, tileA * kBlockA + a);
+        row_tab[a] = SWAP ? feature_entry<DT>(p, tileA * kBlockA + a) : token_entry(p, tileA * kBlockA + a);
         row_cnt[a] = 0u;
         for (int c = a; c < BN; c += 128) {
-            col_tab[c] = SWAP ? token_entry(p, tileB * BN + c) : feature_entry(p, tileB * BN + c);
+            col_tab[c] = SWAP ? token_entry(p, tileB * BN + c) : feature_entry<DT>(p, tileB * BN + c);
             col_cnt[c] = 0u;
         }
         if (p.sites != nullptr) {  // fault sites landing in my slice
@@ -416,7 +420,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
             for (int rr = 1; rr < kMaxSplitK; ++rr)
                 if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
-            finish4<SWAP>(y, ldy, tileA * kBlockA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
+            finish4<SWAP, DT>(y, ldy, tileA * kBlockA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
                           (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4);
         }
     }
@@ -449,29 +453,30 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     return fn;
 }
 
-static bool make_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int64_t ld, int box_rows) {
+static bool make_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int64_t ld, int box_rows,
+                     int dtype) {
     auto enc = get_encode();
     if (!enc) return false;
     cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
     cuuint64_t strides[1] = {(cuuint64_t)(ld * 2)};
     cuuint32_t box[2] = {(cuuint32_t)kBlockK, (cuuint32_t)box_rows};
     cuuint32_t es[2] = {1, 1};
-    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+    CUresult r = enc(m, dtype == FT2_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
 
-template <int BN, bool SWAP>
+template <int BN, bool SWAP, int DT>
 static cudaError_t set_attrs() {
     static cudaError_t res = [] {
-        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              Cfg<BN>::kBytes);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
         // full shared-memory carveout so two ~105 KB decode CTAs share an SM
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP>, cudaFuncAttributePreferredSharedMemoryCarveout,
+            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT>, cudaFuncAttributePreferredSharedMemoryCarveout,
                                      (int)cudaSharedmemCarveoutMaxShared);
         return e;
     }();
@@ -479,12 +484,12 @@ static cudaError_t set_attrs() {
 }
 
 // How many (1, sk, 1) clusters of this instantiation can be resident at once.
-template <int BN, bool SWAP>
+template <int BN, bool SWAP, int DT = 0>
 static int max_clusters(int sk) {
     static int cache[kMaxSplitK + 1] = {0};
     if (sk < 1 || sk > kMaxSplitK) return -1;
     if (cache[sk] != 0) return cache[sk];
-    if (set_attrs<BN, SWAP>() != cudaSuccess) return cache[sk] = -1;
+    if (set_attrs<BN, SWAP, DT>() != cudaSuccess) return cache[sk] = -1;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(1, (unsigned)sk, 1);
     cfg.blockDim = dim3(kGemmThreads);
@@ -497,7 +502,7 @@ static int max_clusters(int sk) {
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     int n = 0;
-    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BN, SWAP>, &cfg) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BN, SWAP, DT>, &cfg) != cudaSuccess) {
         cudaGetLastError();
         n = -1;
     }
@@ -532,10 +537,13 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     // so that every SM streams weights.  Measured on B200 (tools/
     // sweep_splitk.sh, profiles/): the best split is the largest one with
     // tiles * splitk <= 2 * SMs (two ~105 KB CTAs fit an SM), >= 4 k-blocks of
-    // 64 per CTA, and a cluster of at most 12 CTAs.
+    // 64 per CTA, and a cluster of at most 8 CTAs (12 when <= 16 tiles).
     int best = 1;
+    // clusters above the portable size 8 only pay off when few (<= 16) of
+    // them are needed (measured: 16 tiles x 12 beats x 8; 32 tiles x 9 loses to x 8)
+    const int sk_cap = tiles <= 16 ? kMaxSplitPlanned : 8;
     if (g.swap) {
-        for (int sk = 2; sk <= kMaxSplitPlanned; ++sk) {
+        for (int sk = 2; sk <= sk_cap; ++sk) {
             if (tiles * sk > 2 * sms || g.nkb < 4 * sk) break;
             if (max_clusters_bn(g.bn, sk) < 1) break;
             best = sk;
@@ -556,14 +564,14 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
         for (int sk = 2; sk <= 8 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
         int occ = -1;
         if (g.bn == 32) {
-            set_attrs<32, true>();
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gemm_kernel<32, true>, kGemmThreads, Cfg<32>::kBytes);
+            set_attrs<32, true, 0>();
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gemm_kernel<32, true, 0>, kGemmThreads, Cfg<32>::kBytes);
         }
         size_t avail2 = 0, avail1 = 0;
-        cudaOccupancyAvailableDynamicSMemPerBlock(&avail2, gemm_kernel<32, true>, 2, kGemmThreads);
-        cudaOccupancyAvailableDynamicSMemPerBlock(&avail1, gemm_kernel<32, true>, 1, kGemmThreads);
+        cudaOccupancyAvailableDynamicSMemPerBlock(&avail2, gemm_kernel<32, true, 0>, 2, kGemmThreads);
+        cudaOccupancyAvailableDynamicSMemPerBlock(&avail1, gemm_kernel<32, true, 0>, 1, kGemmThreads);
         cudaFuncAttributes fa;
-        cudaFuncGetAttributes(&fa, gemm_kernel<32, true>);
+        cudaFuncGetAttributes(&fa, gemm_kernel<32, true, 0>);
         int smem_sm = 0, dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
@@ -577,15 +585,15 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
 // The cluster split-K needs no global workspace.
 size_t gemm_ws_bytes(int32_t, int32_t, int32_t) { return 0; }
 
-template <int BN, bool SWAP>
+template <int BN, bool SWAP, int DT>
 static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st, int* n_launch) {
     CUtensorMap ma, mb;
     const void* pa = SWAP ? (const void*)a.w : (const void*)a.x;
     const void* pb = SWAP ? (const void*)a.x : (const void*)a.w;
     const int64_t lda = SWAP ? a.ldw : a.ldx, ldb = SWAP ? a.ldx : a.ldw;
-    if (!make_map(&ma, pa, p.rowsA, a.K, lda, kBlockA)) return cudaErrorInvalidValue;
-    if (!make_map(&mb, pb, p.rowsB, a.K, ldb, BN)) return cudaErrorInvalidValue;
-    cudaError_t e = set_attrs<BN, SWAP>();
+    if (!make_map(&ma, pa, p.rowsA, a.K, lda, kBlockA, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
+    if (!make_map(&mb, pb, p.rowsB, a.K, ldb, BN, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
+    cudaError_t e = set_attrs<BN, SWAP, DT>();
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);
@@ -601,7 +609,7 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     attr[1].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = p.splitk > 1 ? 2 : 1;
-    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP>, ma, mb, p);
+    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP, DT>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -635,12 +643,21 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cur_step = a.cur_step;
     p.base_row = a.base_row;
     p.w_static = a.w_static;
-    if (!g.swap) return launch_cfg<128, false>(a, p, st, n_launch);
+    if (a.dtype == FT2_FP16) {
+        if (!g.swap) return launch_cfg<128, false, 1>(a, p, st, n_launch);
+        switch (g.bn) {
+            case 16: return launch_cfg<16, true, 1>(a, p, st, n_launch);
+            case 32: return launch_cfg<32, true, 1>(a, p, st, n_launch);
+            case 64: return launch_cfg<64, true, 1>(a, p, st, n_launch);
+            default: return launch_cfg<128, true, 1>(a, p, st, n_launch);
+        }
+    }
+    if (!g.swap) return launch_cfg<128, false, 0>(a, p, st, n_launch);
     switch (g.bn) {
-        case 16: return launch_cfg<16, true>(a, p, st, n_launch);
-        case 32: return launch_cfg<32, true>(a, p, st, n_launch);
-        case 64: return launch_cfg<64, true>(a, p, st, n_launch);
-        default: return launch_cfg<128, true>(a, p, st, n_launch);
+        case 16: return launch_cfg<16, true, 0>(a, p, st, n_launch);
+        case 32: return launch_cfg<32, true, 0>(a, p, st, n_launch);
+        case 64: return launch_cfg<64, true, 0>(a, p, st, n_launch);
+        default: return launch_cfg<128, true, 0>(a, p, st, n_launch);
     }
 }
 

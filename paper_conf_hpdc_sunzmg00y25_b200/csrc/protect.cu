@@ -53,6 +53,7 @@ __device__ __forceinline__ void load_bounds2(const ProtectK& p, int s, uint32_t&
     kH2 = kh | (kh << 16);
 }
 
+template <int DT>
 __global__ void __launch_bounds__(kPThreads) protect_kernel(ProtectK p) {
     uint32_t kL2 = 0, kH2 = 0;
     if (p.row_mode == 2) load_bounds2(p, 0, kL2, kH2);
@@ -87,7 +88,7 @@ __global__ void __launch_bounds__(kPThreads) protect_kernel(ProtectK p) {
             if (diff) {  // rare: exact correction of this vector
                 uint32_t cnt = 0, c;
 #pragma unroll
-                for (int j = 0; j < 4; ++j) { w[j] = clip2(w[j], kL2, kH2, &c); cnt += c; }
+                for (int j = 0; j < 4; ++j) { w[j] = clip2<DT>(w[j], kL2, kH2, &c); cnt += c; }
                 *q[u] = make_uint4(w[0], w[1], w[2], w[3]);
                 if (p.counts) atomicAdd(&p.counts[s], cnt);
             }
@@ -112,7 +113,7 @@ cudaError_t launch_protect(const ProtectArgs& a, cudaStream_t st, int* n_launch)
     p.counts = a.counts;
     if (g_pblocks_per_sm == 0) {
         int b = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, protect_kernel, kPThreads, 0);
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, protect_kernel<0>, kPThreads, 0);
         if (e != cudaSuccess) return e;
         g_pblocks_per_sm = b > 0 ? b : 1;
     }
@@ -120,7 +121,8 @@ cudaError_t launch_protect(const ProtectArgs& a, cudaStream_t st, int* n_launch)
     uint32_t want = (p.total_vec + per_cta - 1) / per_cta;
     uint32_t max_grid = (uint32_t)(num_sms() * g_pblocks_per_sm);
     uint32_t grid = want > max_grid ? max_grid : (want < 1 ? 1 : want);
-    protect_kernel<<<grid, kPThreads, 0, st>>>(p);
+    if (a.dtype == FT2_FP16) protect_kernel<1><<<grid, kPThreads, 0, st>>>(p);
+    else protect_kernel<0><<<grid, kPThreads, 0, st>>>(p);
     ++*n_launch;
     return cudaGetLastError();
 }

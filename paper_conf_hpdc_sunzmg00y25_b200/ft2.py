@@ -10,8 +10,16 @@ import ctypes
 import torch
 
 from . import _lib
-from ._lib import (FT2_BF16, FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FaultSite, SiteGeometry, Tensor, check,
+from ._lib import (FT2_BF16, FT2_FP16, FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FaultSite, SiteGeometry, Tensor, check,
                    load)
+
+_DTYPES = {torch.bfloat16: FT2_BF16, torch.float16: FT2_FP16}
+
+
+def _dtype_of(t: torch.Tensor) -> int:
+    if t.dtype not in _DTYPES:
+        raise TypeError(f"ft2: unsupported activation dtype {t.dtype} (bfloat16 / float16)")
+    return _DTYPES[t.dtype]
 
 SITE_BYTES = ctypes.sizeof(FaultSite)
 
@@ -26,8 +34,7 @@ def _ptr(t):
 
 
 def _as_ft2_tensor(y: torch.Tensor) -> Tensor:
-    if y.dtype != torch.bfloat16:
-        raise TypeError("ft2: only bfloat16 activations are implemented")
+    dt = _dtype_of(y)
     if not y.is_cuda:
         raise ValueError("ft2: tensor must live on a CUDA device (no CPU fallback)")
     if y.dim() == 1:
@@ -39,7 +46,7 @@ def _as_ft2_tensor(y: torch.Tensor) -> Tensor:
         y = y2
     if y.stride(1) != 1:
         raise ValueError("ft2: rows must be contiguous (stride(-1) == 1)")
-    return Tensor(y.data_ptr(), y.shape[0], y.shape[1], y.stride(0), FT2_BF16)
+    return Tensor(y.data_ptr(), y.shape[0], y.shape[1], y.stride(0), dt)
 
 
 def workspace_bytes(num_seqs: int) -> int:
@@ -66,7 +73,7 @@ def bounds_from_prefill(y, bounds_out, workspace, seq_offsets=None, num_seqs=Non
 
 def bounds_finalize(keys, bounds_out, scale=2.0, stream=None):
     S = keys.numel() // 2
-    check("ft2_bounds_finalize", load().ft2_bounds_finalize(_ptr(keys), S, float(scale), FT2_BF16,
+    check("ft2_bounds_finalize", load().ft2_bounds_finalize(_ptr(keys), S, float(scale), _dtype_of(bounds_out),
                                                             _ptr(bounds_out), _stream(stream)))
 
 
@@ -92,7 +99,7 @@ def protect_fused_gemm(x, w, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None, row
         workspace = default_gemm_workspace(x.device)
     ws = workspace.numel() * workspace.element_size()
     st = load().ft2_protect_fused_gemm(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y), y.stride(0),
-                                       M, N, K, int(mode), col_begin, col_end, _ptr(row_to_seq), _ptr(bounds), S,
+                                       M, N, K, int(mode), _dtype_of(x), col_begin, col_end, _ptr(row_to_seq), _ptr(bounds), S,
                                        _ptr(corrected_count), _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),
                                        _ptr(workspace), ws, _stream(stream))
     check("ft2_protect_fused_gemm", st)
@@ -119,13 +126,13 @@ def gemm_workspace_bytes(M, N, K) -> int:
 
 
 def make_fault_sites(seed, trial0, n_trials, model, layer_width, n_steps, prompt_len, out=None,
-                     layer_uniform=True, step_policy=0, device=None, stream=None):
+                     layer_uniform=True, step_policy=0, device=None, stream=None, dtype=FT2_BF16):
     """ft2_make_fault_sites -> uint8 tensor [n_trials * 24] (ft2_fault_site records)."""
     widths = (ctypes.c_int32 * len(layer_width))(*[int(v) for v in layer_width])
     g = SiteGeometry(n_steps, prompt_len, len(layer_width), widths, int(layer_uniform), int(step_policy))
     if out is None:
         out = torch.empty(n_trials * SITE_BYTES, dtype=torch.uint8, device=device or "cuda")
-    st = load().ft2_make_fault_sites(seed, trial0, n_trials, model, FT2_BF16, ctypes.byref(g), _ptr(out),
+    st = load().ft2_make_fault_sites(seed, trial0, n_trials, model, dtype, ctypes.byref(g), _ptr(out),
                                      _stream(stream))
     check("ft2_make_fault_sites", st)
     return out

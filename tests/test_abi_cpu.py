@@ -58,8 +58,10 @@ def test_validation_without_gpu(L):
     # misaligned base, n % 8
     assert L.ft2_protect(Tensor(0x1002, 4, 16, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
     assert L.ft2_protect(Tensor(0x1000, 4, 12, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
-    # dtype not implemented
-    assert L.ft2_protect(Tensor(0x1000, 4, 16, 16, 1), None, P(0x2000), 1, None, None) == FT2_ERR_UNSUPPORTED
+    # dtype not implemented (FP32); FP16 passes validation
+    assert L.ft2_protect(Tensor(0x1000, 4, 16, 16, 2), None, P(0x2000), 1, None, None) == FT2_ERR_UNSUPPORTED
+    assert L.ft2_protect_fused_gemm(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, 4, 16, 16, 0, 2, 0, 16,
+                                    None, None, 0, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_UNSUPPORTED
     # zero-size -> OK with no launch
     n0 = L.ft2_launch_count()
     assert L.ft2_protect(Tensor(0x1000, 0, 16, 16, 0), None, P(0x2000), 1, None, None) == FT2_OK
@@ -78,8 +80,8 @@ def test_validation_without_gpu(L):
     assert bfp(2.0, fin=0, cor=1, k=P(0x5000)) == FT2_ERR_INVALID_ARG
     assert bfp(2.0, S=2) == FT2_ERR_INVALID_ARG       # several sequences need seq_offsets
     # fused gemm: misaligned K
-    assert L.ft2_protect_fused_gemm(P(0x1000), 12, P(0x2000), 12, None, P(0x3000), 16, 4, 16, 12, 0, 0, 16,
+    assert L.ft2_protect_fused_gemm(P(0x1000), 12, P(0x2000), 12, None, P(0x3000), 16, 4, 16, 12, 0, 0, 0, 16,
                                     None, None, 0, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_MISALIGNED
     # fused gemm CHECK without bounds
-    assert L.ft2_protect_fused_gemm(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, 4, 16, 16, 1, 0, 16,
+    assert L.ft2_protect_fused_gemm(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, 4, 16, 16, 1, 0, 0, 16,
                                     None, None, 1, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_INVALID_ARG
