@@ -395,6 +395,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     }
     // ---------------------------------------------- finish the slice (all warps)
     named_bar(2, kGemmThreads);  // tables, site list and my own rows are in shared memory
+    if (splitk > 1 && warp < 2) cluster_wait();  // pair the prologue arrive of the non-epilogue warps
     griddep_wait();              // (no-op for threads that already waited)
     if (splitk > 1) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
     if (tid == 64) FT2_TRACE(6);

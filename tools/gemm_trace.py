@@ -23,8 +23,15 @@ for M, N, K in shapes:
     y = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
     bnd = torch.tensor([[-1e30, 1e30]], dtype=torch.bfloat16, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    nflush = int(os.environ.get("NOFLUSH", "0")) == 0
+    big = [ft2_synth.gen_bf16_torch((N, K), 40 + i, 1, scale_log2=-6, device="cuda") for i in range(4)] if not nflush else []
+    it = [0]
     def step():
-        flush.zero_()                # evict W from L2 (as a 2.6 GB weight stream would)
+        if nflush:
+            flush.zero_()            # evict W from L2 (as a 2.6 GB weight stream would)
+        else:                        # stream other weights through L2 with a read-only GEMM (no dirty lines)
+            torch.matmul(x0[:, :64], big[it[0] % 4][:, :64].t())
+            it[0] += 1
         x = torch.relu(x0)           # the preceding torch kernel
         ft2.protect_fused_gemm(x, w, y, mode=1 | 16, bounds=bnd, num_seqs=1)
     for _ in range(3): step()
