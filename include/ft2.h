@@ -147,6 +147,11 @@ size_t ft2_workspace_bytes(int32_t num_seqs);
  *              keys_out[2s+1] = key(hi_raw), -1 where the sequence has no finite
  *              value; element-wise MAX of these over shards gives the keys of
  *              the unsharded tensor (min/max are exact and associative).
+ * nan_vulnerable_count  NULL or uint32 [num_seqs]: WRITTEN with the number of
+ *              NaN-vulnerable values, those in (-2,-1) U (1,2) whose exponent-MSB
+ *              flip gives NaN (Fig. 7; L202 reports their share per
+ *              layer; L212: the alternative criticality proxy).  Computed in the
+ *              same sweep; when NULL the sweep does not count them.
  * nonfinite_count  NULL or uint32 [num_seqs]: WRITTEN with the number of
  *              non-finite elements of each sequence.
  * workspace    ft2_workspace_bytes(num_seqs) bytes, see above.
@@ -154,7 +159,7 @@ size_t ft2_workspace_bytes(int32_t num_seqs);
 ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int32_t num_seqs,
                                    float scale, int32_t finalize, int32_t correct_nonfinite,
                                    void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
-                                   void* workspace, void* stream);
+                                   uint32_t* nan_vulnerable_count, void* workspace, void* stream);
 
 /* Bounds from (all-reduced) keys in the ft2_bounds_from_prefill keys_out
  * encoding: the second half of the tensor-parallel path. */

@@ -74,6 +74,7 @@ def lib():
             ("ft2o_protected_linear", None, [P, i64, P, i64, P, i32, i32, i32, P, i64, P, P, i32, P,
                                              P, i32, i32, i32, P]),
             ("ft2o_site_size", i32, []),
+            ("ft2o_nan_vulnerable_count", None, [P, i64, i64, i64, P, i32, P, ctypes.c_int]),
             ("ft2o_isnan_dt", ctypes.c_int, [u16, ctypes.c_int]), ("ft2o_isinf_dt", ctypes.c_int, [u16, ctypes.c_int]),
             ("ft2o_isfinite_dt", ctypes.c_int, [u16, ctypes.c_int]),
             ("ft2o_to_f64_dt", ctypes.c_double, [u16, ctypes.c_int]),
@@ -148,6 +149,16 @@ def bounds(y, seq_offsets=None, scale: float = 2.0, correct_nonfinite: bool = Fa
     nf = np.zeros(S, np.uint32)
     lib().ft2o_bounds_dt(_p(y), rows, n, ld, _p(so), S, scale, int(correct_nonfinite), _p(b), _p(k), _p(nf), dtype)
     return b, k, nf
+
+
+def nan_vulnerable_count(y, seq_offsets=None, dtype=DT_BF16):
+    """Per-sequence count of values in (-2,-1) U (1,2)."""
+    y = np.ascontiguousarray(y, dtype=np.uint16)
+    so = None if seq_offsets is None else np.ascontiguousarray(seq_offsets, dtype=np.int32)
+    S = 1 if so is None else so.size - 1
+    out = np.zeros(S, np.uint32)
+    lib().ft2o_nan_vulnerable_count(_p(y), y.shape[0], y.shape[1], y.shape[1], _p(so), S, _p(out), dtype)
+    return out
 
 
 def bounds_from_keys(raw_keys, scale: float = 2.0, dtype=DT_BF16):

@@ -252,6 +252,26 @@ EXPORT void ft2o_bounds_from_keys(const int32_t* raw_keys, int32_t num_seqs, flo
     ft2o_bounds_from_keys_dt(raw_keys, num_seqs, scale, bounds, 0);
 }
 
+/* NaN-vulnerable values, PAPER.md L185 (Sec. 4.1.1, Fig. 7): "Values with
+ * specific exponent bits can become NaN after a single-bit flip, and most of
+ * them are in the intervals (-2, -1) or (1, 2) ... the NaN-vulnerable area";
+ * L202/L212: their share is the alternative criticality proxy.  Count, per
+ * sequence, the elements whose value v satisfies 1 < |v| < 2. */
+EXPORT void ft2o_nan_vulnerable_count(const uint16_t* y, int64_t rows, int64_t n, int64_t ld,
+                                      const int32_t* seq_offsets, int32_t num_seqs, uint32_t* out, int dtype) {
+    for (int32_t s = 0; s < num_seqs; ++s) {
+        int64_t r0 = seq_offsets ? seq_offsets[s] : 0;
+        int64_t r1 = seq_offsets ? seq_offsets[s + 1] : rows;
+        uint32_t c = 0;
+        for (int64_t r = r0; r < r1; ++r)
+            for (int64_t j = 0; j < n; ++j) {
+                double v = fabs(ft2o_to_f64_dt(y[r * ld + j], dtype));
+                if (v > 1.0 && v < 2.0) c++;
+            }
+        out[s] = c;
+    }
+}
+
 /* --------------------------------------------------------------- Philox --- */
 /* Philox4x32-10 (Salmon, Moraes, Dror, Shaw, SC'11), the counter-based
  * generator the fault-site reading R6 uses. */

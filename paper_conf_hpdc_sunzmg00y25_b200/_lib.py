@@ -59,7 +59,7 @@ def load(path: str = LIB):
     st = ctypes.c_int
     sig = {
         "ft2_workspace_bytes": (ctypes.c_size_t, [i32]),
-        "ft2_bounds_from_prefill": (st, [Tensor, P, i32, f32, i32, i32, P, P, P, P, P]),
+        "ft2_bounds_from_prefill": (st, [Tensor, P, i32, f32, i32, i32, P, P, P, P, P, P]),
         "ft2_bounds_finalize": (st, [P, i32, f32, ctypes.c_int, P, P]),
         "ft2_protect": (st, [Tensor, P, P, i32, P, P]),
         "ft2_gemm_workspace_bytes": (ctypes.c_size_t, [i32, i32, i32]),

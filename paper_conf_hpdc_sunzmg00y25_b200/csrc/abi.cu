@@ -59,8 +59,8 @@ size_t ft2_workspace_bytes(int32_t num_seqs) {
 
 ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int32_t num_seqs, float scale,
                                    int32_t finalize, int32_t correct_nonfinite, void* bounds_out,
-                                   int32_t* keys_out, uint32_t* nonfinite_count, void* workspace,
-                                   void* stream) {
+                                   int32_t* keys_out, uint32_t* nonfinite_count, uint32_t* nan_vulnerable_count,
+                                   void* workspace, void* stream) {
     ft2_status s = check_tensor(y);
     if (s != FT2_OK) return s;
     if (num_seqs < 1 || num_seqs > FT2_MAX_SEQS) return num_seqs < 1 ? FT2_ERR_INVALID_ARG : FT2_ERR_UNSUPPORTED;
@@ -92,6 +92,7 @@ ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int
     a.bounds_out = static_cast<uint16_t*>(bounds_out);
     a.keys_out = keys_out;
     a.nonfinite_out = nonfinite_count;
+    a.nv_out = nan_vulnerable_count;
     a.ws = static_cast<uint32_t*>(workspace);
     a.dtype = y.dtype;
     int nl = 0;

@@ -28,7 +28,7 @@ constexpr int kThreads = 256;
 constexpr int kUnroll = 4;
 
 size_t bounds_ws_bytes(int32_t S) {
-    size_t head = (size_t)(3 * S + 4) * 4;
+    size_t head = (size_t)(4 * S + 4) * 4;
     head = (head + 7) & ~(size_t)7;
     return head + (size_t)kPatchCap * 8;
 }
@@ -48,6 +48,7 @@ struct BoundsK {
     uint16_t* bounds_out;
     int32_t* keys_out;
     uint32_t* nonfinite_out;
+    uint32_t* nv_out;     // NaN-vulnerable counts or NULL
     uint32_t* ws;
 };
 
@@ -76,6 +77,17 @@ __device__ __forceinline__ void record_patch(const BoundsK& p, uint32_t* list_co
     else atomicExch(overflow, 1u);
 }
 
+// NaN-vulnerable halves of a packed word (Fig. 7: values in
+// (-2,-1) U (1,2), whose exponent-MSB flip gives NaN): |h| strictly between 1
+// and 2 <=> (h & 0x7FFF) in [one + 1, two - 1].
+template <int DT>
+__device__ __forceinline__ uint32_t nv_halves(uint32_t w) {
+    constexpr uint32_t one = DT == 1 ? 0x3C00u : 0x3F80u, two = DT == 1 ? 0x4000u : 0x4000u;
+    const uint32_t h = w & 0x7FFF7FFFu;
+    const uint32_t c = vmax_u16x2(vmin_u16x2(h, (two - 1) * 0x10001u), (one + 1) * 0x10001u);
+    return 2u - nonzero_halves(c ^ h);
+}
+
 // Slow exact path for one vector: min/max over finite keys, count the rest.
 template <int DT>
 __device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, uint32_t& kmin, uint32_t& kmax,
@@ -98,17 +110,17 @@ __device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, ui
     }
 }
 
-template <int DT>
+template <int DT, bool NV>
 __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
-    __shared__ uint32_t sh_min[kThreads / 32], sh_max[kThreads / 32], sh_nf[kThreads / 32];
+    __shared__ uint32_t sh_min[kThreads / 32], sh_max[kThreads / 32], sh_nf[kThreads / 32], sh_nv[kThreads / 32];
     __shared__ int sh_last;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int S = p.S;
-    uint32_t* ws_done = p.ws + 3 * S;
-    uint32_t* ws_lc = p.ws + 3 * S + 1;
-    uint32_t* ws_ov = p.ws + 3 * S + 2;
+    uint32_t* ws_done = p.ws + 4 * S;
+    uint32_t* ws_lc = p.ws + 4 * S + 1;
+    uint32_t* ws_ov = p.ws + 4 * S + 2;
     unsigned long long* list = reinterpret_cast<unsigned long long*>(
-        reinterpret_cast<char*>(p.ws) + (((size_t)(3 * S + 4) * 4 + 7) & ~(size_t)7));
+        reinterpret_cast<char*>(p.ws) + (((size_t)(4 * S + 4) * 4 + 7) & ~(size_t)7));
 
     uint32_t v = blockIdx.x * p.chunk;
     uint32_t v_end = min(v + p.chunk, p.total_vec);
@@ -129,7 +141,7 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
             seg_end = min(v_end, (uint32_t)p.seq_offsets[s + 1] * p.n8);
         }
         // ---- fast sweep of [v, seg_end): packed key min/max, 4 x 16 B in flight
-        uint32_t mn2 = 0xFFFFFFFFu, mx2 = 0u;
+        uint32_t mn2 = 0xFFFFFFFFu, mx2 = 0u, nv = 0u;
         for (uint32_t base = v + tid; base < seg_end; base += kThreads * kUnroll) {
             uint4 d[kUnroll];
 #pragma unroll
@@ -143,7 +155,11 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
                 uint32_t k0 = key2(d[u].x), k1 = key2(d[u].y), k2 = key2(d[u].z), k3 = key2(d[u].w);
                 uint32_t a = vmin_u16x2(vmin_u16x2(k0, k1), vmin_u16x2(k2, k3));
                 uint32_t b = vmax_u16x2(vmax_u16x2(k0, k1), vmax_u16x2(k2, k3));
-                if (vi < seg_end) { mn2 = vmin_u16x2(mn2, a); mx2 = vmax_u16x2(mx2, b); }
+                if (vi < seg_end) {
+                    mn2 = vmin_u16x2(mn2, a);
+                    mx2 = vmax_u16x2(mx2, b);
+                    if (NV) nv += nv_halves<DT>(d[u].x) + nv_halves<DT>(d[u].y) + nv_halves<DT>(d[u].z) + nv_halves<DT>(d[u].w);
+                }
             }
         }
         uint32_t kmin = min(mn2 & 0xFFFFu, mn2 >> 16);
@@ -159,17 +175,21 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
         kmin = __reduce_min_sync(0xFFFFFFFFu, kmin);
         kmax = __reduce_max_sync(0xFFFFFFFFu, kmax);
         nf = __reduce_add_sync(0xFFFFFFFFu, nf);
-        if (lane == 0) { sh_min[warp] = kmin; sh_max[warp] = kmax; sh_nf[warp] = nf; }
+        if (NV) nv = __reduce_add_sync(0xFFFFFFFFu, nv);
+        if (lane == 0) { sh_min[warp] = kmin; sh_max[warp] = kmax; sh_nf[warp] = nf; sh_nv[warp] = nv; }
         __syncthreads();
         if (tid == 0) {
-            uint32_t a = sh_min[0], b = sh_max[0], c = sh_nf[0];
+            uint32_t a = sh_min[0], b = sh_max[0], c = sh_nf[0], e = sh_nv[0];
 #pragma unroll
-            for (int i = 1; i < kThreads / 32; ++i) { a = min(a, sh_min[i]); b = max(b, sh_max[i]); c += sh_nf[i]; }
-            if (a <= b) {  // at least one finite value in this segment
-                atomicMax(&p.ws[3 * s + 0], 0x10000u - a);
-                atomicMax(&p.ws[3 * s + 1], b + 1u);
+            for (int i = 1; i < kThreads / 32; ++i) {
+                a = min(a, sh_min[i]); b = max(b, sh_max[i]); c += sh_nf[i]; e += sh_nv[i];
             }
-            if (c) atomicAdd(&p.ws[3 * s + 2], c);
+            if (NV && e) atomicAdd(&p.ws[4 * s + 3], e);
+            if (a <= b) {  // at least one finite value in this segment
+                atomicMax(&p.ws[4 * s + 0], 0x10000u - a);
+                atomicMax(&p.ws[4 * s + 1], b + 1u);
+            }
+            if (c) atomicAdd(&p.ws[4 * s + 2], c);
         }
         __syncthreads();
         v = seg_end;
@@ -184,9 +204,9 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
     __threadfence();
 
     for (int s = tid; s < S; s += kThreads) {
-        uint32_t los = atomicAdd(&p.ws[3 * s + 0], 0u);
-        uint32_t his = atomicAdd(&p.ws[3 * s + 1], 0u);
-        uint32_t nfc = atomicAdd(&p.ws[3 * s + 2], 0u);
+        uint32_t los = atomicAdd(&p.ws[4 * s + 0], 0u);
+        uint32_t his = atomicAdd(&p.ws[4 * s + 1], 0u);
+        uint32_t nfc = atomicAdd(&p.ws[4 * s + 2], 0u);
         bool have = los != 0u && his != 0u;
         uint32_t kmin = 0x10000u - los, kmax = his - 1u;
         if (p.finalize) {
@@ -203,9 +223,13 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
             p.keys_out[2 * s + 1] = have ? (int32_t)kmax : -1;
         }
         if (p.nonfinite_out) p.nonfinite_out[s] = nfc;
-        p.ws[3 * s + 0] = 0u;
-        p.ws[3 * s + 1] = 0u;
-        p.ws[3 * s + 2] = 0u;
+        if (NV) {
+            p.nv_out[s] = atomicAdd(&p.ws[4 * s + 3], 0u);
+            p.ws[4 * s + 3] = 0u;
+        }
+        p.ws[4 * s + 0] = 0u;
+        p.ws[4 * s + 1] = 0u;
+        p.ws[4 * s + 2] = 0u;
     }
     __syncthreads();
     if (p.correct) {
@@ -276,7 +300,8 @@ __global__ void finalize_kernel(const int32_t* keys, int32_t S, float scale, uin
 static int g_blocks_per_sm = 0;
 
 cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
-    auto kern = a.dtype == FT2_FP16 ? bounds_kernel<1> : bounds_kernel<0>;
+    auto kern = a.nv_out ? (a.dtype == FT2_FP16 ? bounds_kernel<1, true> : bounds_kernel<0, true>)
+                         : (a.dtype == FT2_FP16 ? bounds_kernel<1, false> : bounds_kernel<0, false>);
     BoundsK p;
     p.y = a.y;
     p.ld = a.ld;
@@ -292,10 +317,11 @@ cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
     p.bounds_out = a.bounds_out;
     p.keys_out = a.keys_out;
     p.nonfinite_out = a.nonfinite_out;
+    p.nv_out = a.nv_out;
     p.ws = a.ws;
     if (g_blocks_per_sm == 0) {
         int b = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel<0>, kThreads, 0);
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel<0, false>, kThreads, 0);
         if (e != cudaSuccess) return e;
         g_blocks_per_sm = b > 0 ? b : 1;
     }

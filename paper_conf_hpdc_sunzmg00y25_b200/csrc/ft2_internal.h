@@ -8,10 +8,10 @@
 namespace ft2impl {
 
 // Workspace of the bounds reduction (u32 words unless noted):
-//   [3s+0] lo slot  = 0x10000 - min key  (0 = no finite value yet)
-//   [3s+1] hi slot  = max key + 1        (0 = none)
-//   [3s+2] non-finite count
-//   [3S+0] CTA completion counter, [3S+1] patch-list count, [3S+2] overflow flag
+//   [4s+0] lo slot  = 0x10000 - min key  (0 = no finite value yet)
+//   [4s+1] hi slot  = max key + 1        (0 = none)
+//   [4s+2] non-finite count, [4s+3] NaN-vulnerable count
+//   [4S+0] CTA completion counter, [4S+1] patch-list count, [4S+2] overflow flag
 //   then (8-byte aligned) u64 patch list [kPatchCap]: offset | seq << 48
 constexpr int kPatchCap = 4096;
 size_t bounds_ws_bytes(int32_t S);
@@ -27,6 +27,7 @@ struct BoundsArgs {
     uint16_t* bounds_out;
     int32_t* keys_out;
     uint32_t* nonfinite_out;
+    uint32_t* nv_out;  // NaN-vulnerable counts or NULL
     uint32_t* ws;
     int32_t dtype;  // FT2_BF16 or FT2_FP16
 };

@@ -61,13 +61,14 @@ def make_workspace(num_seqs: int, device=None) -> torch.Tensor:
 
 def bounds_from_prefill(y, bounds_out, workspace, seq_offsets=None, num_seqs=None, scale=2.0,
                         finalize=True, correct_nonfinite=False, keys_out=None, nonfinite_count=None,
-                        stream=None):
+                        nan_vulnerable_count=None, stream=None):
     """ft2_bounds_from_prefill.  bounds_out: bf16 [S, 2] (or None when finalize=False)."""
     t = _as_ft2_tensor(y)
     S = num_seqs if num_seqs is not None else (1 if seq_offsets is None else seq_offsets.numel() - 1)
     st = load().ft2_bounds_from_prefill(t, _ptr(seq_offsets), S, float(scale), int(finalize),
                                         int(correct_nonfinite), _ptr(bounds_out), _ptr(keys_out),
-                                        _ptr(nonfinite_count), _ptr(workspace), _stream(stream))
+                                        _ptr(nonfinite_count), _ptr(nan_vulnerable_count), _ptr(workspace),
+                                        _stream(stream))
     check("ft2_bounds_from_prefill", st)
 
 

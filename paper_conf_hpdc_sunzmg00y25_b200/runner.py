@@ -67,6 +67,25 @@ class ModelConfig:
     def critical_names(self):
         return [n for n, _, _, c in self.linears() if c]
 
+    def coverage_names(self, coverage: str = "ft2"):
+        """Linear layers a protection scheme covers (Table 1).
+
+        "ft2": the critical layers (the heuristic of Sec. 4.1.2); "maximals":
+        OUT_PROJ/FC2/DOWN_PROJ; "globalclipper": V_PROJ/OUT_PROJ; "all": every
+        linear layer; "none": Ranger's coverage of linear layers (it protects
+        activation layers only, L315).  Llama's o_proj plays OUT_PROJ's role.
+        """
+        role = {"o_proj": "out_proj"}
+        sets = {"ft2": None, "all": None, "none": set(),
+                "maximals": {"out_proj", "fc2", "down_proj"}, "globalclipper": {"v_proj", "out_proj"}}
+        if coverage not in sets:
+            raise ValueError(f"unknown coverage {coverage!r}; one of {sorted(sets)}")
+        if coverage == "ft2":
+            return self.critical_names()
+        if coverage == "all":
+            return [n for n, _, _, _ in self.linears()]
+        return [n for n, _, _, _ in self.linears() if role.get(n, n) in sets[coverage]]
+
     def critical_widths(self):
         """Output width of every protected layer, block-major (the bounds/site layer ids)."""
         per = [o for _, o, _, c in self.linears() if c]
@@ -129,7 +148,7 @@ class Runner:
     """Batched greedy generation with FT2 on the critical layers."""
 
     def __init__(self, cfg: ModelConfig, batch: int, prompt_len: int, gen_len: int, seed: int = 1,
-                 device="cuda", scale: float = 2.0):
+                 device="cuda", scale: float = 2.0, coverage: str = "ft2"):
         self.cfg = cfg
         self.B = batch
         self.T = prompt_len
@@ -145,7 +164,8 @@ class Runner:
         self.lnf_w = torch.ones(h, dtype=torch.bfloat16, device=dv)
         self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
         self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h)
-        self.crit_names = cfg.critical_names()
+        self.coverage = coverage
+        self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
         self.state = FT2State(self.n_crit, batch, dv)
@@ -165,6 +185,7 @@ class Runner:
         self.time_phases = False
         self._phase_events = []
         self.mode = "fused"
+        self._nv = None          # NaN-vulnerable profiling counts [n_layers * n_lin, B] (profile_nan_vulnerable)
         if cfg.arch == "llama":
             inv = 1.0 / (10000 ** (torch.arange(0, D, 2, device=dv, dtype=torch.float32) / D))
             t = torch.arange(self.Tmax, device=dv, dtype=torch.float32)
@@ -213,6 +234,10 @@ class Runner:
             y = F.linear(x2, w, b)
             if sites is not None:
                 F2.inject_faults(y, sites, lid, 0, base_row=self.seq_offsets, n_sites=self.B)
+            if self._nv is not None:
+                li = self._lin_id(blk.idx, name)
+                F2.bounds_from_prefill(y, None, self._nv_ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
+                                       finalize=False, keys_out=self._nv_keys, nan_vulnerable_count=self._nv[li])
             if crit and self.mode != "off":
                 cid = self._crit_id(blk.idx, name)
                 st = self.state
@@ -373,6 +398,34 @@ class Runner:
             ev[2].record()
             self._phase_events.append(ev)
         return self.out_tokens
+
+    def profile_nan_vulnerable(self, prompt_ids):
+        """Share of NaN-vulnerable values in every linear layer's output.
+
+        PAPER.md L202 / Fig. 8(b): a fault-free profiling run records, per
+        linear layer, the percentage of output values in (-2,-1) U (1,2) --
+        those a flip of the highest exponent bit turns into NaN (L185, Fig. 7);
+        L212 names it the first proxy for layer criticality.  Runs one
+        unprotected prefill (mode "off") and counts inside the bounds sweep.
+        Returns (per-name share averaged over blocks and sequences, raw counts
+        [n_layers, n_lin, B] as int64, elements per (layer, sequence) [n_lin]).
+        """
+        B = self.B
+        n_lin = len(self.lin_names)
+        self._nv = torch.zeros((self.cfg.n_layers * n_lin, B), dtype=torch.int32, device=self.device)
+        self._nv_keys = torch.zeros((B, 2), dtype=torch.int32, device=self.device)
+        self._nv_ws = F2.make_workspace(B, device=self.device)
+        mode, self.mode = self.mode, "off"
+        try:
+            self.prefill(prompt_ids)
+            torch.cuda.synchronize()
+            counts = self._nv.view(self.cfg.n_layers, n_lin, B).to(torch.int64).cpu()
+        finally:
+            self._nv = None
+            self.mode = mode
+        elems = torch.tensor([o * self.T for _, o, _, _ in self.cfg.linears()], dtype=torch.int64)
+        share = counts.sum(dim=(0, 2)).double() / (elems.double() * self.cfg.n_layers * B)
+        return {n: float(share[i]) for i, n in enumerate(self.lin_names)}, counts, elems
 
     def phase_times(self):
         """(prefill ms, decode ms per step) averaged over the generate() calls

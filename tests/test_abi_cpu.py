@@ -73,7 +73,7 @@ def test_validation_without_gpu(L):
     def bfp(scale, **kw):
         a = dict(args, **kw)
         return L.ft2_bounds_from_prefill(good, a["so"], a["S"], scale, a["fin"], a["cor"], a["b"], a["k"], a["nf"],
-                                         a["ws"], None)
+                                         None, a["ws"], None)
     assert bfp(0.5) == FT2_ERR_INVALID_ARG
     assert bfp(float("nan")) == FT2_ERR_INVALID_ARG
     assert bfp(2.0, ws=None) == FT2_ERR_INVALID_ARG

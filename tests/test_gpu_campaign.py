@@ -58,3 +58,40 @@ def test_shards_sum_to_unsharded(tiny):
         for t in range(b, e, tiny.B):
             parts.add(campaign.run_batch(tiny, prompts, 9, t, 0))
     assert parts == full
+
+
+def test_coverage_none_equals_unprotected_and_all_detects():
+    """Table 1 coverages: with no protected linear layer (Ranger's linear-layer
+    coverage) FT2-on is FT2-off, trial by trial; covering every linear layer
+    corrects at least one fault."""
+    from paper_conf_hpdc_sunzmg00y25_b200 import campaign
+    from paper_conf_hpdc_sunzmg00y25_b200.runner import ModelConfig, Runner
+    cfg = ModelConfig("llama", 256, 512, 2, 4, 512, 512, False)
+    p = torch.randint(0, 512, (16, 8), generator=torch.Generator().manual_seed(4)).cuda()
+    none = Runner(cfg, batch=16, prompt_len=8, gen_len=6, seed=3, coverage="none")
+    r = campaign.run_batch(none, p, seed=5, trial0=0, fault_model=2)
+    assert none.n_crit == 0 and r.sdc_on == r.sdc_off and r.detected_on == 0 and r.golden_mismatch == 0
+    full = Runner(cfg, batch=16, prompt_len=8, gen_len=6, seed=3, coverage="all")
+    assert full.n_crit == 7 * 2
+    r = campaign.run_batch(full, p, seed=5, trial0=0, fault_model=2)
+    assert r.detected_on > 0
+
+
+def test_nan_vulnerable_profile_matches_oracle(tiny):
+    """PAPER.md L202 / Fig. 8(b): NaN-vulnerable share of each linear layer's
+    fault-free output; block 0's q_proj counts are recomputed with the oracle
+    from the same (deterministic) cuBLAS output."""
+    import torch.nn.functional as F
+    p = torch.randint(0, 512, (16, 8), generator=torch.Generator().manual_seed(6)).cuda()
+    share, counts, elems = tiny.profile_nan_vulnerable(p)
+    assert set(share) == set(tiny.lin_names) and all(0.0 <= v <= 1.0 for v in share.values())
+    assert counts.shape == (2, len(tiny.lin_names), 16)
+    blk = tiny.blocks[0]
+    pos = torch.arange(8, device="cuda")
+    x = tiny._embed(p, pos.unsqueeze(0).expand(16, 8))
+    h2 = tiny._norm(x, blk.ln1_w, blk.ln1_b).reshape(-1, tiny.cfg.hidden)
+    y = F.linear(h2, blk.w["q_proj"], blk.b["q_proj"])
+    yh = y.view(torch.int16).cpu().numpy().view(np.uint16)
+    want = oracle.nan_vulnerable_count(yh, seq_offsets=np.arange(0, 17 * 8, 8))
+    assert counts[0, 0].numpy().astype(np.uint32).tolist() == want.tolist()
+    assert int(elems[0]) == 8 * tiny.cfg.hidden

@@ -50,9 +50,12 @@ def test_fp16_bounds_and_correction(ft2, shape, so):
     yd = devh(y)
     b = torch.zeros((S, 2), dtype=torch.float16, device="cuda")
     nf = torch.zeros(S, dtype=torch.int32, device="cuda")
+    nv = torch.zeros(S, dtype=torch.int32, device="cuda")
+    rnv = oracle.nan_vulnerable_count(y, seq_offsets=so, dtype=F16)
     ft2.bounds_from_prefill(yd, b, ft2.make_workspace(S), seq_offsets=None if so is None else dev_i32(so),
-                            num_seqs=S, correct_nonfinite=True, nonfinite_count=nf)
+                            num_seqs=S, correct_nonfinite=True, nonfinite_count=nf, nan_vulnerable_count=nv)
     assert np.array_equal(hosth(b), rb) and np.array_equal(hosth(yd), ref)
+    assert np.array_equal(nv.cpu().numpy().astype(np.uint32), rnv)
     assert np.array_equal(nf.cpu().numpy().astype(np.uint32), rnf)
 
 

@@ -135,6 +135,28 @@ def test_bounds_bit_exact(ft2, shape, so, correct):
     assert np.array_equal(out, ref)   # correction (or untouched input)
 
 
+@pytest.mark.parametrize("shape,so", BOUNDS_CASES)
+def test_nan_vulnerable_count_bit_exact(ft2, shape, so):
+    """NaN-vulnerable values (Fig. 7), counted in the bounds sweep."""
+    y = _tensor(*shape, seed=shape[0] * 3 + shape[1])
+    y.reshape(-1)[5::97] = 0x3FC0          # 1.5: inside (1, 2)
+    y.reshape(-1)[11::89] = 0xBF80         # -1.0: boundary, not counted
+    want = oracle.nan_vulnerable_count(y, seq_offsets=so)
+    ref = y.copy()
+    rb, _, _ = oracle.bounds(ref, seq_offsets=so, correct_nonfinite=True)
+    S = 1 if so is None else len(so) - 1
+    yd = dev(y)
+    b = torch.zeros((S, 2), dtype=torch.bfloat16, device="cuda")
+    nv = torch.full((S,), -1, dtype=torch.int32, device="cuda")
+    ws = ft2.make_workspace(S)
+    ft2.bounds_from_prefill(yd, b, ws, seq_offsets=None if so is None else dev_i32(so), num_seqs=S,
+                            correct_nonfinite=True, nan_vulnerable_count=nv)
+    torch.cuda.synchronize()
+    assert np.array_equal(nv.cpu().numpy().astype(np.uint32), want) and int(want.sum()) > 0
+    assert np.array_equal(host(b), rb) and np.array_equal(host(yd), ref)
+    assert int(ws.abs().sum().item()) == 0
+
+
 @pytest.mark.parametrize("scale", [1.0, 1.25, 2.0, 3.0])
 def test_bounds_scales(ft2, scale):
     y = _tensor(64, 512, seed=17)

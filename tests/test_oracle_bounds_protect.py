@@ -216,3 +216,21 @@ def test_protect_nan_maps_to_clamped_zero():
         y = np.array([[0x7FC0, 0xFFC1]], np.uint16)
         oracle.protect(y, _bounds_pair(lo, hi))
         assert y.tolist() == [[want, want]]
+
+
+def test_nan_vulnerable_count_definition():
+    # the NaN-vulnerable values are exactly those an exponent-MSB
+    # flip turns into NaN, i.e. 1 < |v| < 2 -- checked against numpy decoding and
+    # against the flip itself, for bf16 and fp16, per sequence
+    import ml_dtypes
+    for dt, exp_msb, npdt in ((oracle.DT_BF16, 1 << 14, ml_dtypes.bfloat16), (oracle.DT_FP16, 1 << 14, np.float16)):
+        y = _rand_tensor(40, 64, 31)
+        y[::3, ::5] = np.array([0x3F90 if dt == 0 else 0x3C10], np.uint16)   # plant values in (1, 2)
+        so = [0, 10, 25, 40]
+        got = oracle.nan_vulnerable_count(y, so, dtype=dt)
+        v = np.abs(y.view(npdt).astype(np.float64))
+        want = [int(((v[a:b] > 1) & (v[a:b] < 2)).sum()) for a, b in zip(so[:-1], so[1:])]
+        assert got.tolist() == want and sum(want) > 0
+        flipped = (y ^ np.uint16(exp_msb)).view(npdt).astype(np.float64)
+        nan_after = np.isnan(flipped) & ~np.isnan(y.view(npdt).astype(np.float64))
+        assert int(nan_after.sum()) == sum(want)
