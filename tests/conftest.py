@@ -9,6 +9,9 @@ if ROOT not in sys.path:
 
 
 def pytest_configure(config):
+    # a fresh checkout has no libft2.so / liboracle yet: build both (nvcc cross-compiles without a GPU)
+    import __graft_entry__
+    __graft_entry__.build()
     config.addinivalue_line("markers", "gpu: needs a CUDA B200 (sm_100a) device")
     config.addinivalue_line("markers", "slow: long-running CPU test")
 
