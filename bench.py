@@ -60,16 +60,42 @@ def load_peaks():
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
+    """SM clock + throttle reasons sampled DURING the timed region.  Uses NVML
+    in-process (a 100 ms polling thread: one ioctl per sample, no subprocess
+    competing with the host-side launch path); falls back to `nvidia-smi -lms`."""
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
-    def __init__(self, dev_index: int):
+    def __init__(self, dev_index: int, period_s: float = 0.1):
         self.dev = dev_index
+        self.period = period_s
         self.proc = None
+        self.nvml = None
         self.lines = []
+        self.samples = []     # (sm_mhz, max_mhz, reasons bitmask)
+
+    def _nvml_handle(self):
+        import pynvml as N
+        import torch
+        N.nvmlInit()
+        pr = torch.cuda.get_device_properties(self.dev)
+        dom, bus, dev = (getattr(pr, k, None) for k in ("pci_domain_id", "pci_bus_id", "pci_device_id"))
+        if all(isinstance(v, int) for v in (dom, bus, dev)):   # CUDA_VISIBLE_DEVICES-safe mapping
+            return N, N.nvmlDeviceGetHandleByPciBusId(f"{dom:08X}:{bus:02X}:{dev:02X}.0")
+        return N, N.nvmlDeviceGetHandleByIndex(self.dev)
 
     def start(self):
+        try:
+            N, h = self._nvml_handle()
+            self.nvml = (N, h)
+            self.stop_ev = threading.Event()
+            self.th = threading.Thread(target=self._poll, daemon=True)
+            self.th.start()
+            return
+        except Exception:
+            self.nvml = None
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
@@ -79,11 +105,34 @@ class ClockSampler:
         except Exception:
             self.proc = None
 
+    def _poll(self):
+        N, h = self.nvml
+        get_reasons = getattr(N, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            N.nvmlDeviceGetCurrentClocksThrottleReasons
+        mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+        while not self.stop_ev.is_set():
+            try:
+                self.samples.append((N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM), mx, int(get_reasons(h))))
+            except Exception:
+                pass
+            self.stop_ev.wait(self.period)
+
     def _read(self):
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
     def stop(self):
+        if self.nvml is not None:
+            self.stop_ev.set()
+            self.th.join(timeout=2)
+            N = self.nvml[0]
+            bits = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20,
+                    "sw_power_cap": 0x4}
+            reasons = sorted({n for _, _, r in self.samples for n, b in bits.items() if r & b})
+            sm = [c for c, _, _ in self.samples]
+            return {"sm_mhz": statistics.median(sm) if sm else None,
+                    "sm_max_mhz": max(m for _, m, _ in self.samples) if self.samples else None,
+                    "reasons": reasons, "samples": len(sm), "source": "nvml"}
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         self.proc.terminate()
@@ -93,7 +142,6 @@ class ClockSampler:
             self.proc.kill()
         self.th.join(timeout=2)
         sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:
             p = [x.strip() for x in ln.split(",")]
             if len(p) < 6:
@@ -103,11 +151,11 @@ class ClockSampler:
                 mx.append(float(p[1]))
             except ValueError:
                 continue
-            for n, v in zip(names, p[2:6]):
+            for n, v in zip(self.NAMES, p[2:6]):
                 if v.lower() == "active":
                     reasons.add(n)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm), "source": "nvidia-smi"}
 
 
 # ------------------------------------------------------------ CPU baseline

@@ -4,7 +4,7 @@
 // Each CTA owns a contiguous range of 16-byte vectors (8 bf16) of the prefill
 // output and splits it at sequence boundaries.  Per segment every thread keeps
 // a packed-u16x2 min and max of order keys over its 128-bit coalesced loads
-// (4 loads in flight per thread: PRMT+LOP3 for the keys, VIMNMX.U16x2 for the
+// (4-8 loads in flight per thread: PRMT+LOP3 for the keys, VIMNMX.U16x2 for the
 // min/max -- 2 ALU ops per element), the warp combines with redux.sync
 // (CREDUX), the CTA through shared memory, and the grid through u32 atomicMax
 // on a self-cleaning workspace.  The last CTA to finish (threadfence
@@ -20,12 +20,12 @@
 
 #include "ft2_device.cuh"
 #include "ft2_internal.h"
+#include "sm100_ptx.cuh"
 
 namespace ft2impl {
 using namespace ft2dev;
 
 constexpr int kThreads = 256;
-constexpr int kUnroll = 4;
 
 size_t bounds_ws_bytes(int32_t S) {
     size_t head = (size_t)(4 * S + 4) * 4;
@@ -110,7 +110,9 @@ __device__ __forceinline__ void slow_vec(const BoundsK& p, uint32_t v, int s, ui
     }
 }
 
-template <int DT, bool NV>
+// kUnroll 16-byte loads in flight per thread: 8 for tensors one sweep covers
+// (latency-bound, e.g. prefill outputs), 4 for the bandwidth-bound large ones.
+template <int DT, bool NV, int kUnroll>
 __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
     __shared__ uint32_t sh_min[kThreads / 32], sh_max[kThreads / 32], sh_nf[kThreads / 32], sh_nv[kThreads / 32];
     __shared__ int sh_last;
@@ -195,18 +197,21 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
         v = seg_end;
     }
 
-    // ---- grid combine: the last CTA finalises
-    __threadfence();
+    // ---- grid combine: the last CTA finalises.  One acq_rel atomic per CTA
+    // (release: cumulative over this CTA's REDs and patch records, which the
+    // barrier orders before it; acquire for the last CTA), then every slot is
+    // read with independent L2 loads: two L2 round trips on the critical path.
     __syncthreads();
-    if (tid == 0) sh_last = (atomicAdd(ws_done, 1u) == gridDim.x - 1);
+    if (tid == 0) sh_last = (atom_add_acq_rel_gpu(ws_done, 1u) == gridDim.x - 1);
     __syncthreads();
     if (!sh_last) return;
-    __threadfence();
 
+    const uint32_t lc0 = p.correct ? __ldcg(ws_lc) : 0u, ov0 = p.correct ? __ldcg(ws_ov) : 0u;
     for (int s = tid; s < S; s += kThreads) {
-        uint32_t los = atomicAdd(&p.ws[4 * s + 0], 0u);
-        uint32_t his = atomicAdd(&p.ws[4 * s + 1], 0u);
-        uint32_t nfc = atomicAdd(&p.ws[4 * s + 2], 0u);
+        // lo, hi, non-finite, NaN-vulnerable slots (the workspace is 8-byte aligned)
+        const uint2 wa = __ldcg(reinterpret_cast<const uint2*>(p.ws + 4 * s));
+        const uint2 wb = __ldcg(reinterpret_cast<const uint2*>(p.ws + 4 * s + 2));
+        const uint32_t los = wa.x, his = wa.y, nfc = wb.x;
         bool have = los != 0u && his != 0u;
         uint32_t kmin = 0x10000u - los, kmax = his - 1u;
         if (p.finalize) {
@@ -223,22 +228,15 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
             p.keys_out[2 * s + 1] = have ? (int32_t)kmax : -1;
         }
         if (p.nonfinite_out) p.nonfinite_out[s] = nfc;
-        if (NV) {
-            p.nv_out[s] = atomicAdd(&p.ws[4 * s + 3], 0u);
-            p.ws[4 * s + 3] = 0u;
-        }
-        p.ws[4 * s + 0] = 0u;
-        p.ws[4 * s + 1] = 0u;
-        p.ws[4 * s + 2] = 0u;
+        if (NV) p.nv_out[s] = wb.y;
+        *reinterpret_cast<uint2*>(p.ws + 4 * s) = make_uint2(0u, 0u);
+        *reinterpret_cast<uint2*>(p.ws + 4 * s + 2) = make_uint2(0u, 0u);
     }
-    __syncthreads();
-    if (p.correct) {
-        __threadfence_block();
-        uint32_t cnt = atomicAdd(ws_lc, 0u);
-        uint32_t ov = atomicAdd(ws_ov, 0u);
-        if (!ov) {
-            for (uint32_t i = tid; i < cnt; i += kThreads) {
-                unsigned long long e = list[i];
+    __syncthreads();  // bounds_out of every sequence written (read back by the patch fix-up)
+    if (p.correct && lc0 != 0u) {
+        if (!ov0) {
+            for (uint32_t i = tid; i < lc0; i += kThreads) {
+                unsigned long long e = __ldcg(list + i);
                 int s = (int)(e >> 48);
                 uint64_t off = e & 0xFFFFFFFFFFFFull;
                 uint16_t b = p.y[off];
@@ -269,13 +267,10 @@ __global__ void __launch_bounds__(kThreads) bounds_kernel(BoundsK p) {
                 }
             }
         }
-    }
-    __syncthreads();
-    if (p.correct) {  // leave the patch list zero-filled as well
-        uint32_t used = min(atomicAdd(ws_lc, 0u), (uint32_t)kPatchCap);
+        __syncthreads();  // leave the patch list zero-filled as well
+        const uint32_t used = min(lc0, (uint32_t)kPatchCap);
         for (uint32_t i = tid; i < used; i += kThreads) list[i] = 0ull;
     }
-    __syncthreads();
     if (tid == 0) {
         *ws_lc = 0u;
         *ws_ov = 0u;
@@ -300,8 +295,6 @@ __global__ void finalize_kernel(const int32_t* keys, int32_t S, float scale, uin
 static int g_blocks_per_sm = 0;
 
 cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
-    auto kern = a.nv_out ? (a.dtype == FT2_FP16 ? bounds_kernel<1, true> : bounds_kernel<0, true>)
-                         : (a.dtype == FT2_FP16 ? bounds_kernel<1, false> : bounds_kernel<0, false>);
     BoundsK p;
     p.y = a.y;
     p.ld = a.ld;
@@ -321,17 +314,26 @@ cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
     p.ws = a.ws;
     if (g_blocks_per_sm == 0) {
         int b = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel<0, false>, kThreads, 0);
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds_kernel<0, false, 4>, kThreads, 0);
         if (e != cudaSuccess) return e;
         g_blocks_per_sm = b > 0 ? b : 1;
     }
-    const uint32_t per_iter = kThreads * kUnroll;
-    uint32_t max_grid = (uint32_t)(num_sms() * g_blocks_per_sm);
-    uint32_t want = (p.total_vec + 2 * per_iter - 1) / (2 * per_iter);  // >= 2 sweeps per CTA
+    const uint32_t max_grid = (uint32_t)(num_sms() * g_blocks_per_sm);
+    const bool one_sweep = p.total_vec <= max_grid * (uint32_t)(kThreads * 8);
+    const uint32_t per_iter = kThreads * (one_sweep ? 8 : 4);
+    uint32_t want = (p.total_vec + per_iter - 1) / per_iter;  // one sweep per thread if possible
     uint32_t grid = want < 1 ? 1 : (want > max_grid ? max_grid : want);
     p.chunk = (p.total_vec + grid - 1) / grid;
     grid = (p.total_vec + p.chunk - 1) / p.chunk;
     if (grid < 1) grid = 1;
+    void (*kern)(BoundsK);
+    const bool fp16 = a.dtype == FT2_FP16, nv = a.nv_out != nullptr;
+    if (one_sweep)
+        kern = nv ? (fp16 ? bounds_kernel<1, true, 8> : bounds_kernel<0, true, 8>)
+                  : (fp16 ? bounds_kernel<1, false, 8> : bounds_kernel<0, false, 8>);
+    else
+        kern = nv ? (fp16 ? bounds_kernel<1, true, 4> : bounds_kernel<0, true, 4>)
+                  : (fp16 ? bounds_kernel<1, false, 4> : bounds_kernel<0, false, 4>);
     kern<<<grid, kThreads, 0, st>>>(p);
     ++*n_launch;
     return cudaGetLastError();

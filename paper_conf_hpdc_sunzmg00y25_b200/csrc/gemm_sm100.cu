@@ -89,6 +89,8 @@ struct GemmK {
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
     int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
+    int32_t rows_per_slot;  // ceil(128 / splitk): rows of one split-K receive slot
+    uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
 };
 
 // Per-row / per-column epilogue table entry.  Feature side: bias, flags
@@ -128,9 +130,13 @@ __device__ __forceinline__ TabE token_entry(const GemmK& p, int m) {
     return e;
 }
 
-template <int BN>
+// DEEP: one CTA per SM with a ring deep enough (~180 KB) that a CTA's whole K
+// slice is in flight at once -- one DRAM round trip for few-tile decode
+// shapes.  Otherwise ~105 KB so two CTAs share an SM.
+template <int BN, bool DEEP = false>
 struct Cfg {
-    static constexpr int STAGES = BN <= 16 ? 5 : (BN <= 32 ? 4 : (BN <= 64 ? 3 : 4));
+    static constexpr int STAGES = DEEP ? (BN <= 16 ? 10 : (BN <= 32 ? 9 : 7))
+                                       : (BN <= 16 ? 5 : (BN <= 32 ? 4 : (BN <= 64 ? 3 : 4)));
     static constexpr int kABytes = kBlockA * kBlockK * 2;
     static constexpr int kBBytes = BN * kBlockK * 2;
     static constexpr int kStageBytes = kABytes + kBBytes;
@@ -225,11 +231,11 @@ __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, i
     }
 }
 
-template <int BN, bool SWAP, int DT>
+template <int BN, bool SWAP, int DT, bool DEEP>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
                 const __grid_constant__ GemmK p) {
-    using C = Cfg<BN>;
+    using C = Cfg<BN, DEEP>;
     constexpr int STAGES = C::STAGES;
     extern __shared__ uint8_t smem_raw[];
     // 1024-byte alignment (128B swizzle) by offset arithmetic on the shared
@@ -258,7 +264,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     const int kb1 = (int)((int64_t)(split + 1) * p.nkb / splitk);
     const int nk = kb1 - kb0;
     // rows of the tile this CTA finishes: all of them, or its split-K slice
-    const int r0 = (split * kBlockA) / splitk, r1 = ((split + 1) * kBlockA) / splitk;
+    const int r0 = (int)(((uint32_t)(split * kBlockA) * p.sk_magic) >> 24);
+    const int r1 = (int)(((uint32_t)((split + 1) * kBlockA) * p.sk_magic) >> 24);
 
     if (warp == 0 && lane == 0) {
         FT2_TRACE(0);
@@ -362,21 +369,43 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 }
             }
         }
+        // Receive-slot geometry of accumulator row a (independent of the
+        // accumulator, so computed while the main loop streams): its owner
+        // is the split whose row slice holds a, r0(r) = floor(128 r / splitk)
+        // evaluated as (128 r * sk_magic) >> 24 (exact for these ranges).
+        const int RS = p.rows_per_slot;
+        const int owner = ((a + 1) * splitk - 1) >> 7;
+        const int own_r0 = (int)(((uint32_t)(owner * kBlockA) * p.sk_magic) >> 24);
+        const uint32_t slot_off = (uint32_t)(((split * RS + (a - own_r0)) * C::kRecvStride) * 4);
+        const bool local = owner == split;
+        const uint32_t dst = local ? smem_u32(recv) + slot_off : mapa(smem_u32(recv) + slot_off, (uint32_t)owner);
+        const uint32_t dbar = local ? 0u : mapa(smem_u32(recv_bar), (uint32_t)owner);
+        const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
+        // finish-loop geometry: item v -> (row lr, column quad c4)
+        const int e = tid - 64;  // 0..127
+        const int nrow = r1 - r0;
+        const int nvec = nrow * (BN / 4);
+        const uint32_t inv = (uint32_t)((1u << 20) + nrow - 1) / (uint32_t)nrow;  // v / nrow == (v * inv) >> 20
+        if (splitk > 1) cluster_wait();  // every peer's receive barrier is initialised
         mbar_wait(tmem_full, 0);
         if (a == 0) FT2_TRACE(5);
         tc_fence_after();
         // Stage accumulator row a as fp32 in the receive slot of its owner
         // (this CTA without split-K; a cluster peer with it).
-        const int RS = (kBlockA + splitk - 1) / splitk;  // rows per receive slot
-        int owner = 0;
-        while (owner + 1 < splitk && a >= ((owner + 1) * kBlockA) / splitk) ++owner;
-        const uint32_t slot_off =
-            (uint32_t)(((split * RS + (a - (owner * kBlockA) / splitk)) * C::kRecvStride) * 4);
-        if (splitk > 1) cluster_wait();  // every peer's receive barrier is initialised
-        const bool local = owner == split;
-        const uint32_t dst = local ? smem_u32(recv) + slot_off : mapa(smem_u32(recv) + slot_off, (uint32_t)owner);
-        const uint32_t dbar = local ? 0u : mapa(smem_u32(recv_bar), (uint32_t)owner);
-        const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
+        if constexpr (BN == 32) {  // one TMEM load for the whole row, then the pushes back to back
+            uint32_t r[32];
+            tmem_ld32(taddr, r);
+            tmem_wait_ld();
+            if (nk == 0) {
+#pragma unroll
+                for (int j = 0; j < 32; ++j) r[j] = 0u;
+            }
+#pragma unroll
+            for (int j = 0; j < 32; j += 4) {
+                if (local) st_shared_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
+                else st_async_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
+            }
+        } else
 #pragma unroll 1
         for (int c0 = 0; c0 < BN; c0 += 16) {
             uint32_t r[16];
@@ -392,25 +421,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 else st_async_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
             }
         }
-    }
-    // ---------------------------------------------- finish the slice (all warps)
-    named_bar(2, kGemmThreads);  // tables, site list and my own rows are in shared memory
-    if (splitk > 1 && warp < 2) cluster_wait();  // pair the prologue arrive of the non-epilogue warps
-    griddep_wait();              // (no-op for threads that already waited)
-    if (splitk > 1) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
-    if (tid == 64) FT2_TRACE(6);
-    {
+        if (tid == 64) FT2_TRACE(8);
+        // ------------------------------------ finish the slice (epilogue warps)
+        named_bar(2, 128);  // tables, site list and my own rows are in shared memory
+        if (tid == 64) FT2_TRACE(9);
+        if (splitk > 1) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
+        if (tid == 64) FT2_TRACE(6);
         const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
-        const int RS = (kBlockA + splitk - 1) / splitk;
-        const int nrow = r1 - r0;
-        const int nvec = nrow * (BN / 4);
-        const uint32_t inv = (uint32_t)((1u << 20) + nrow - 1) / (uint32_t)nrow;  // v / nrow == (v * inv) >> 20
         uint16_t* const y = p.y;
         const int64_t ldy = p.ldy;
 #pragma unroll 1
-        for (int v = tid; v < nvec; v += kGemmThreads) {
-            // item v -> (row lr, column quad c4); consecutive threads take
-            // consecutive rows (coalesced stores in swap-AB mode)
+        for (int v = e; v < nvec; v += 128) {
+            // consecutive threads take consecutive rows (coalesced stores in swap-AB mode)
             const int c4 = (int)(((uint32_t)v * inv) >> 20), lr = v - c4 * nrow, la = r0 + lr;
             const float* src = recv + lr * C::kRecvStride + c4 * 4;
             float4 part[kMaxSplitK];
@@ -421,17 +443,20 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
             for (int rr = 1; rr < kMaxSplitK; ++rr)
                 if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
+            if (tid == 64) FT2_TRACE(11);
             finish4<SWAP, DT>(y, ldy, tileA * kBlockA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
-                          (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4);
+                              (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4);
+        }
+        if (tid == 64) FT2_TRACE(7);
+        if (p.counts != nullptr && p.mode == FT2_GEMM_CHECK) {
+            named_bar(3, 128);  // every finish4 of this CTA has counted
+            if (!SWAP && row_cnt[e] != 0u) atomicAdd(&p.counts[row_tab[e].seq], row_cnt[e]);
+            for (int c = e; SWAP && c < BN; c += 128)
+                if (col_cnt[c] != 0u) atomicAdd(&p.counts[col_tab[c].seq], col_cnt[c]);
         }
     }
-    if (tid == 64) FT2_TRACE(7);
-    if (p.counts != nullptr && p.mode == FT2_GEMM_CHECK) {
-        named_bar(2, kGemmThreads);  // every finish4 of this CTA has counted
-        if (!SWAP && tid < kBlockA && row_cnt[tid] != 0u) atomicAdd(&p.counts[row_tab[tid].seq], row_cnt[tid]);
-        for (int c = tid; SWAP && c < BN; c += kGemmThreads)
-            if (col_cnt[c] != 0u) atomicAdd(&p.counts[col_tab[c].seq], col_cnt[c]);
-    }
+    // warps 0 and 1 pair their prologue cluster arrive (no finish work for them)
+    if (splitk > 1 && warp < 2) cluster_wait();
     tc_fence_before();
     __syncthreads();
     if (warp == 1) {
@@ -468,16 +493,31 @@ static bool make_map(CUtensorMap* m, const void* base, int64_t rows, int64_t K, 
     return r == CUDA_SUCCESS;
 }
 
-template <int BN, bool SWAP, int DT>
+// Experiment knobs (read once): FT2_GEMM_SMEM_PAD adds dynamic shared memory
+// (fewer CTAs per SM), FT2_GEMM_SPREAD=1 asks for the spread cluster policy.
+static int smem_pad() {
+    static const int v = [] { const char* e = getenv("FT2_GEMM_SMEM_PAD"); return e ? atoi(e) : 0; }();
+    return v;
+}
+static int env_int(const char* name, int dflt) {
+    const char* e = getenv(name);
+    return e ? atoi(e) : dflt;
+}
+static int spread_policy() {
+    static const int v = [] { const char* e = getenv("FT2_GEMM_SPREAD"); return e ? atoi(e) : 0; }();
+    return v;
+}
+
+template <int BN, bool SWAP, int DT, bool DEEP>
 static cudaError_t set_attrs() {
     static cudaError_t res = [] {
-        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             Cfg<BN>::kBytes);
+        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT, DEEP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg<BN, DEEP>::kBytes + smem_pad());
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT, DEEP>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
         // full shared-memory carveout so two ~105 KB decode CTAs share an SM
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT>, cudaFuncAttributePreferredSharedMemoryCarveout,
+        if (e == cudaSuccess && env_int("FT2_GEMM_CARVEOUT", 1))
+            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT, DEEP>, cudaFuncAttributePreferredSharedMemoryCarveout,
                                      (int)cudaSharedmemCarveoutMaxShared);
         return e;
     }();
@@ -485,16 +525,16 @@ static cudaError_t set_attrs() {
 }
 
 // How many (1, sk, 1) clusters of this instantiation can be resident at once.
-template <int BN, bool SWAP, int DT = 0>
+template <int BN, bool SWAP, int DT = 0, bool DEEP = false>
 static int max_clusters(int sk) {
     static int cache[kMaxSplitK + 1] = {0};
     if (sk < 1 || sk > kMaxSplitK) return -1;
     if (cache[sk] != 0) return cache[sk];
-    if (set_attrs<BN, SWAP, DT>() != cudaSuccess) return cache[sk] = -1;
+    if (set_attrs<BN, SWAP, DT, DEEP>() != cudaSuccess) return cache[sk] = -1;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(1, (unsigned)sk, 1);
     cfg.blockDim = dim3(kGemmThreads);
-    cfg.dynamicSmemBytes = Cfg<BN>::kBytes;
+    cfg.dynamicSmemBytes = Cfg<BN, DEEP>::kBytes + smem_pad();
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 1;
@@ -503,14 +543,22 @@ static int max_clusters(int sk) {
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     int n = 0;
-    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BN, SWAP, DT>, &cfg) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BN, SWAP, DT, DEEP>, &cfg) != cudaSuccess) {
         cudaGetLastError();
         n = -1;
     }
     return cache[sk] = (n > 0 ? n : -1);
 }
 
-static int max_clusters_bn(int bn, int sk) {
+static int max_clusters_bn(int bn, int sk, bool deep = false) {
+    if (deep) {
+        switch (bn) {
+            case 16: return max_clusters<16, true, 0, true>(sk);
+            case 32: return max_clusters<32, true, 0, true>(sk);
+            case 64: return max_clusters<64, true, 0, true>(sk);
+            default: return -1;
+        }
+    }
     switch (bn) {
         case 16: return max_clusters<16, true>(sk);
         case 32: return max_clusters<32, true>(sk);
@@ -518,10 +566,18 @@ static int max_clusters_bn(int bn, int sk) {
         default: return max_clusters<128, true>(sk);
     }
 }
+static int deep_stages(int bn) {
+    switch (bn) {
+        case 16: return Cfg<16, true>::STAGES;
+        case 32: return Cfg<32, true>::STAGES;
+        case 64: return Cfg<64, true>::STAGES;
+        default: return 0;
+    }
+}
 
 // Tiling plan: orientation, tile width, split-K factor.
 struct GemmPlan {
-    int swap, bn, tilesA, tilesB, splitk, nkb;
+    int swap, bn, tilesA, tilesB, splitk, nkb, deep;
 };
 
 static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
@@ -558,21 +614,44 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
         best = sk;
     }
     g.splitk = best;
+    g.deep = 0;
+    // Few-tile decode shapes: one CTA per SM with the CTA's whole K slice in
+    // flight (one DRAM round trip) when all clusters fit in one wave.
+    static const int deep_env = env_int("FT2_GEMM_DEEP", 0);  // measured slower in situ: opt-in
+    if (g.swap && g.bn <= 64 && deep_env != 0) {
+        const int st = deep_stages(g.bn);
+        int dk = 0;
+        for (int sk = 1; sk <= 8; ++sk) {
+            if (tiles * sk > sms) break;
+            if (max_clusters_bn(g.bn, sk, true) < tiles) continue;
+            dk = sk;
+            if ((g.nkb + sk - 1) / sk <= st) break;  // smallest split with a single round trip
+        }
+        if (dk > 0 && ((g.nkb + dk - 1) / dk <= st || deep_env == 1)) {
+            g.deep = 1;
+            g.splitk = dk;
+            if (sk_env > 0) {
+                int sk = sk_env < g.nkb ? sk_env : g.nkb;
+                while (sk > 1 && max_clusters_bn(g.bn, sk, true) < 1) --sk;
+                g.splitk = sk;
+            }
+        }
+    }
     static const bool dbg = getenv("FT2_GEMM_DEBUG") != nullptr;
     if (dbg) {
-        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d bn=%d tiles=%dx%d nkb=%d splitk=%d clusters(sk)=", M, N, K,
-                g.swap, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk);
+        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d bn=%d tiles=%dx%d nkb=%d splitk=%d deep=%d clusters(sk)=", M,
+                N, K, g.swap, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk, g.deep);
         for (int sk = 2; sk <= 8 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
         int occ = -1;
         if (g.bn == 32) {
-            set_attrs<32, true, 0>();
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gemm_kernel<32, true, 0>, kGemmThreads, Cfg<32>::kBytes);
+            set_attrs<32, true, 0, false>();
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gemm_kernel<32, true, 0, false>, kGemmThreads, Cfg<32>::kBytes);
         }
         size_t avail2 = 0, avail1 = 0;
-        cudaOccupancyAvailableDynamicSMemPerBlock(&avail2, gemm_kernel<32, true, 0>, 2, kGemmThreads);
-        cudaOccupancyAvailableDynamicSMemPerBlock(&avail1, gemm_kernel<32, true, 0>, 1, kGemmThreads);
+        cudaOccupancyAvailableDynamicSMemPerBlock(&avail2, gemm_kernel<32, true, 0, false>, 2, kGemmThreads);
+        cudaOccupancyAvailableDynamicSMemPerBlock(&avail1, gemm_kernel<32, true, 0, false>, 1, kGemmThreads);
         cudaFuncAttributes fa;
-        cudaFuncGetAttributes(&fa, gemm_kernel<32, true, 0>);
+        cudaFuncGetAttributes(&fa, gemm_kernel<32, true, 0, false>);
         int smem_sm = 0, dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
@@ -586,7 +665,7 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
 // The cluster split-K needs no global workspace.
 size_t gemm_ws_bytes(int32_t, int32_t, int32_t) { return 0; }
 
-template <int BN, bool SWAP, int DT>
+template <int BN, bool SWAP, int DT, bool DEEP = false>
 static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st, int* n_launch) {
     CUtensorMap ma, mb;
     const void* pa = SWAP ? (const void*)a.w : (const void*)a.x;
@@ -594,23 +673,26 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     const int64_t lda = SWAP ? a.ldw : a.ldx, ldb = SWAP ? a.ldx : a.ldw;
     if (!make_map(&ma, pa, p.rowsA, a.K, lda, kBlockA, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
     if (!make_map(&mb, pb, p.rowsB, a.K, ldb, BN, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
-    cudaError_t e = set_attrs<BN, SWAP, DT>();
+    cudaError_t e = set_attrs<BN, SWAP, DT, DEEP>();
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);
     cfg.blockDim = dim3(kGemmThreads);
-    cfg.dynamicSmemBytes = Cfg<BN>::kBytes;
+    cfg.dynamicSmemBytes = Cfg<BN, DEEP>::kBytes + smem_pad();
     cfg.stream = st;
-    cudaLaunchAttribute attr[2];
+    cudaLaunchAttribute attr[3];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    static const int pdl = env_int("FT2_GEMM_PDL", 1);
+    attr[0].val.programmaticStreamSerializationAllowed = pdl;
     attr[1].id = cudaLaunchAttributeClusterDimension;
     attr[1].val.clusterDim.x = 1;
     attr[1].val.clusterDim.y = (unsigned)p.splitk;
     attr[1].val.clusterDim.z = 1;
+    attr[2].id = cudaLaunchAttributeClusterSchedulingPolicyPreference;
+    attr[2].val.clusterSchedulingPolicyPreference = cudaClusterSchedulingPolicySpread;
     cfg.attrs = attr;
-    cfg.numAttrs = p.splitk > 1 ? 2 : 1;
-    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP, DT>, ma, mb, p);
+    cfg.numAttrs = p.splitk > 1 ? (spread_policy() ? 3 : 2) : 1;
+    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP, DT, DEEP>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -644,6 +726,22 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cur_step = a.cur_step;
     p.base_row = a.base_row;
     p.w_static = a.w_static;
+    p.rows_per_slot = (kBlockA + g.splitk - 1) / g.splitk;
+    p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
+    if (g.deep) {
+        if (a.dtype == FT2_FP16) {
+            switch (g.bn) {
+                case 16: return launch_cfg<16, true, 1, true>(a, p, st, n_launch);
+                case 32: return launch_cfg<32, true, 1, true>(a, p, st, n_launch);
+                default: return launch_cfg<64, true, 1, true>(a, p, st, n_launch);
+            }
+        }
+        switch (g.bn) {
+            case 16: return launch_cfg<16, true, 0, true>(a, p, st, n_launch);
+            case 32: return launch_cfg<32, true, 0, true>(a, p, st, n_launch);
+            default: return launch_cfg<64, true, 0, true>(a, p, st, n_launch);
+        }
+    }
     if (a.dtype == FT2_FP16) {
         if (!g.swap) return launch_cfg<128, false, 1>(a, p, st, n_launch);
         switch (g.bn) {
@@ -665,6 +763,22 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
 }  // namespace ft2impl
 
 #ifdef FT2_GEMM_TRACE
+namespace ft2impl {
+__device__ unsigned long long g_marks[64];
+__global__ void mark_kernel(int slot) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_marks[slot & 63] = t;
+}
+}  // namespace ft2impl
+// one-thread kernel that records the global timer (launch-gap measurements)
+extern "C" int ft2_debug_mark(int slot, cudaStream_t st) {
+    ft2impl::mark_kernel<<<1, 32, 0, st>>>(slot);
+    return (int)cudaGetLastError();
+}
+extern "C" int ft2_debug_marks_read(void* dst) {
+    return (int)cudaMemcpyFromSymbol(dst, ft2impl::g_marks, sizeof(ft2impl::g_marks));
+}
 extern "C" int ft2_debug_trace_read(void* dst, size_t bytes) {
     if (bytes > sizeof(ft2impl::g_trace)) bytes = sizeof(ft2impl::g_trace);
     return (int)cudaMemcpyFromSymbol(dst, ft2impl::g_trace, bytes);

@@ -20,8 +20,9 @@ are not part of the method).  The method itself runs in libft2.so:
   epilogue's cost).
 
 Weights are seeded synthetic (ft2_synth recipe, scaled 2^-ceil(log2 sqrt K));
-no checkpoint is loaded.  Decode steps are captured once into a CUDA graph and
-replayed per token.
+no checkpoint is loaded.  The first-token pass and the decode step are each
+captured once per mode into a CUDA graph (static prompt / token buffers) and
+replayed: one prefill replay and G-1 decode replays per request.
 """
 from __future__ import annotations
 
@@ -176,6 +177,7 @@ class Runner:
                         for _ in range(cfg.n_layers)]
         self.seq_offsets = torch.arange(0, (batch + 1) * prompt_len, prompt_len, dtype=torch.int32, device=dv)
         # decode-step static buffers (CUDA-graph inputs/outputs)
+        self.prompt_static = torch.zeros((batch, prompt_len), dtype=torch.int64, device=dv)
         self.tok = torch.zeros(batch, dtype=torch.int64, device=dv)
         self.pos = torch.zeros(1, dtype=torch.int64, device=dv)
         self.out_tokens = torch.zeros((batch, gen_len), dtype=torch.int64, device=dv)
@@ -360,6 +362,32 @@ class Runner:
             self.tok.copy_(save[0]); self.pos.copy_(save[1]); self.out_tokens.copy_(save[2])
         return self.graphs[key]
 
+    def _prefill_graph(self, mode):
+        """CUDA graph of the whole first-token pass (embedding, 24 blocks with
+        the FT2 bound sweeps on the critical layers, LM head, first token) on
+        the static prompt buffer; one per mode."""
+        key = ("prefill", mode)
+        if key not in self.graphs:
+            self.mode = mode
+            self._site_step = None
+
+            def body():
+                first = self.prefill(self.prompt_static)
+                self.out_tokens[:, 0] = first
+                self.tok.copy_(first)
+                self.pos.fill_(self.T)
+
+            s = torch.cuda.Stream()
+            s.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(s):
+                body()   # warm-up (allocations, cuBLAS/cuDNN plans)
+            torch.cuda.current_stream().wait_stream(s)
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                body()
+            self.graphs[key] = g
+        return self.graphs[key]
+
     def ft2_launches_per_request(self, mode):
         """Library kernels launched by one generate() in `mode` (prefill + decode replays)."""
         if mode == "off":
@@ -378,10 +406,14 @@ class Runner:
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)] if self.time_phases else None
         if ev:
             ev[0].record()
-        first = self.prefill(prompt_ids)
-        self.out_tokens[:, 0] = first
-        self.tok.copy_(first)
-        self.pos.fill_(self.T)
+        if use_graph:
+            self.prompt_static.copy_(prompt_ids, non_blocking=True)
+            self._prefill_graph(mode).replay()
+        else:
+            first = self.prefill(prompt_ids)
+            self.out_tokens[:, 0] = first
+            self.tok.copy_(first)
+            self.pos.fill_(self.T)
         if ev:
             ev[1].record()
         if use_graph:

@@ -6,6 +6,7 @@ import pytest
 import torch
 
 import oracle
+import oracle.stats  # noqa: F401  (submodule used below)
 
 pytestmark = pytest.mark.gpu
 
