@@ -178,6 +178,7 @@ class Runner:
         self.seq_offsets = torch.arange(0, (batch + 1) * prompt_len, prompt_len, dtype=torch.int32, device=dv)
         # decode-step static buffers (CUDA-graph inputs/outputs)
         self.prompt_static = torch.zeros((batch, prompt_len), dtype=torch.int64, device=dv)
+        self.graph_prefill = True   # first-token pass as a CUDA graph (False: eager)
         self.tok = torch.zeros(batch, dtype=torch.int64, device=dv)
         self.pos = torch.zeros(1, dtype=torch.int64, device=dv)
         self.out_tokens = torch.zeros((batch, gen_len), dtype=torch.int64, device=dv)
@@ -406,7 +407,7 @@ class Runner:
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)] if self.time_phases else None
         if ev:
             ev[0].record()
-        if use_graph:
+        if use_graph and self.graph_prefill:
             self.prompt_static.copy_(prompt_ids, non_blocking=True)
             self._prefill_graph(mode).replay()
         else:
