@@ -51,6 +51,15 @@ def parse():
     return ap.parse_args()
 
 
+def load_traffic():
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch from this round's
+    committed ncu --set full capture (profiles/r1_ncu_traffic.json)."""
+    try:
+        return json.load(open(os.path.join(ROOT, "profiles", "r1_ncu_traffic.json")))
+    except Exception:
+        return {}
+
+
 def load_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -373,6 +382,10 @@ def main():
 
     if not args.no_extras:
         res.update(kernel_rooflines(runner, dev, ft2))
+        rf = res["roofline"]
+        dec_us = 1000.0 * phases["fused"]["decode_ms_per_step"]
+        # the kernel's share of a decode step (compare with the ncu launch list in profiles/)
+        rf["share_of_decode_step"] = rf["launches_per_graph"] * rf["avg_launch_us"] / dec_us
     if rank == 0 and world == 1 and not args.no_extras:
         cb = oracle_sample(args.model, B, T, G)
         res["cpu_baseline"] = {"value": cb["tokens_per_s"], "unit": "tokens/s", "cores": cb["cores"],
@@ -439,8 +452,10 @@ def kernel_rooflines(runner, dev, ft2):
                  for x, w, b, y, _ in launches)
     per_launch_us = 1000.0 * ms / len(launches)
     ach = nbytes / (ms / 1e3) / 1e9
+    traffic = load_traffic()
+    gemm_tr = traffic.get("gemm_decode_opt1.3b", {}).get("avg_per_launch_bytes") if runner.cfg.hidden == 2048 else None
     gemm = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
-            "traffic": None, "kernel": "ft2 gemm_kernel (tcgen05, CHECK epilogue)",
+            "traffic": gemm_tr, "traffic_source": traffic.get("source") if gemm_tr else None, "kernel": "ft2 gemm_kernel (tcgen05, CHECK epilogue)",
             "shapes": f"M={B}; (N,K) per block: " + ", ".join(
                 f"{blk_w.shape[0]}x{blk_w.shape[1]}" for blk_w in [runner.blocks[0].w[n] for n in runner.crit_names]),
             "launches_per_graph": len(launches), "avg_launch_us": per_launch_us,
@@ -471,7 +486,8 @@ def kernel_rooflines(runner, dev, ft2):
     nb = rows * n * 2
     prot = {
         "bounds": {"bound": "hbm", "achieved": nb / (ms_b / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
-                   "frac": nb / (ms_b / 1e3) / 1e9 / hbm_peak, "traffic": None, "us": 1000 * ms_b,
+                   "frac": nb / (ms_b / 1e3) / 1e9 / hbm_peak,
+                   "traffic": traffic.get("bounds_65536x11008", {}).get("per_launch_bytes"), "us": 1000 * ms_b,
                    "shape": [rows, n], "algorithmic_bytes": "2 B read per element"},
         "protect": {"bound": "hbm", "achieved": nb / (ms_p / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
                     "frac": nb / (ms_p / 1e3) / 1e9 / hbm_peak, "traffic": None, "us": 1000 * ms_p,
