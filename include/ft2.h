@@ -216,6 +216,40 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
                                   const int32_t* base_row, void* workspace, size_t ws_bytes,
                                   void* stream);
 
+/* The critical linear layer during first-token generation (prefill) with the
+ * first-token bound derivation fused into its GEMM epilogue (SURVEY.md 8(f)
+ * NEXT(1)): PAPER.md L150 (bounds profiled on the first token), L221-L233
+ * (min/max of the layer output, scaling factor 2), L225/L237/L241 (NaN/Inf in
+ * the first token detected and corrected), L272 (after the critical layer).
+ *   y = inject(bf16_rne(x W^T + b))        (as ft2_protect_fused_gemm PLAIN,
+ *                                            faults of step 0 = the prefill)
+ *   then, on y: exactly ft2_bounds_from_prefill(y, seq_offsets, num_seqs,
+ *   scale, finalize = 1, correct_nonfinite, bounds_out, keys_out,
+ *   nonfinite_count, NULL, workspace)
+ * without reading y back: every output tile's per-row key extrema are reduced
+ * per sequence in the epilogue (shared-memory table per CTA, one flush), the
+ * last CTA scales the bounds (R3) and patches the recorded non-finite outputs
+ * (R4).  Bounds, keys and counts are bit-identical to the two-call sequence
+ * (GEMM, then ft2_bounds_from_prefill) on the same inputs.
+ * x [M x K], w [N x K], bias [N] or NULL, y [M x N]: as ft2_protect_fused_gemm.
+ * seq_offsets [num_seqs + 1] (rows outside [seq_offsets[0], seq_offsets[S]) are
+ * padding, reading A18) or NULL for one sequence; scale, correct_nonfinite,
+ * bounds_out, keys_out, nonfinite_count, workspace: as ft2_bounds_from_prefill
+ * (workspace = ft2_workspace_bytes(num_seqs) bytes, zero-filled once, left zero).
+ * sites/n_sites/cur_layer/base_row: faults of step 0 (base_row = seq_offsets).
+ * The GEMM is a persistent 128x256-tile tcgen05 kernel (one CTA per SM, TMEM
+ * double-buffered accumulators); it is also what ft2_protect_fused_gemm runs
+ * for M > 128.  Limits: N % 8 == 0, K % 8 == 0, ld* % 8 == 0, 16-byte aligned
+ * x/w/y, M * N / 8 < 2^31, num_seqs <= FT2_MAX_SEQS.  M == 0: FT2_OK, no launch,
+ * outputs untouched. */
+ft2_status ft2_prefill_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw,
+                                  const void* bias, void* y, int64_t ldy, int32_t M, int32_t N,
+                                  int32_t K, ft2_dtype dtype, const int32_t* seq_offsets,
+                                  int32_t num_seqs, float scale, int32_t correct_nonfinite,
+                                  void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
+                                  const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
+                                  const int32_t* base_row, void* workspace, void* stream);
+
 /* Seeded fault sites for trials [trial0, trial0 + n_trials) (reading R6:
  * Philox4x32-10 keyed by seed, counter = trial id; uniform step, layer, neuron
  * and bit position(s) per PAPER.md L84, L90, L95).  Bit-exact with the CPU

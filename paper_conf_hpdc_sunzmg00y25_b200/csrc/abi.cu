@@ -197,6 +197,61 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
     return finish(e, nl);
 }
 
+ft2_status ft2_prefill_fused_gemm(const void* x, int64_t ldx, const void* w, int64_t ldw, const void* bias, void* y,
+                                  int64_t ldy, int32_t M, int32_t N, int32_t K, ft2_dtype dtype,
+                                  const int32_t* seq_offsets, int32_t num_seqs, float scale, int32_t correct_nonfinite,
+                                  void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
+                                  const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
+                                  const int32_t* base_row, void* workspace, void* stream) {
+    if (M < 0 || N < 0 || K < 0) return FT2_ERR_INVALID_ARG;
+    if (dtype != FT2_BF16 && dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
+    if (num_seqs < 1 || num_seqs > FT2_MAX_SEQS) return num_seqs < 1 ? FT2_ERR_INVALID_ARG : FT2_ERR_UNSUPPORTED;
+    if (!(std::isfinite(scale)) || scale < 1.0f) return FT2_ERR_INVALID_ARG;
+    if (x == nullptr || w == nullptr || y == nullptr || bounds_out == nullptr || workspace == nullptr)
+        return FT2_ERR_INVALID_ARG;
+    if (seq_offsets == nullptr && num_seqs != 1) return FT2_ERR_INVALID_ARG;
+    if (ldx < K || ldw < K || ldy < N) return FT2_ERR_INVALID_ARG;
+    if (n_sites < 0 || (n_sites > 0 && sites == nullptr)) return FT2_ERR_INVALID_ARG;
+    if (!al16(x) || !al16(w) || !al16(y) || (bias && ((uintptr_t)bias & 1u)) || (K % 8) || (N % 8) ||
+        (ldx % 8) || (ldw % 8) || (ldy % 8) || ((uintptr_t)workspace & 7u) || ((uintptr_t)bounds_out & 3u))
+        return FT2_ERR_MISALIGNED;
+    if (M == 0 || N == 0) return FT2_OK;  // as ft2_bounds_from_prefill: nothing to reduce
+    if (K == 0) return FT2_ERR_UNSUPPORTED;
+    if ((int64_t)M * (N / 8) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
+    GemmArgs a = {};
+    a.x = static_cast<const uint16_t*>(x);
+    a.ldx = ldx;
+    a.w = static_cast<const uint16_t*>(w);
+    a.ldw = ldw;
+    a.bias = static_cast<const uint16_t*>(bias);
+    a.y = static_cast<uint16_t*>(y);
+    a.ldy = ldy;
+    a.M = M;
+    a.N = N;
+    a.K = K;
+    a.mode = FT2_GEMM_PLAIN;
+    a.col_begin = 0;
+    a.col_end = N;
+    a.sites = n_sites > 0 ? sites : nullptr;
+    a.n_sites = n_sites;
+    a.cur_layer = cur_layer;
+    a.cur_step = 0;  // the first token (prefill) is step 0 of the fault-site geometry
+    a.base_row = base_row;
+    a.dtype = dtype;
+    PrefillDerive d;
+    d.seq_offsets = seq_offsets;
+    d.S = num_seqs;
+    d.scale = scale;
+    d.correct = correct_nonfinite ? 1 : 0;
+    d.bounds_out = static_cast<uint16_t*>(bounds_out);
+    d.keys_out = keys_out;
+    d.nonfinite_out = nonfinite_count;
+    d.ws = static_cast<uint32_t*>(workspace);
+    int nl = 0;
+    cudaError_t e = launch_prefill_gemm(a, &d, static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
 ft2_status ft2_make_fault_sites(uint64_t seed, uint64_t trial0, int32_t n_trials, ft2_fault_model model,
                                 ft2_dtype dtype, const ft2_site_geometry* geom, ft2_fault_site* sites_out,
                                 void* stream) {

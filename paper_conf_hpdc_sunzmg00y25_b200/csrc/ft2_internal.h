@@ -75,6 +75,21 @@ struct GemmArgs {
 size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch);
 
+// First-token bound derivation fused into the prefill GEMM epilogue
+// (ft2_prefill_fused_gemm): the ft2_bounds_from_prefill outputs, finalize = 1.
+struct PrefillDerive {
+    const int32_t* seq_offsets;  // [S + 1] or NULL (one sequence)
+    int32_t S;
+    float scale;
+    int32_t correct;
+    uint16_t* bounds_out;
+    int32_t* keys_out;
+    uint32_t* nonfinite_out;
+    uint32_t* ws;  // bounds workspace (bounds_ws_bytes(S))
+};
+// Persistent 128x256-tile tcgen05 GEMM for M > 128 (PLAIN / CHECK, or DERIVE when d != NULL)
+cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaStream_t st, int* n_launch);
+
 int num_sms();
 
 }  // namespace ft2impl

@@ -1,0 +1,472 @@
+// gemm_prefill_sm100.cu -- a critical linear layer at prefill shapes (M = sum
+// of prompt lengths > 128 tokens) with FT2's first-token work fused into the
+// epilogue, for sm_100a.
+//
+//   PLAIN   y = inject(bf16_rne(x W^T + b))
+//   CHECK   ... then check-and-clip against the row's sequence bounds (R5)
+//   DERIVE  ... then the first-token bounds of y: per sequence the min/max
+//           order key over the finite outputs (R2), combined across tiles and
+//           CTAs, widened x scale by the last CTA (R3), which also corrects the
+//           recorded non-finite outputs (R4) -- ft2_bounds_from_prefill on the
+//           layer output without reading it back from HBM.
+// PAPER.md L150 (bounds from the first token), L221-L233 (min/max, scaling
+// factor 2), L225/L237/L241 (NaN in the first token is detected and
+// corrected), L259/L272 (check after the critical layer).  Order of the
+// epilogue: GEMM -> +bias -> bf16 -> inject -> check / derive (A19, A20).
+//
+// Persistent, warp-specialised, one CTA per SM (192 threads):
+//   warp 0      TMA producer: 128x64 A (x) and 256x64 B (W) boxes, 128B
+//               swizzle, into a 4-stage ring (48 KB per stage).
+//   warp 1      TMEM allocator (512 columns = two 128x256 fp32 accumulators)
+//               and the single-thread tcgen05.mma.cta_group::1.kind::f16
+//               issuer (M=128, N=256, K=16).
+//   warps 2-5   epilogue: tcgen05.ld 32 columns at a time (one TMEM lane =
+//               one output row per thread), while the MMA warp fills the other
+//               accumulator with the next tile (TMEM double buffering).
+// Tiles are 128 x 256, handed out round-robin (tile = blockIdx.x + i * grid).
+// DERIVE keeps a per-CTA table of the sequences' key extrema in shared memory
+// (warp-reduced when a warp's 32 rows belong to one sequence) and flushes it
+// once; the bounds workspace protocol is the one of ft2_bounds_from_prefill
+// (bounds_common.cuh), so both produce bit-identical bounds.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+#include <stdlib.h>
+
+#include "bounds_common.cuh"
+#include "ft2_device.cuh"
+#include "ft2_internal.h"
+#include "sm100_ptx.cuh"
+
+namespace ft2impl {
+using namespace ft2dev;
+
+constexpr int kPBM = 128, kPBN = 256, kPBK = 64, kPStages = 4, kPThreads = 192;
+constexpr int kPABytes = kPBM * kPBK * 2;            // 16 KB
+constexpr int kPBBytes = kPBN * kPBK * 2;            // 32 KB
+constexpr int kPStageBytes = kPABytes + kPBBytes;    // 48 KB
+constexpr int kPTileBytes = kPStages * kPStageBytes;  // 192 KB
+constexpr int kPSeqTab = 512;                        // sequences kept in the per-CTA table
+constexpr int kPMaxRowSites = 4;                     // fault sites one row may hold per tile
+constexpr int kPMiscBytes = 256;
+constexpr int kPSmemBytes = 1024 + kPTileBytes + kPMiscBytes + 3 * kPSeqTab * 4;
+constexpr int kPGemmDerive = 2;
+
+struct PrefK {
+    int32_t M, N, K, tilesM, ntiles, nkb;
+    int32_t mode, col_begin, col_end;
+    const uint16_t* bias;
+    uint16_t* y;
+    int64_t ldy;
+    // CHECK: row -> sequence as in ft2_protect
+    const int32_t* row_to_seq;
+    int32_t S, row_mode;
+    const uint16_t* bounds;
+    uint32_t* counts;
+    // DERIVE: the ft2_bounds_from_prefill arguments (finalize = 1)
+    BoundsK bp;
+    // faults
+    const ft2_fault_site* sites;
+    int32_t n_sites, cur_layer, cur_step;
+    const int32_t* base_row;
+};
+
+__device__ __forceinline__ uint32_t pack_rne2(float a, float b, int dt) {
+    return dt == 1 ? ((uint32_t)rne16<1>(a) | ((uint32_t)rne16<1>(b) << 16))
+                   : ((uint32_t)rne16<0>(a) | ((uint32_t)rne16<0>(b) << 16));
+}
+
+template <int DT>
+__global__ void __launch_bounds__(kPThreads, 1)
+    prefill_gemm_kernel(const __grid_constant__ CUtensorMap map_x, const __grid_constant__ CUtensorMap map_w,
+                        const __grid_constant__ PrefK p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+    uint8_t* tiles = smem;
+    uint8_t* misc = smem + kPTileBytes;
+    uint64_t* full = reinterpret_cast<uint64_t*>(misc);
+    uint64_t* empty = full + kPStages;
+    uint64_t* tmem_full = empty + kPStages;  // [2]
+    uint64_t* tmem_empty = tmem_full + 2;    // [2]
+    uint32_t* tmem_base_sh = reinterpret_cast<uint32_t*>(tmem_empty + 2);
+    uint32_t* last_sh = tmem_base_sh + 1;
+    uint32_t* tab_lo = reinterpret_cast<uint32_t*>(misc + kPMiscBytes);  // 0x10000 - min key (0: none)
+    uint32_t* tab_hi = tab_lo + kPSeqTab;                                 // max key + 1 (0: none)
+    uint32_t* tab_nf = tab_hi + kPSeqTab;                                 // non-finite count
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const bool derive = p.mode == kPGemmDerive;
+    const bool use_tab = derive && p.bp.S <= kPSeqTab;
+    if (warp == 0 && lane == 0) {
+        prefetch_tmap(&map_x);
+        prefetch_tmap(&map_w);
+        for (int s = 0; s < kPStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+        for (int b = 0; b < 2; ++b) { mbar_init(&tmem_full[b], 1); mbar_init(&tmem_empty[b], 4); }
+        fence_mbar_init();
+    }
+    if (warp == 1) tmem_alloc(tmem_base_sh, 512);
+    if (use_tab)
+        for (int s = tid; s < p.bp.S; s += kPThreads) { tab_lo[s] = 0u; tab_hi[s] = 0u; tab_nf[s] = 0u; }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_base_sh;
+    griddep_launch();
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---------------------------------------------------- TMA producer
+            griddep_wait();  // x may be the previous kernel's output
+            uint32_t stage = 0, phase = 0;
+            for (int t = blockIdx.x; t < p.ntiles; t += gridDim.x) {
+                const int m0 = (t % p.tilesM) * kPBM, n0 = (t / p.tilesM) * kPBN;
+                for (int kb = 0; kb < p.nkb; ++kb) {
+                    mbar_wait(&empty[stage], phase ^ 1u);
+                    uint8_t* st = tiles + stage * kPStageBytes;
+                    mbar_expect_tx(&full[stage], kPStageBytes);
+                    tma_load_2d(&map_x, &full[stage], st, kb * kPBK, m0);
+                    tma_load_2d(&map_w, &full[stage], st + kPABytes, kb * kPBK, n0);
+                    if (++stage == kPStages) { stage = 0; phase ^= 1u; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ----------------------------------------------------- MMA issuer
+            constexpr uint32_t idesc =
+                (make_idesc(kPBM, kPBN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
+            uint32_t stage = 0, phase = 0;
+            int tc = 0;
+            for (int t = blockIdx.x; t < p.ntiles; t += gridDim.x, ++tc) {
+                const int buf = tc & 1;
+                mbar_wait(&tmem_empty[buf], ((uint32_t)(tc >> 1) & 1u) ^ 1u);  // the epilogue drained it
+                tc_fence_after();
+                const uint32_t d = tmem_base + (uint32_t)(buf * kPBN);
+                for (int kb = 0; kb < p.nkb; ++kb) {
+                    mbar_wait(&full[stage], phase);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(tiles + stage * kPStageBytes);
+                    const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + kPABytes);
+#pragma unroll
+                    for (int k = 0; k < kPBK / 16; ++k)
+                        tc_mma(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                    tc_commit(&empty[stage]);
+                    if (++stage == kPStages) { stage = 0; phase ^= 1u; }
+                }
+                tc_commit(&tmem_full[buf]);
+            }
+        }
+    } else {
+        // --------------------------------------------------------- epilogue
+        const int q = warp & 3;  // TMEM lane quarter of this warp
+        const int e = q * 32 + lane;
+        griddep_wait();  // bias / bounds / sites / y may belong to the previous kernel
+        uint32_t* ws_lc = p.bp.ws + 4 * p.bp.S + 1;
+        uint32_t* ws_ov = p.bp.ws + 4 * p.bp.S + 2;
+        unsigned long long* list = reinterpret_cast<unsigned long long*>(
+            reinterpret_cast<char*>(p.bp.ws) + (((size_t)(4 * p.bp.S + 4) * 4 + 7) & ~(size_t)7));
+        int tc = 0;
+        for (int t = blockIdx.x; t < p.ntiles; t += gridDim.x, ++tc) {
+            const int buf = tc & 1;
+            const int m0 = (t % p.tilesM) * kPBM, n0 = (t / p.tilesM) * kPBN;
+            const int m = m0 + e;
+            const bool row_ok = m < p.M;
+            // row information (independent of the accumulator)
+            int seq = -1;
+            uint32_t kL2 = 0u, kH2 = 0xFFFFFFFFu;
+            if (row_ok) {
+                if (derive) {
+                    seq = p.bp.seq_offsets ? seq_of_row(p.bp.seq_offsets, p.bp.S, (uint32_t)m) : 0;
+                    if (seq >= p.bp.S) seq = -1;  // padding rows after the last sequence (A18)
+                } else if (p.mode == FT2_GEMM_CHECK) {
+                    const int s = p.row_mode == 2 ? 0 : (p.row_mode == 1 ? m : p.row_to_seq[m]);
+                    if (s >= 0 && s < p.S) {
+                        const uint32_t k = key2((uint32_t)p.bounds[2 * s] | ((uint32_t)p.bounds[2 * s + 1] << 16));
+                        kL2 = (k & 0xFFFFu) * 0x10001u;
+                        kH2 = (k >> 16) * 0x10001u;
+                        seq = s;
+                    }
+                }
+            }
+            // fault sites of this row inside this tile (fault-injection runs only)
+            uint32_t site_c[kPMaxRowSites], site_m[kPMaxRowSites];
+            int nsite = 0;
+            if (p.sites != nullptr && row_ok) {
+                for (int i = 0; i < p.n_sites; ++i) {
+                    const ft2_fault_site st = p.sites[i];
+                    if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
+                    const int64_t r = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
+                                      (p.cur_step == 0 ? (int64_t)st.token : 0);
+                    const int64_t c = (int64_t)st.col - n0;
+                    if (r == m && c >= 0 && c < kPBN && (int64_t)st.col < p.N && nsite < kPMaxRowSites) {
+                        site_c[nsite] = (uint32_t)c;
+                        site_m[nsite] = st.xor_mask & 0xFFFFu;
+                        ++nsite;
+                    }
+                }
+            }
+            uint32_t mn2 = 0xFFFFFFFFu, mx2 = 0u, ncorr = 0u;
+            mbar_wait(&tmem_full[buf], (uint32_t)(tc >> 1) & 1u);
+            tc_fence_after();
+            const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * kPBN);
+            uint16_t* yrow = p.y + (int64_t)m * p.ldy;
+#pragma unroll 1
+            for (int c0 = 0; c0 < kPBN; c0 += 32) {
+                uint32_t r[32];
+                tmem_ld32(taddr + (uint32_t)c0, r);
+                tmem_wait_ld();
+                const int nb = n0 + c0;
+                if (!row_ok || nb >= p.N) continue;
+                const int nvalid = min(32, p.N - nb);
+                // bias (the same 32 values for every thread: broadcast loads)
+                float bv[32];
+                if (p.bias) {
+                    const uint4* bq = reinterpret_cast<const uint4*>(p.bias + nb);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        uint4 u = nvalid == 32 ? __ldg(bq + j) : make_uint4(0u, 0u, 0u, 0u);
+                        if (nvalid < 32) {
+                            uint32_t tmp[4] = {0u, 0u, 0u, 0u};
+                            for (int h = 0; h < 8; ++h)
+                                if (j * 8 + h < nvalid) tmp[h >> 1] |= (uint32_t)p.bias[nb + j * 8 + h] << ((h & 1) * 16);
+                            u = make_uint4(tmp[0], tmp[1], tmp[2], tmp[3]);
+                        }
+                        const uint32_t uw[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+                        for (int h = 0; h < 4; ++h) {
+                            bv[j * 8 + 2 * h] = to_f32<DT>((uint16_t)(uw[h] & 0xFFFFu));
+                            bv[j * 8 + 2 * h + 1] = to_f32<DT>((uint16_t)(uw[h] >> 16));
+                        }
+                    }
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) bv[j] = 0.f;
+                }
+                uint32_t w[16];
+#pragma unroll
+                for (int j = 0; j < 16; ++j)
+                    w[j] = pack_rne2(__uint_as_float(r[2 * j]) + bv[2 * j], __uint_as_float(r[2 * j + 1]) + bv[2 * j + 1], DT);
+                for (int i = 0; i < nsite; ++i) {
+                    const uint32_t d = site_c[i] - (uint32_t)c0;
+                    if (d < 32u) {
+#pragma unroll
+                        for (int j = 0; j < 16; ++j)
+                            if ((d >> 1) == (uint32_t)j) w[j] ^= site_m[i] << ((d & 1u) * 16);
+                    }
+                }
+                if (p.mode == FT2_GEMM_CHECK && seq >= 0) {
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) {
+                        const int c = nb + 2 * j;
+                        const uint32_t pm = ((c >= p.col_begin && c < p.col_end) ? 0x0000FFFFu : 0u) |
+                                            ((c + 1 >= p.col_begin && c + 1 < p.col_end) ? 0xFFFF0000u : 0u);
+                        uint32_t ch = 0u;
+                        const uint32_t o = clip2<DT>(w[j], kL2, kH2, &ch);
+                        const uint32_t nw = (o & pm) | (w[j] & ~pm);
+                        ncorr += nonzero_halves(nw ^ w[j]);
+                        w[j] = nw;
+                    }
+                }
+                if (derive) {
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) {
+                        // columns beyond N must not contribute: neutral keys
+                        const uint32_t k = key2(w[j]);
+                        const uint32_t kmn = 2 * j + 1 < nvalid ? k : (2 * j < nvalid ? (k | 0xFFFF0000u) : 0xFFFFFFFFu);
+                        const uint32_t kmx = 2 * j + 1 < nvalid ? k : (2 * j < nvalid ? (k & 0x0000FFFFu) : 0u);
+                        mn2 = vmin_u16x2(mn2, kmn);
+                        mx2 = vmax_u16x2(mx2, kmx);
+                    }
+                }
+                if (nvalid == 32 && ((reinterpret_cast<uintptr_t>(yrow + nb) & 15u) == 0)) {
+                    uint4* dst = reinterpret_cast<uint4*>(yrow + nb);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) dst[j] = make_uint4(w[4 * j], w[4 * j + 1], w[4 * j + 2], w[4 * j + 3]);
+                } else {
+                    for (int j = 0; j < nvalid; ++j) yrow[nb + j] = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
+                }
+            }
+            // accumulator buffer drained: hand it back to the MMA warp
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&tmem_empty[buf]);
+            if (p.mode == FT2_GEMM_CHECK && ncorr != 0u && p.counts != nullptr && seq >= 0)
+                atomicAdd(&p.counts[seq], ncorr);
+            if (derive) {
+                uint32_t kmin = min(mn2 & 0xFFFFu, mn2 >> 16), kmax = max(mx2 & 0xFFFFu, mx2 >> 16);
+                uint32_t nf = 0u;
+                if (seq >= 0 && (kmin < Fmt<DT>::kKeyLo || kmax > Fmt<DT>::kKeyHi)) {
+                    // a non-finite output in this row segment: exact pass over
+                    // what this thread just stored (rare; R2 excludes it, R4 patches it)
+                    kmin = 0xFFFFu;
+                    kmax = 0u;
+                    const int nend = min(p.N, n0 + kPBN);
+                    for (int n = n0; n < nend; ++n) {
+                        const uint16_t b = yrow[n];
+                        if (nonfinite1<DT>(b)) {
+                            ++nf;
+                            if (p.bp.correct)
+                                record_patch(p.bp, ws_lc, ws_ov, list, seq, (uint64_t)((int64_t)m * p.ldy + n));
+                        } else {
+                            const uint32_t k = key1(b);
+                            kmin = min(kmin, k);
+                            kmax = max(kmax, k);
+                        }
+                    }
+                }
+                if (seq < 0) { kmin = 0xFFFFu + 1u; kmax = 0u; }
+                // one sequence across the warp's 32 rows (the common case): warp-reduce first
+                const int seq0 = __shfl_sync(0xFFFFFFFFu, seq, 0);
+                const bool uni = __all_sync(0xFFFFFFFFu, seq == seq0);
+                if (uni) {
+                    kmin = __reduce_min_sync(0xFFFFFFFFu, kmin);
+                    kmax = __reduce_max_sync(0xFFFFFFFFu, kmax);
+                    nf = __reduce_add_sync(0xFFFFFFFFu, nf);
+                }
+                if ((!uni || lane == 0) && seq >= 0) {
+                    const bool have = kmin <= kmax;
+                    if (use_tab) {
+                        if (have) {
+                            atomicMax(&tab_lo[seq], 0x10000u - kmin);
+                            atomicMax(&tab_hi[seq], kmax + 1u);
+                        }
+                        if (nf) atomicAdd(&tab_nf[seq], nf);
+                    } else {
+                        if (have) {
+                            atomicMax(&p.bp.ws[4 * seq + 0], 0x10000u - kmin);
+                            atomicMax(&p.bp.ws[4 * seq + 1], kmax + 1u);
+                        }
+                        if (nf) atomicAdd(&p.bp.ws[4 * seq + 2], nf);
+                    }
+                }
+            }
+        }
+    }
+
+    // ----------------------------------------------------------- teardown
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 1) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, 512);
+    }
+    if (!derive) return;
+    if (use_tab) {
+        for (int s = tid; s < p.bp.S; s += kPThreads) {
+            if (tab_lo[s]) atomicMax(&p.bp.ws[4 * s + 0], tab_lo[s]);
+            if (tab_hi[s]) atomicMax(&p.bp.ws[4 * s + 1], tab_hi[s]);
+            if (tab_nf[s]) atomicAdd(&p.bp.ws[4 * s + 2], tab_nf[s]);
+        }
+    }
+    // grid combine: the last CTA finalises (release covers this CTA's REDs and
+    // patch records through the barrier; acquire for the last CTA)
+    __syncthreads();
+    if (tid == 0) *last_sh = atom_add_acq_rel_gpu(p.bp.ws + 4 * p.bp.S, 1u) == gridDim.x - 1 ? 1u : 0u;
+    __syncthreads();
+    if (*last_sh) bounds_finalize_tail<DT, false>(p.bp, tid, kPThreads);
+}
+
+// ---------------------------------------------------------------- host side
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+        void* ptr = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+        return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    }();
+    return fn;
+}
+
+static bool make_map_p(CUtensorMap* m, const void* base, int64_t rows, int64_t K, int64_t ld, int box_rows, int dt) {
+    auto enc = encode_fn();
+    if (!enc) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * 2)};
+    cuuint32_t box[2] = {(cuuint32_t)kPBK, (cuuint32_t)box_rows};
+    cuuint32_t es[2] = {1, 1};
+    return enc(m, dt == FT2_FP16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+               const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <int DT>
+static cudaError_t launch_prefill_dt(const CUtensorMap& mx, const CUtensorMap& mw, const PrefK& p, int grid,
+                                     cudaStream_t st) {
+    static cudaError_t attr = cudaFuncSetAttribute(prefill_gemm_kernel<DT>,
+                                                   cudaFuncAttributeMaxDynamicSharedMemorySize, kPSmemBytes);
+    if (attr != cudaSuccess) return attr;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(kPThreads);
+    cfg.dynamicSmemBytes = kPSmemBytes;
+    cfg.stream = st;
+    cudaLaunchAttribute a[1];
+    a[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    a[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = a;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, prefill_gemm_kernel<DT>, mx, mw, p);
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaStream_t st, int* n_launch) {
+    CUtensorMap mx, mw;
+    if (!make_map_p(&mx, a.x, a.M, a.K, a.ldx, kPBM, a.dtype)) return cudaErrorInvalidValue;
+    if (!make_map_p(&mw, a.w, a.N, a.K, a.ldw, kPBN, a.dtype)) return cudaErrorInvalidValue;
+    PrefK p = {};
+    p.M = a.M;
+    p.N = a.N;
+    p.K = a.K;
+    p.tilesM = (a.M + kPBM - 1) / kPBM;
+    p.ntiles = p.tilesM * ((a.N + kPBN - 1) / kPBN);
+    p.nkb = (a.K + kPBK - 1) / kPBK;
+    p.mode = d ? kPGemmDerive : a.mode;
+    p.col_begin = a.col_begin;
+    p.col_end = a.col_end;
+    p.bias = a.bias;
+    p.y = a.y;
+    p.ldy = a.ldy;
+    p.row_to_seq = a.row_to_seq;
+    p.S = a.S;
+    p.row_mode = a.row_to_seq ? 0 : (a.S == 1 ? 2 : 1);
+    p.bounds = a.bounds;
+    p.counts = a.counts;
+    p.sites = a.sites;
+    p.n_sites = a.sites ? a.n_sites : 0;
+    p.cur_layer = a.cur_layer;
+    p.cur_step = a.cur_step;
+    p.base_row = a.base_row;
+    BoundsK& b = p.bp;
+    b.y = a.y;
+    b.ld = a.ldy;
+    b.n8 = (uint32_t)(a.N / 8);
+    b.total_vec = (uint32_t)((int64_t)a.M * (a.N / 8));
+    b.chunk = 0;
+    b.div_n8 = make_fastdiv(b.n8 > 0 ? b.n8 : 1);
+    b.contiguous = a.ldy == a.N;
+    if (d) {
+        b.seq_offsets = d->seq_offsets;
+        b.S = d->S;
+        b.scale = d->scale;
+        b.finalize = 1;
+        b.correct = d->correct;
+        b.bounds_out = d->bounds_out;
+        b.keys_out = d->keys_out;
+        b.nonfinite_out = d->nonfinite_out;
+        b.nv_out = nullptr;
+        b.ws = d->ws;
+    } else {
+        b.S = 0;
+        b.ws = nullptr;
+    }
+    const int grid = p.ntiles < num_sms() ? p.ntiles : num_sms();
+    cudaError_t e = a.dtype == FT2_FP16 ? launch_prefill_dt<1>(mx, mw, p, grid, st)
+                                        : launch_prefill_dt<0>(mx, mw, p, grid, st);
+    ++*n_launch;
+    return e;
+}
+
+}  // namespace ft2impl

@@ -698,6 +698,8 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
 }
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
+    // prefill shapes (M > 128 tokens): the persistent 128x256 kernel (gemm_prefill_sm100.cu)
+    if (a.M > 128) return launch_prefill_gemm(a, nullptr, st, n_launch);
     const GemmPlan g = plan_gemm(a.M, a.N, a.K);
     GemmK p = {};
     p.M = a.M;
@@ -743,7 +745,6 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
         }
     }
     if (a.dtype == FT2_FP16) {
-        if (!g.swap) return launch_cfg<128, false, 1>(a, p, st, n_launch);
         switch (g.bn) {
             case 16: return launch_cfg<16, true, 1>(a, p, st, n_launch);
             case 32: return launch_cfg<32, true, 1>(a, p, st, n_launch);
@@ -751,7 +752,6 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
             default: return launch_cfg<128, true, 1>(a, p, st, n_launch);
         }
     }
-    if (!g.swap) return launch_cfg<128, false, 0>(a, p, st, n_launch);
     switch (g.bn) {
         case 16: return launch_cfg<16, true, 0>(a, p, st, n_launch);
         case 32: return launch_cfg<32, true, 0>(a, p, st, n_launch);

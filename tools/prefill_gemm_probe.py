@@ -21,7 +21,7 @@ for M, N, K in shapes:
     bnd = torch.zeros((B, 2), dtype=torch.bfloat16, device="cuda")
     wsp = ft2.make_workspace(B)
     out = {"M": M, "N": N, "K": K}
-    for kind in ("cublas", "ft2_plain", "cublas+bounds"):
+    for kind in ("cublas", "ft2_plain", "cublas+bounds", "ft2_derive"):
         def run():
             for i in range(R):
                 w = ws[i % 4]
@@ -29,6 +29,8 @@ for M, N, K in shapes:
                     torch.addmm(b, x, w.t(), out=y)
                     if kind == "cublas+bounds":
                         ft2.bounds_from_prefill(y, bnd, wsp, seq_offsets=so, num_seqs=B, correct_nonfinite=True)
+                elif kind == "ft2_derive":
+                    ft2.prefill_fused_gemm(x, w, y, bnd, wsp, bias=b, seq_offsets=so, num_seqs=B)
                 else:
                     ft2.protect_fused_gemm(x, w, y, bias=b, mode=0)
         run(); torch.cuda.synchronize()
