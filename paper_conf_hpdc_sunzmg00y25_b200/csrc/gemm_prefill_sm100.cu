@@ -41,11 +41,17 @@
 namespace ft2impl {
 using namespace ft2dev;
 
-constexpr int kPBM = 128, kPBN = 256, kPBK = 64, kPStages = 4, kPThreads = 192;
-constexpr int kPABytes = kPBM * kPBK * 2;            // 16 KB
-constexpr int kPBBytes = kPBN * kPBK * 2;            // 32 KB
-constexpr int kPStageBytes = kPABytes + kPBBytes;    // 48 KB
-constexpr int kPTileBytes = kPStages * kPStageBytes;  // 192 KB
+constexpr int kPBM = 128, kPBN = 256, kPBK = 64, kPThreads = 192;
+constexpr int kPABytes = kPBM * kPBK * 2;  // 16 KB: one CTA's 128 rows of x
+constexpr int kPTileBytes = 192 * 1024;    // the shared-memory ring
+// MC = 1: a CTA loads the whole 256-row weight box (48 KB stages, 4 deep);
+// MC = 2: CTA pair, each CTA loads 128 weight rows (32 KB stages, 6 deep)
+template <int MC>
+struct PCfg {
+    static constexpr int kBBytes = kPBN / MC * kPBK * 2;
+    static constexpr int kStageBytes = kPABytes + kBBytes;
+    static constexpr int kStages = kPTileBytes / kStageBytes;
+};
 constexpr int kPSeqTab = 512;                        // sequences kept in the per-CTA table
 constexpr int kPMaxRowSites = 4;                     // fault sites one row may hold per tile
 constexpr int kPMiscBytes = 256;
@@ -76,7 +82,31 @@ __device__ __forceinline__ uint32_t pack_rne2(float a, float b, int dt) {
                    : ((uint32_t)rne16<0>(a) | ((uint32_t)rne16<0>(b) << 16));
 }
 
-template <int DT>
+// Tile of the CTA at step i of the persistent loop.  MC == 2: a cluster of two
+// CTAs (an SM pair) computes a 256 x 256 tile with tcgen05.mma.cta_group::2:
+// CTA r holds rows [128 r, 128 r + 128) of the x box and of the weight box,
+// the leader (rank 0) issues the MMA over both, and each CTA's TMEM receives
+// its own 128 output rows x 256 columns -- the weight box is read from L2 and
+// staged in shared memory once per pair.
+template <int MC>
+__device__ __forceinline__ bool tile_of(const PrefK& p, int i, int& m0, int& n0) {
+    if (MC == 1) {
+        const int t = blockIdx.x + i * gridDim.x;
+        if (t >= p.ntiles) return false;
+        m0 = (t % p.tilesM) * kPBM;
+        n0 = (t / p.tilesM) * kPBN;
+        return true;
+    }
+    const int pairsM = (p.tilesM + 1) >> 1;
+    const int npairs = pairsM * (p.ntiles / p.tilesM);
+    const int pr = (int)(blockIdx.x >> 1) + i * (int)(gridDim.x >> 1);
+    if (pr >= npairs) return false;
+    m0 = ((pr % pairsM) * 2 + (int)(blockIdx.x & 1)) * kPBM;
+    n0 = (pr / pairsM) * kPBN;
+    return true;
+}
+
+template <int DT, int MC>
 __global__ void __launch_bounds__(kPThreads, 1)
     prefill_gemm_kernel(const __grid_constant__ CUtensorMap map_x, const __grid_constant__ CUtensorMap map_w,
                         const __grid_constant__ PrefK p) {
@@ -84,6 +114,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     uint8_t* tiles = smem;
     uint8_t* misc = smem + kPTileBytes;
+    constexpr int kPStages = PCfg<MC>::kStages, kPStageBytes = PCfg<MC>::kStageBytes;
     uint64_t* full = reinterpret_cast<uint64_t*>(misc);
     uint64_t* empty = full + kPStages;
     uint64_t* tmem_full = empty + kPStages;  // [2]
@@ -100,17 +131,28 @@ __global__ void __launch_bounds__(kPThreads, 1)
     if (warp == 0 && lane == 0) {
         prefetch_tmap(&map_x);
         prefetch_tmap(&map_w);
+        // MC = 2: the leader's full[] counts both CTAs' bytes, its tmem_empty[]
+        // both CTAs' epilogue warps; empty[] / tmem_full[] are signalled in
+        // both CTAs by the leader's multicast commits
         for (int s = 0; s < kPStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-        for (int b = 0; b < 2; ++b) { mbar_init(&tmem_full[b], 1); mbar_init(&tmem_empty[b], 4); }
+        for (int b = 0; b < 2; ++b) { mbar_init(&tmem_full[b], 1); mbar_init(&tmem_empty[b], 4 * MC); }
         fence_mbar_init();
     }
-    if (warp == 1) tmem_alloc(tmem_base_sh, 512);
+    if (warp == 1) {
+        if (MC == 1) tmem_alloc(tmem_base_sh, 512);
+        else tmem_alloc2(tmem_base_sh, 512);
+    }
     if (use_tab)
         for (int s = tid; s < p.bp.S; s += kPThreads) { tab_lo[s] = 0u; tab_hi[s] = 0u; tab_nf[s] = 0u; }
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
+    if (MC > 1) {  // the peer's barriers are initialised before anything signals them
+        cluster_arrive_relaxed();
+        cluster_wait();
+    }
     const uint32_t tmem_base = *tmem_base_sh;
+    const uint32_t crank = MC > 1 ? cluster_ctarank() : 0u;
     griddep_launch();
 
     if (warp == 0) {
@@ -118,26 +160,39 @@ __global__ void __launch_bounds__(kPThreads, 1)
             // ---------------------------------------------------- TMA producer
             griddep_wait();  // x may be the previous kernel's output
             uint32_t stage = 0, phase = 0;
-            for (int t = blockIdx.x; t < p.ntiles; t += gridDim.x) {
-                const int m0 = (t % p.tilesM) * kPBM, n0 = (t / p.tilesM) * kPBN;
+            int m0, n0;
+            for (int i = 0; tile_of<MC>(p, i, m0, n0); ++i) {
                 for (int kb = 0; kb < p.nkb; ++kb) {
                     mbar_wait(&empty[stage], phase ^ 1u);
                     uint8_t* st = tiles + stage * kPStageBytes;
-                    mbar_expect_tx(&full[stage], kPStageBytes);
-                    tma_load_2d(&map_x, &full[stage], st, kb * kPBK, m0);
-                    tma_load_2d(&map_w, &full[stage], st + kPABytes, kb * kPBK, n0);
+                    if (MC == 1) {
+                        mbar_expect_tx(&full[stage], kPStageBytes);
+                        tma_load_2d(&map_x, &full[stage], st, kb * kPBK, m0);
+                        tma_load_2d(&map_w, &full[stage], st + kPABytes, kb * kPBK, n0);
+                    } else {  // my 128 rows of x and of the weight box; the leader's barrier counts both CTAs
+                        const uint32_t lbar = mapa(smem_u32(&full[stage]), 0u);
+                        if (crank == 0) mbar_expect_tx(&full[stage], 2 * kPStageBytes);
+                        tma_load_2d_2sm(&map_x, lbar, st, kb * kPBK, m0);
+                        tma_load_2d_2sm(&map_w, lbar, st + kPABytes, kb * kPBK, n0 + (int)crank * (kPBN / 2));
+                    }
+                    if (++stage == kPStages) { stage = 0; phase ^= 1u; }
+                }
+            }
+            if (MC > 1) {  // drain: every stage's release has arrived before the CTA may exit
+                for (int s = 0; s < kPStages; ++s) {
+                    mbar_wait(&empty[stage], phase ^ 1u);
                     if (++stage == kPStages) { stage = 0; phase ^= 1u; }
                 }
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
-            // ----------------------------------------------------- MMA issuer
+        if (lane == 0 && crank == 0) {
+            // ----------------------------------------- MMA issuer (the pair's leader)
             constexpr uint32_t idesc =
-                (make_idesc(kPBM, kPBN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
+                (make_idesc(kPBM * MC, kPBN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
             uint32_t stage = 0, phase = 0;
-            int tc = 0;
-            for (int t = blockIdx.x; t < p.ntiles; t += gridDim.x, ++tc) {
+            int tc = 0, m0, n0;
+            for (int i = 0; tile_of<MC>(p, i, m0, n0); ++i, ++tc) {
                 const int buf = tc & 1;
                 mbar_wait(&tmem_empty[buf], ((uint32_t)(tc >> 1) & 1u) ^ 1u);  // the epilogue drained it
                 tc_fence_after();
@@ -148,12 +203,18 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     const uint32_t sa = smem_u32(tiles + stage * kPStageBytes);
                     const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + kPABytes);
 #pragma unroll
-                    for (int k = 0; k < kPBK / 16; ++k)
-                        tc_mma(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > 0 || k > 0) ? 1u : 0u);
-                    tc_commit(&empty[stage]);
+                    for (int k = 0; k < kPBK / 16; ++k) {
+                        if (MC == 1)
+                            tc_mma(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                        else
+                            tc_mma2(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                    }
+                    if (MC == 1) tc_commit(&empty[stage]);
+                    else tc_commit2_mc(&empty[stage], (uint16_t)3u);  // both producers may refill it
                     if (++stage == kPStages) { stage = 0; phase ^= 1u; }
                 }
-                tc_commit(&tmem_full[buf]);
+                if (MC == 1) tc_commit(&tmem_full[buf]);
+                else tc_commit2_mc(&tmem_full[buf], (uint16_t)3u);  // both CTAs' epilogues
             }
         }
     } else {
@@ -165,10 +226,9 @@ __global__ void __launch_bounds__(kPThreads, 1)
         uint32_t* ws_ov = p.bp.ws + 4 * p.bp.S + 2;
         unsigned long long* list = reinterpret_cast<unsigned long long*>(
             reinterpret_cast<char*>(p.bp.ws) + (((size_t)(4 * p.bp.S + 4) * 4 + 7) & ~(size_t)7));
-        int tc = 0;
-        for (int t = blockIdx.x; t < p.ntiles; t += gridDim.x, ++tc) {
+        int tc = 0, m0, n0;
+        for (int i = 0; tile_of<MC>(p, i, m0, n0); ++i, ++tc) {
             const int buf = tc & 1;
-            const int m0 = (t % p.tilesM) * kPBM, n0 = (t / p.tilesM) * kPBN;
             const int m = m0 + e;
             const bool row_ok = m < p.M;
             // row information (independent of the accumulator)
@@ -286,10 +346,13 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     for (int j = 0; j < nvalid; ++j) yrow[nb + j] = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
                 }
             }
-            // accumulator buffer drained: hand it back to the MMA warp
+            // accumulator buffer drained: hand it back to the MMA warp (the leader's)
             tc_fence_before();
             __syncwarp();
-            if (lane == 0) mbar_arrive(&tmem_empty[buf]);
+            if (lane == 0) {
+                if (MC == 1) mbar_arrive(&tmem_empty[buf]);
+                else mbar_arrive_cluster(mapa(smem_u32(&tmem_empty[buf]), 0u));
+            }
             if (p.mode == FT2_GEMM_CHECK && ncorr != 0u && p.counts != nullptr && seq >= 0)
                 atomicAdd(&p.counts[seq], ncorr);
             if (derive) {
@@ -346,9 +409,14 @@ __global__ void __launch_bounds__(kPThreads, 1)
     // ----------------------------------------------------------- teardown
     tc_fence_before();
     __syncthreads();
+    if (MC > 1) {  // no CTA leaves while its peer may still signal its barriers
+        cluster_arrive_relaxed();
+        cluster_wait();
+    }
     if (warp == 1) {
         tc_fence_after();
-        tmem_dealloc(tmem_base, 512);
+        if (MC == 1) tmem_dealloc(tmem_base, 512);
+        else tmem_dealloc2(tmem_base, 512);
     }
     if (!derive) return;
     if (use_tab) {
@@ -392,10 +460,10 @@ static bool make_map_p(CUtensorMap* m, const void* base, int64_t rows, int64_t K
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int DT>
+template <int DT, int MC>
 static cudaError_t launch_prefill_dt(const CUtensorMap& mx, const CUtensorMap& mw, const PrefK& p, int grid,
                                      cudaStream_t st) {
-    static cudaError_t attr = cudaFuncSetAttribute(prefill_gemm_kernel<DT>,
+    static cudaError_t attr = cudaFuncSetAttribute(prefill_gemm_kernel<DT, MC>,
                                                    cudaFuncAttributeMaxDynamicSharedMemorySize, kPSmemBytes);
     if (attr != cudaSuccess) return attr;
     cudaLaunchConfig_t cfg = {};
@@ -403,19 +471,22 @@ static cudaError_t launch_prefill_dt(const CUtensorMap& mx, const CUtensorMap& m
     cfg.blockDim = dim3(kPThreads);
     cfg.dynamicSmemBytes = kPSmemBytes;
     cfg.stream = st;
-    cudaLaunchAttribute a[1];
+    cudaLaunchAttribute a[2];
     a[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     a[0].val.programmaticStreamSerializationAllowed = 1;
+    a[1].id = cudaLaunchAttributeClusterDimension;
+    a[1].val.clusterDim.x = MC;
+    a[1].val.clusterDim.y = 1;
+    a[1].val.clusterDim.z = 1;
     cfg.attrs = a;
-    cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, prefill_gemm_kernel<DT>, mx, mw, p);
+    cfg.numAttrs = MC > 1 ? 2 : 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, prefill_gemm_kernel<DT, MC>, mx, mw, p);
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaStream_t st, int* n_launch) {
     CUtensorMap mx, mw;
     if (!make_map_p(&mx, a.x, a.M, a.K, a.ldx, kPBM, a.dtype)) return cudaErrorInvalidValue;
-    if (!make_map_p(&mw, a.w, a.N, a.K, a.ldw, kPBN, a.dtype)) return cudaErrorInvalidValue;
     PrefK p = {};
     p.M = a.M;
     p.N = a.N;
@@ -462,9 +533,23 @@ cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaS
         b.S = 0;
         b.ws = nullptr;
     }
-    const int grid = p.ntiles < num_sms() ? p.ntiles : num_sms();
-    cudaError_t e = a.dtype == FT2_FP16 ? launch_prefill_dt<1>(mx, mw, p, grid, st)
-                                        : launch_prefill_dt<0>(mx, mw, p, grid, st);
+
+    static const int mc_env = [] { const char* v = getenv("FT2_PREFILL_MC"); return v ? atoi(v) : 2; }();
+    const int mc = (mc_env == 2 && p.tilesM >= 2) ? 2 : 1;  // CTA pairs (cta_group::2) unless one m-tile
+    if (!make_map_p(&mw, a.w, a.N, a.K, a.ldw, mc == 2 ? kPBN / 2 : kPBN, a.dtype)) return cudaErrorInvalidValue;
+    int grid;
+    if (mc == 2) {
+        const int npairs = ((p.tilesM + 1) / 2) * (p.ntiles / p.tilesM);
+        const int maxpairs = num_sms() / 2;
+        grid = 2 * (npairs < maxpairs ? npairs : maxpairs);
+    } else {
+        grid = p.ntiles < num_sms() ? p.ntiles : num_sms();
+    }
+    cudaError_t e;
+    if (mc == 2) e = a.dtype == FT2_FP16 ? launch_prefill_dt<1, 2>(mx, mw, p, grid, st)
+                                         : launch_prefill_dt<0, 2>(mx, mw, p, grid, st);
+    else e = a.dtype == FT2_FP16 ? launch_prefill_dt<1, 1>(mx, mw, p, grid, st)
+                                 : launch_prefill_dt<0, 1>(mx, mw, p, grid, st);
     ++*n_launch;
     return e;
 }
