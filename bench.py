@@ -70,14 +70,15 @@ def load_peaks():
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
     """SM clock + throttle reasons sampled DURING the timed region.  Uses NVML
-    in-process (a 100 ms polling thread: one ioctl per sample, no subprocess
+    in-process (a 500 ms polling thread: each query takes a driver lock that
+    stalls graph launches, measured ~5% slower requests at 100 ms; no subprocess
     competing with the host-side launch path); falls back to `nvidia-smi -lms`."""
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
     NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
-    def __init__(self, dev_index: int, period_s: float = 0.1):
+    def __init__(self, dev_index: int, period_s: float = 0.5):
         self.dev = dev_index
         self.period = period_s
         self.proc = None
@@ -496,7 +497,49 @@ def kernel_rooflines(runner, dev, ft2):
     }
     del y
     torch.cuda.empty_cache()
-    return {"roofline": gemm, "protect_kernels_roofline": prot}
+    return {"roofline": gemm, "protect_kernels_roofline": prot, "prefill_derive_roofline": prefill_derive_roofline(
+        dev, ft2, peaks, time_it)}
+
+
+def prefill_derive_roofline(dev, ft2, peaks, time_it):
+    """ft2_prefill_fused_gemm (first-token bounds fused into the tcgen05
+    cta_group::2 GEMM epilogue) at a Llama-2-7B up_proj prefill shape, against
+    the measured dense bf16 peak; cuBLAS + the standalone sweep beside it."""
+    import torch
+
+    import ft2_synth
+
+    M, N, K, B = 4096, 11008, 4096, 32
+    x = ft2_synth.gen_bf16_torch((M, K), 20, 1, device=dev)
+    ws_ = [ft2_synth.gen_bf16_torch((N, K), 21 + i, 1, scale_log2=-6, device=dev) for i in range(2)]
+    b = ft2_synth.gen_bf16_torch((N,), 22, 1, device=dev)
+    y = torch.empty((M, N), dtype=torch.bfloat16, device=dev)
+    so = torch.arange(0, M + 1, M // B, dtype=torch.int32, device=dev)
+    bnd = torch.zeros((B, 2), dtype=torch.bfloat16, device=dev)
+    wsp = ft2.make_workspace(B, device=dev)
+    it = [0]
+
+    def derive():
+        it[0] += 1
+        ft2.prefill_fused_gemm(x, ws_[it[0] % 2], y, bnd, wsp, bias=b, seq_offsets=so, num_seqs=B)
+
+    def cublas_sweep():
+        it[0] += 1
+        torch.addmm(b, x, ws_[it[0] % 2].t(), out=y)
+        ft2.bounds_from_prefill(y, bnd, wsp, seq_offsets=so, num_seqs=B, correct_nonfinite=True)
+
+    ms_d = time_it(derive, R=10)
+    ms_c = time_it(cublas_sweep, R=10)
+    flops = 2.0 * M * N * K
+    peak = (peaks or {}).get("bf16_tflops", 2250.0)
+    ach = flops / (ms_d / 1e3) / 1e12
+    del x, ws_, y
+    torch.cuda.empty_cache()
+    return {"bound": "tensor", "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
+            "traffic": None, "kernel": "ft2 prefill_gemm_kernel (tcgen05 cta_group::2, DERIVE epilogue)",
+            "shape": [M, N, K], "sequences": B, "us": 1000 * ms_d, "cublas_plus_sweep_us": 1000 * ms_c,
+            "peak_source": "measured (MEASURED_PEAKS.json bf16_tflops, cuBLAS burst)" if peaks else
+            "fallback 2250 (nominal dense bf16)", "algorithmic_flops": "2*M*N*K per launch"}
 
 
 if __name__ == "__main__":

@@ -14,16 +14,22 @@
 // corrected), L259/L272 (check after the critical layer).  Order of the
 // epilogue: GEMM -> +bias -> bf16 -> inject -> check / derive (A19, A20).
 //
-// Persistent, warp-specialised, one CTA per SM (192 threads):
-//   warp 0      TMA producer: 128x64 A (x) and 256x64 B (W) boxes, 128B
-//               swizzle, into a 4-stage ring (48 KB per stage).
-//   warp 1      TMEM allocator (512 columns = two 128x256 fp32 accumulators)
-//               and the single-thread tcgen05.mma.cta_group::1.kind::f16
-//               issuer (M=128, N=256, K=16).
-//   warps 2-5   epilogue: tcgen05.ld 32 columns at a time (one TMEM lane =
-//               one output row per thread), while the MMA warp fills the other
+// Persistent, warp-specialised, one CTA per SM (320 threads), normally as a
+// CTA pair (cluster of 2, tcgen05.mma.cta_group::2) computing 256 x 256 tiles:
+//   warp 0      TMA producer: this CTA's 128 rows of the x box and 128 rows of
+//               the W box (128B swizzle) into a 6-stage ring of 32 KB stages;
+//               completion is counted on the leader CTA's barrier.
+//   warp 1      TMEM allocator (512 columns = two 128x256 fp32 accumulators per
+//               CTA); in the leader, the single-thread MMA issuer (M=256 over
+//               the pair, N=256, K=16), whose commits are multicast to both CTAs.
+//   warps 2-9   epilogue: two warps per TMEM lane quarter (one per 128-column
+//               half), tcgen05.ld 32 columns at a time (one TMEM lane = one
+//               output row per thread), while the MMA fills the other
 //               accumulator with the next tile (TMEM double buffering).
-// Tiles are 128 x 256, handed out round-robin (tile = blockIdx.x + i * grid).
+// The pair halves each SM's shared-memory operand traffic (the weight box is
+// staged once per 256 rows of x), which the single-CTA 128x256 variant (used
+// when there is only one 128-row m-tile) cannot sustain at the MMA rate.
+// Tiles are handed out round-robin (tile = cluster + i * clusters).
 // DERIVE keeps a per-CTA table of the sequences' key extrema in shared memory
 // (warp-reduced when a warp's 32 rows belong to one sequence) and flushes it
 // once; the bounds workspace protocol is the one of ft2_bounds_from_prefill
@@ -41,7 +47,9 @@
 namespace ft2impl {
 using namespace ft2dev;
 
-constexpr int kPBM = 128, kPBN = 256, kPBK = 64, kPThreads = 192;
+constexpr int kPBM = 128, kPBN = 256, kPBK = 64;
+constexpr int kPEpiWarps = 8;                      // two per TMEM lane quarter, one per 128-column half
+constexpr int kPThreads = 64 + 32 * kPEpiWarps;    // + producer warp + MMA warp
 constexpr int kPABytes = kPBM * kPBK * 2;  // 16 KB: one CTA's 128 rows of x
 constexpr int kPTileBytes = 192 * 1024;    // the shared-memory ring
 // MC = 1: a CTA loads the whole 256-row weight box (48 KB stages, 4 deep);
@@ -135,7 +143,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
         // both CTAs' epilogue warps; empty[] / tmem_full[] are signalled in
         // both CTAs by the leader's multicast commits
         for (int s = 0; s < kPStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-        for (int b = 0; b < 2; ++b) { mbar_init(&tmem_full[b], 1); mbar_init(&tmem_empty[b], 4 * MC); }
+        for (int b = 0; b < 2; ++b) { mbar_init(&tmem_full[b], 1); mbar_init(&tmem_empty[b], kPEpiWarps * MC); }
         fence_mbar_init();
     }
     if (warp == 1) {
@@ -221,6 +229,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
         // --------------------------------------------------------- epilogue
         const int q = warp & 3;  // TMEM lane quarter of this warp
         const int e = q * 32 + lane;
+        const int h0 = ((warp - 2) >> 2) * (kPBN / 2);  // first column of this warp's half
         griddep_wait();  // bias / bounds / sites / y may belong to the previous kernel
         uint32_t* ws_lc = p.bp.ws + 4 * p.bp.S + 1;
         uint32_t* ws_ov = p.bp.ws + 4 * p.bp.S + 2;
@@ -271,7 +280,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
             const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * kPBN);
             uint16_t* yrow = p.y + (int64_t)m * p.ldy;
 #pragma unroll 1
-            for (int c0 = 0; c0 < kPBN; c0 += 32) {
+            for (int c0 = h0; c0 < h0 + kPBN / 2; c0 += 32) {
                 uint32_t r[32];
                 tmem_ld32(taddr + (uint32_t)c0, r);
                 tmem_wait_ld();
@@ -363,8 +372,8 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     // what this thread just stored (rare; R2 excludes it, R4 patches it)
                     kmin = 0xFFFFu;
                     kmax = 0u;
-                    const int nend = min(p.N, n0 + kPBN);
-                    for (int n = n0; n < nend; ++n) {
+                    const int nend = min(p.N, n0 + h0 + kPBN / 2);
+                    for (int n = n0 + h0; n < nend; ++n) {
                         const uint16_t b = yrow[n];
                         if (nonfinite1<DT>(b)) {
                             ++nf;
