@@ -46,6 +46,11 @@ def parse():
     ap.add_argument("--prompt", type=int, default=128)
     ap.add_argument("--gen", type=int, default=60)
     ap.add_argument("--no-extras", action="store_true", help="skip the kernel roofline / cpu baseline legs")
+    ap.add_argument("--leg", default=None, choices=["c3", "c4", "c5"],
+                    help="run one measurement leg alone and print its JSON (c3: Llama-2-7B decode GEMMs; "
+                         "c4: Llama-2-13B tensor-parallel bounds over the ranks (NCCL MAX all-reduce); "
+                         "c5: SDC fault-injection campaign, trials sharded over ranks)")
+    ap.add_argument("--trials", type=int, default=3072, help="c5: trials per fault model (the paper: 10^5)")
     ap.add_argument("--profile", action="store_true",
                     help="warm up, then run exactly one fused request (for ncu launch lists) and exit")
     return ap.parse_args()
@@ -260,6 +265,25 @@ def main():
 
     import paper_conf_hpdc_sunzmg00y25_b200 as ft2
     from paper_conf_hpdc_sunzmg00y25_b200.runner import CONFIGS, Runner
+
+    if args.leg == "c3":
+        if rank == 0:
+            print(json.dumps({"leg": "c3", **c3_decode_gemm(dev, ft2, load_peaks())}), flush=True)
+        return 0
+    if args.leg == "c4":
+        res = c4_tp_bounds(args, dev, rank, world)
+        if rank == 0:
+            print(json.dumps(res), flush=True)
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+    if args.leg == "c5":
+        res = c5_campaign(args, dev, rank, world)
+        if rank == 0:
+            print(json.dumps(res), flush=True)
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
 
     cfg = CONFIGS[args.model]
     B, T, G = args.batch, args.prompt, args.gen
@@ -498,7 +522,266 @@ def kernel_rooflines(runner, dev, ft2):
     del y
     torch.cuda.empty_cache()
     return {"roofline": gemm, "protect_kernels_roofline": prot, "prefill_derive_roofline": prefill_derive_roofline(
-        dev, ft2, peaks, time_it)}
+        dev, ft2, peaks, time_it), "c3_llama7b_decode_gemm": c3_decode_gemm(dev, ft2, peaks)}
+
+
+def c4_tp_bounds(args, dev, rank, world, B=32, T=128, blocks=40, R=20):
+    """configs[3]: Llama-2-13B-shaped critical layers tensor-parallel over the
+    ranks.  Per prefill (B=32 x T=128 = 4096 tokens)
+    every rank sweeps its column shard of the 80 column-parallel critical
+    outputs (v_proj 5120/P, up_proj 13824/P wide) for raw keys, runs ONE
+    int32 MAX all-reduce of [80, 32, 2] keys (NCCL over NVLink), finalizes the
+    bounds, and bounds the 80 row-parallel outputs (o_proj, down_proj, full
+    5120 wide after the model's own sum all-reduce) locally.  The bounds are
+    checked bit-exact against the unsharded single-GPU sweep of the same
+    tensors.  Timed on the device, max over ranks; the all-reduce alone too."""
+    import torch
+    import torch.distributed as dist
+
+    import ft2_synth
+    import paper_conf_hpdc_sunzmg00y25_b200 as ft2
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+
+    rows = B * T
+    so = torch.arange(0, rows + 1, T, dtype=torch.int32, device=dev)
+    col_layers, row_layers = [], []
+    full_cols = {}
+    for blk in range(blocks):
+        for j, n in ((0, 5120), (1, 13824)):
+            # 4 distinct seeded outputs per layer class, rotated: the reuse
+            # distance (4 blocks, > 600 MB) exceeds L2, so every sweep reads HBM
+            key = (n, blk % 4)
+            if key not in full_cols:
+                full_cols[key] = ft2_synth.gen_bf16_torch((rows, n), 900 + 8 * j + blk % 4, 5, device=dev)
+            b, e = tp.column_shard(n, world, rank)
+            col_layers.append((full_cols[key], b, e))
+        if blk < 4:
+            row_layers.append(ft2_synth.gen_bf16_torch((rows, 5120), 950 + blk, 5, device=dev))
+        else:
+            row_layers.append(row_layers[blk % 4])
+    L = len(col_layers)
+    keys = torch.zeros((L, B, 2), dtype=torch.int32, device=dev)
+    bcol = torch.zeros((L, B, 2), dtype=torch.bfloat16, device=dev)
+    brow = torch.zeros((len(row_layers), B, 2), dtype=torch.bfloat16, device=dev)
+    wss = ft2.make_workspace(B, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def sweeps():
+        for i, (y, b, e) in enumerate(col_layers):
+            ft2.bounds_from_prefill(y[:, b:e], None, wss, seq_offsets=so, num_seqs=B, finalize=False,
+                                    keys_out=keys[i])
+
+    def allreduce():
+        if world > 1:
+            tp.allreduce_bounds_keys(keys)
+
+    def finish():
+        ft2.bounds_finalize(keys.view(-1, 2), bcol.view(-1, 2))
+        for i, y in enumerate(row_layers):
+            ft2.bounds_from_prefill(y, brow[i], wss, seq_offsets=so, num_seqs=B, correct_nonfinite=True)
+
+    def phase():
+        sweeps(); allreduce(); finish()
+
+    def dev_time(fn, reps):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(reps):
+            fn()
+        b_.record(stream)
+        torch.cuda.synchronize()
+        us = 1000.0 * a.elapsed_time(b_) / reps
+        if world > 1:
+            t = torch.tensor([us], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            us = float(t.item())
+        return us
+
+    for _ in range(max(3, args.warmup)):
+        phase()
+    us_phase = dev_time(phase, R)
+    us_ar = dev_time(allreduce, 50) if world > 1 else 0.0
+    # bit-exactness against the unsharded single-GPU sweep (P = 1) of the same tensors
+    ref = torch.zeros((L, B, 2), dtype=torch.bfloat16, device=dev)
+    for i, (y, _, _) in enumerate(col_layers):
+        ft2.bounds_from_prefill(y, ref[i], wss, seq_offsets=so, num_seqs=B)
+    exact = bool(torch.equal(ref.view(torch.int16), bcol.view(torch.int16)))
+    if world > 1:
+        f = torch.tensor([0 if exact else 1], device=dev)
+        dist.all_reduce(f, op=dist.ReduceOp.MAX)
+        exact = int(f.item()) == 0
+    shard_bytes = sum(rows * (e - b) * 2 for _, b, e in col_layers) + sum(y.numel() * 2 for y in row_layers)
+    return {"leg": "c4", "metric": "TP first-token bounds phase per prefill (us, max over ranks)", "value": us_phase,
+            "unit": "us", "higher_is_better": False, "n_gpus": world, "scaling": "strong",
+            "config": {"workload": "llama-2-13b-shaped critical layers, TP over the ranks (configs[3]): "
+                                   f"{L} column-parallel sweeps + 1 MAX all-reduce of int32 [{L},{B},2] + finalize "
+                                   f"+ {len(row_layers)} row-parallel sweeps; B={B}, prompt {T}",
+                       "tp": world},
+            "allreduce_us": us_ar, "allreduce_bytes": keys.numel() * 4,
+            "bounds_bitexact_vs_unsharded": exact,
+            "per_rank_bytes_swept": shard_bytes, "l2": "4 distinct tensors per layer class rotated (> L2)",
+            "per_rank_GBps": shard_bytes / (us_phase * 1e-6) / 1e9}
+
+
+def c5_campaign(args, dev, rank, world, model="llama-2-7b", B=256, T=16, S=32):
+    """configs[4]: the SDC fault-injection campaign
+    on a Llama-2-7B-shaped seeded model: prompt 16, 32 decode steps, 224
+    linear layers as fault targets, `--trials` trials per fault model (1-bit,
+    2-bit, EXP), FT2 off and on over the same sites, one trial per batch row
+    (B = 256).  Rank r of N takes trials [r*n/N, (r+1)*n/N) of every model;
+    no data-path collective, one counter all_reduce per model at the end.
+    Timed: all faulty generations of every batch (the golden runs and the
+    per-step graph captures happen once, in an untimed warm-up batch)."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_hpdc_sunzmg00y25_b200 import campaign
+    from paper_conf_hpdc_sunzmg00y25_b200.runner import CONFIGS, Runner
+
+    cfg = CONFIGS[model]
+    runner = Runner(cfg, B, T, S + 1, seed=1, device=dev)
+    prompts = campaign.campaign_prompts(runner)
+    golden = campaign.golden_runs(runner, prompts)
+    # warm-up: captures the prefill graph and the 32 per-step decode graphs of
+    # both modes with faults armed (trials far outside the timed ranges)
+    for _ in range(max(1, args.warmup // 3)):
+        campaign.run_batch(runner, prompts, 4242, 1 << 40, 2, golden=golden)
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    out = {"leg": "c5", "metric": "fault-injection trials/s (FT2 off + on per trial, same sites)",
+           "unit": "trials/s", "n_gpus": world, "higher_is_better": True, "scaling": "strong",
+           "config": {"workload": f"{model}-shaped SDC campaign (configs[4]), B={B} trials per batch, prompt {T}, "
+                                  f"{S} decode steps, 224 linear layers", "trials_per_model": args.trials,
+                      "parallelism": f"trial ranges sharded over {world} rank(s)"},
+           "models": {}}
+    tot_ms, tot_trials = 0.0, 0
+    clk = ClockSampler(int(os.environ.get("LOCAL_RANK", "0")))
+    clk.start()
+    for fm, name in campaign.MODEL_NAMES.items():
+        t0, t1 = campaign.trial_range(args.trials, world, rank)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        res = campaign.CampaignResult()
+        t = t0
+        while t < t1:
+            res.add(campaign.run_batch(runner, prompts, 1, t, fm, golden=golden, take=min(B, t1 - t)))
+            t += B
+        b_.record(stream)
+        torch.cuda.synchronize()
+        ms = a.elapsed_time(b_)
+        if world > 1:
+            v = res.as_tensor(dev)
+            dist.all_reduce(v)
+            res = campaign.CampaignResult.from_tensor(v)
+            m = torch.tensor([ms], device=dev)
+            dist.all_reduce(m, op=dist.ReduceOp.MAX)
+            ms = float(m.item())
+        tot_ms += ms
+        tot_trials += res.trials
+        out["models"][name] = {"trials_per_s": res.trials / (ms / 1e3), "ms": ms, **res.summary()}
+    out["clocks"] = clk.stop()
+    out["value"] = tot_trials / (tot_ms / 1e3)
+    out["ms_total"] = tot_ms
+    out["generations_per_trial"] = 2
+    out["paper_context"] = ("~0.38 trials/s per A100 (11 M injections / 8000 GPU-h, PAPER.md L282); "
+                            "real SDC rates need trained weights -- proxy only")
+    return out
+
+
+def c3_decode_gemm(dev, ft2, peaks, M=32, copies=8, R=10, rounds=5):
+    """configs[2]: the Llama-2-7B critical layers (v, o, up, down; SURVEY.md
+    §8(a) a5) at batch-32 decode.  Per shape, a CUDA graph of `copies`
+    launches over `copies` distinct weight matrices (>= 268 MB, beyond L2)
+    for cuBLAS, cuBLAS + ft2_protect (the paper's structure, L272), the fused
+    GEMM without the check (PLAIN) and with it (CHECK).  Bounds come from a
+    real 16-token-per-sequence prefill of each layer (32 sequences).  Rounds
+    interleave the four variants; medians are reported.  The north-star
+    target is CHECK / PLAIN - 1 <= 2 %."""
+    import torch
+
+    import ft2_synth
+
+    hbm_peak = (peaks or {}).get("hbm_gbs", 6650.0)
+    shapes = [("v_proj", 4096, 4096), ("o_proj", 4096, 4096), ("up_proj", 11008, 4096), ("down_proj", 4096, 11008)]
+    stream = torch.cuda.current_stream()
+    out = {"M": M, "weights_per_graph": copies, "timing": f"graph of {copies} back-to-back launches over "
+           f"{copies} weight copies (> L2), median of {rounds} interleaved rounds x {R} replays",
+           "bounds": "from a 16-token prefill per sequence (32 sequences), ft2_bounds_from_prefill", "shapes": {}}
+    tot = {"cublas": 0.0, "cublas_protect": 0.0, "plain": 0.0, "check": 0.0}
+    tot_bytes = 0
+    for si, (name, N, K) in enumerate(shapes):
+        ws = [ft2_synth.gen_bf16_torch((N, K), 600 + 8 * si + c, 3, scale_log2=ft2_synth.weight_scale_log2(K),
+                                       device=dev) for c in range(copies)]
+        x = ft2_synth.gen_bf16_torch((M, K), 700 + si, 3, device=dev)
+        xp = ft2_synth.gen_bf16_torch((M * 16, K), 710 + si, 3, device=dev)
+        yp = torch.nn.functional.linear(xp, ws[0])
+        bnd = torch.zeros((M, 2), dtype=torch.bfloat16, device=dev)
+        so = torch.arange(0, M * 16 + 1, 16, dtype=torch.int32, device=dev)
+        ft2.bounds_from_prefill(yp, bnd, ft2.make_workspace(M, device=dev), seq_offsets=so, num_seqs=M,
+                                correct_nonfinite=True)
+        ys = [torch.empty((M, N), dtype=torch.bfloat16, device=dev) for _ in range(copies)]
+        cnt = torch.zeros(M, dtype=torch.int32, device=dev)
+
+        def body(kind):
+            for w, y in zip(ws, ys):
+                if kind == "cublas":
+                    torch.mm(x, w.t(), out=y)
+                elif kind == "cublas_protect":
+                    torch.mm(x, w.t(), out=y)
+                    ft2.protect(y, bnd, num_seqs=M, corrected_count=cnt)
+                else:
+                    mode = (1 if kind == "check" else 0) | 16
+                    ft2.protect_fused_gemm(x, w, y, mode=mode, bounds=bnd, num_seqs=M, corrected_count=cnt)
+
+        graphs = {}
+        for kind in tot:
+            body(kind)
+            torch.cuda.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                body(kind)
+            for _ in range(3):
+                g.replay()
+            graphs[kind] = g
+        samples = {k: [] for k in tot}
+        for _ in range(rounds):
+            for kind, g in graphs.items():
+                torch.cuda.synchronize()
+                a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                for _ in range(R):
+                    g.replay()
+                b_.record(stream)
+                torch.cuda.synchronize()
+                samples[kind].append(1000.0 * a.elapsed_time(b_) / (R * copies))
+        us = {k: statistics.median(v) for k, v in samples.items()}
+        nbytes = N * K * 2 + M * K * 2 + M * N * 2
+        tot_bytes += nbytes
+        for k in tot:
+            tot[k] += us[k]
+        ach = nbytes / (us["check"] * 1e-6) / 1e9
+        out["shapes"][name] = {
+            "N": N, "K": K, "us": {k: round(v, 3) for k, v in us.items()},
+            "check_vs_plain_pct": 100.0 * (us["check"] / us["plain"] - 1.0),
+            "check_vs_cublas_protect_pct": 100.0 * (us["check"] / us["cublas_protect"] - 1.0),
+            "roofline": {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+                         "algorithmic_bytes_per_launch": nbytes}}
+        del ws, ys, graphs
+        torch.cuda.empty_cache()
+    ach = tot_bytes / (tot["check"] * 1e-6) / 1e9
+    out["block"] = {"us": {k: round(v, 3) for k, v in tot.items()},
+                    "check_vs_plain_pct": 100.0 * (tot["check"] / tot["plain"] - 1.0),
+                    "check_vs_cublas_pct": 100.0 * (tot["check"] / tot["cublas"] - 1.0),
+                    "cublas_protect_vs_cublas_pct": 100.0 * (tot["cublas_protect"] / tot["cublas"] - 1.0),
+                    "roofline": {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
+                                 "frac": ach / hbm_peak}}
+    return out
 
 
 def prefill_derive_roofline(dev, ft2, peaks, time_it):

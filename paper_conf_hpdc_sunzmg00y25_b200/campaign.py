@@ -15,7 +15,7 @@ no semantic notion of a wrong answer, so this proxy is
 labelled as such and is never compared with the paper's SDC rates
 (parity unpinned).  Reported: proxy-SDC rates with 95% Wald
 margins (L282), the reduction 1 - p_on/p_off (L313) and the detection rate
-(trials whose FT2 corrected-neuron count is non-zero).
+(trials whose row FT2 corrected more neurons in than in its fault-free run).
 
 Sharding: rank r of W takes trials [r*n/W, (r+1)*n/W); per-rank counters are
 summed with one all_reduce at the end (the only collective).
@@ -40,6 +40,7 @@ class CampaignResult:
     sdc_on: int = 0
     detected_on: int = 0
     golden_mismatch: int = 0   # fault-free FT2-on vs FT2-off token differences (false-positive proxy)
+    fault_free_corrected: int = 0   # rows whose fault-free FT2-on run clipped at least one neuron
 
     def add(self, other: "CampaignResult"):
         for f in dataclasses.fields(self):
@@ -63,6 +64,7 @@ class CampaignResult:
             "proxy_sdc_reduction": (1.0 - p_on / p_off) if p_off > 0 else None,
             "detection_rate": self.detected_on / n,
             "fault_free_mismatch_rate": self.golden_mismatch / n,
+            "fault_free_correction_rate": self.fault_free_corrected / n,
             "label": "proxy SDC = generated tokens differ from the golden run (random weights; not the paper's SDC)",
         }
 
@@ -77,44 +79,73 @@ def trial_range(n_trials: int, world: int, rank: int):
     return (rank * n_trials) // world, ((rank + 1) * n_trials) // world
 
 
+OFF_MODE = "fused_plain"   # FT2 off = the same tcgen05 GEMM without the check
+
+
+def golden_runs(runner: Runner, prompt_ids: torch.Tensor, use_graph: bool = True, off_mode: str = OFF_MODE):
+    """Fault-free generations with FT2 off and on (the golden runs of every
+    batch: prompts and weights are fixed for the whole campaign), plus the
+    fault-free corrected-neuron count of every row with FT2 on.
+
+    FT2 off runs the same tcgen05 GEMM as FT2 on, without the check
+    ("fused_plain"), so golden_off and golden_on differ only where the
+    fault-free check clips (off_mode="off" would compare against cuBLAS,
+    whose different summation order alone changes greedy tokens)."""
+    runner.set_sites(None)
+    g_off = runner.generate(prompt_ids, off_mode, use_graph=use_graph).clone()
+    g_on = runner.generate(prompt_ids, "fused", use_graph=use_graph).clone()
+    g_corr = (runner.state.corrected.sum(0) + runner.state.nonfinite.sum(0)).clone()
+    return g_off, g_on, g_corr
+
+
 def run_batch(runner: Runner, prompt_ids: torch.Tensor, seed: int, trial0: int, fault_model: int,
-              step_policy: int = 0) -> CampaignResult:
-    """One batch of B trials (rows) on the runner; returns the counters."""
-    B, G = runner.B, runner.G
-    widths = runner.cfg.linear_widths()
-    sites = F2.make_fault_sites(seed, trial0, B, fault_model, widths, n_steps=G - 1, prompt_len=runner.T,
-                                step_policy=step_policy, device=prompt_ids.device)
-    runner.sites = None
-    golden_off = runner.generate(prompt_ids, "off", use_graph=False).clone()
-    golden_on = runner.generate(prompt_ids, "fused", use_graph=False).clone()
-    runner.sites = sites
-    faulty_off = runner.generate(prompt_ids, "off", use_graph=False).clone()
-    faulty_on = runner.generate(prompt_ids, "fused", use_graph=False).clone()
-    corrected = runner.state.corrected.sum(0) + runner.state.nonfinite.sum(0)   # per trial row
-    runner.sites = None
+              step_policy: int = 0, golden=None, take: int | None = None, use_graph: bool = True,
+              off_mode: str = OFF_MODE) -> CampaignResult:
+    """One batch of B trials (rows) on the runner; returns the counters of its
+    first `take` rows (default all B).  `golden` = golden_runs(...) of the same
+    prompts, computed here when None.  With use_graph the faulty generations
+    replay per-step CUDA graphs captured once (the sites live in the runner's
+    stable sites_buf, rewritten per batch by ft2_make_fault_sites).
+
+    A trial is *detected* when FT2 corrected more neurons in its row than in
+    the fault-free run of the same row (the check also clips a few fault-free
+    outliers; those are counted as fault_free_corrected)."""
+    B = runner.B
+    take = B if take is None else take
+    golden_off, golden_on, golden_corr = golden if golden is not None else \
+        golden_runs(runner, prompt_ids, use_graph, off_mode)
+    runner.make_sites(seed, trial0, fault_model, step_policy=step_policy)
+    faulty_off = runner.generate(prompt_ids, off_mode, use_graph=use_graph)[:take].clone()
+    faulty_on = runner.generate(prompt_ids, "fused", use_graph=use_graph)[:take].clone()
+    corrected = (runner.state.corrected.sum(0) + runner.state.nonfinite.sum(0))[:take]   # per trial row
+    runner.set_sites(None)
+    golden_off, golden_on, golden_corr = golden_off[:take], golden_on[:take], golden_corr[:take]
     r = CampaignResult()
-    r.trials = B
+    r.trials = take
     r.sdc_off = int((faulty_off != golden_off).any(1).sum().item())
     r.sdc_on = int((faulty_on != golden_on).any(1).sum().item())
-    r.detected_on = int((corrected > 0).sum().item())
+    r.detected_on = int((corrected > golden_corr).sum().item())
     r.golden_mismatch = int((golden_on != golden_off).any(1).sum().item())
+    r.fault_free_corrected = int((golden_corr > 0).sum().item())
     return r
 
 
+def campaign_prompts(runner: Runner, prompt_seed: int = 7) -> torch.Tensor:
+    gen = torch.Generator().manual_seed(prompt_seed)
+    return torch.randint(0, runner.cfg.vocab, (runner.B, runner.T), generator=gen).to(runner.device)
+
+
 def run_campaign(runner: Runner, n_trials: int, seed: int, fault_model: int, rank: int = 0, world: int = 1,
-                 group=None, prompt_seed: int = 7) -> CampaignResult:
+                 group=None, prompt_seed: int = 7, use_graph: bool = True) -> CampaignResult:
     """This rank's share of n_trials (batches of runner.B rows), counters summed over ranks."""
     t0, t1 = trial_range(n_trials, world, rank)
     total = CampaignResult()
-    gen = torch.Generator().manual_seed(prompt_seed)
-    prompts = torch.randint(0, runner.cfg.vocab, (runner.B, runner.T), generator=gen).to(runner.device)
+    prompts = campaign_prompts(runner, prompt_seed)
+    golden = golden_runs(runner, prompts, use_graph)
     t = t0
     while t < t1:
-        res = run_batch(runner, prompts, seed, t, fault_model)
-        take = min(runner.B, t1 - t)
-        if take < runner.B:   # partial last batch: only count the first `take` rows
-            res = _recount_partial(runner, prompts, seed, t, fault_model, take)
-        total.add(res)
+        total.add(run_batch(runner, prompts, seed, t, fault_model, golden=golden, take=min(runner.B, t1 - t),
+                            use_graph=use_graph))
         t += runner.B
     if world > 1:
         import torch.distributed as dist
@@ -122,25 +153,3 @@ def run_campaign(runner: Runner, n_trials: int, seed: int, fault_model: int, ran
         dist.all_reduce(v, group=group)
         total = CampaignResult.from_tensor(v)
     return total
-
-
-def _recount_partial(runner, prompts, seed, trial0, fault_model, take):
-    B, G = runner.B, runner.G
-    widths = runner.cfg.linear_widths()
-    sites = F2.make_fault_sites(seed, trial0, B, fault_model, widths, n_steps=G - 1, prompt_len=runner.T,
-                                device=prompts.device)
-    runner.sites = None
-    g_off = runner.generate(prompts, "off", use_graph=False).clone()
-    g_on = runner.generate(prompts, "fused", use_graph=False).clone()
-    runner.sites = sites
-    f_off = runner.generate(prompts, "off", use_graph=False).clone()
-    f_on = runner.generate(prompts, "fused", use_graph=False).clone()
-    corr = (runner.state.corrected.sum(0) + runner.state.nonfinite.sum(0))[:take]
-    runner.sites = None
-    r = CampaignResult()
-    r.trials = take
-    r.sdc_off = int((f_off != g_off)[:take].any(1).sum().item())
-    r.sdc_on = int((f_on != g_on)[:take].any(1).sum().item())
-    r.detected_on = int((corr > 0).sum().item())
-    r.golden_mismatch = int((g_on != g_off)[:take].any(1).sum().item())
-    return r

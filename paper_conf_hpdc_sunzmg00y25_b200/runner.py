@@ -183,8 +183,12 @@ class Runner:
         self.pos = torch.zeros(1, dtype=torch.int64, device=dv)
         self.out_tokens = torch.zeros((batch, gen_len), dtype=torch.int64, device=dv)
         self.sites = None        # optional fault sites (uint8 [B*24]); site i = sequence i
+        # stable site buffer: graphs captured with faults bake in its address, so
+        # a campaign rewrites it per batch (set_sites / make_sites) and replays
+        self.sites_buf = torch.zeros(batch * F2.SITE_BYTES, dtype=torch.uint8, device=dv)
         self.cur_step = torch.zeros(1, dtype=torch.int32, device=dv)
         self.graphs = {}
+        self._pool = torch.cuda.graph_pool_handle() if self.device.type == "cuda" else None   # shared by all graphs
         self.time_phases = False
         self._phase_events = []
         self.mode = "fused"
@@ -342,32 +346,59 @@ class Runner:
         self.tok.copy_(nxt)
         self.pos.add_(1)
 
+    def set_sites(self, sites):
+        """Fault sites for the next generate() calls (uint8 [B*24], site i =
+        sequence i), copied into the stable sites_buf; None = fault-free."""
+        if sites is None:
+            self.sites = None
+            return
+        if sites.data_ptr() != self.sites_buf.data_ptr():
+            self.sites_buf.copy_(sites.view(torch.uint8).reshape(-1)[: self.sites_buf.numel()])
+        self.sites = self.sites_buf
+
+    def make_sites(self, seed, trial0, fault_model, step_policy=0):
+        """ft2_make_fault_sites for trials [trial0, trial0 + B) straight into
+        sites_buf (one site per batch row), and arm them."""
+        F2.make_fault_sites(seed, trial0, self.B, fault_model, self.cfg.linear_widths(), n_steps=self.G - 1,
+                            prompt_len=self.T, step_policy=step_policy, out=self.sites_buf, device=self.device)
+        self.sites = self.sites_buf
+
     def _graph(self, mode, step_for_sites):
-        key = (mode, step_for_sites)
+        """CUDA graph of one decode step.  Fault-free: one graph per mode.  With
+        fault sites armed: one graph per (mode, decode step t), since the
+        injection matches sites against the host-side step index."""
+        faulty = self.sites is not None
+        key = (mode, step_for_sites if faulty else None, faulty)
         if key not in self.graphs:
             self.mode = mode
-            self._site_step = step_for_sites
+            self._site_step = step_for_sites if faulty else None
+            st = self.state
             s = torch.cuda.Stream()
             s.wait_stream(torch.cuda.current_stream())
             with torch.cuda.stream(s):
-                save = (self.tok.clone(), self.pos.clone(), self.out_tokens.clone())
+                save = (self.tok.clone(), self.pos.clone(), self.out_tokens.clone(), st.corrected.clone(),
+                        st.nonfinite.clone())
                 for _ in range(2):   # warm-up (allocations, cuBLAS handles)
                     self._decode_step()
-                self.tok.copy_(save[0]); self.pos.copy_(save[1]); self.out_tokens.copy_(save[2])
+                self._restore(save)
             torch.cuda.current_stream().wait_stream(s)
             g = torch.cuda.CUDAGraph()
             n0 = F2.launch_count()
-            with torch.cuda.graph(g):
+            with torch.cuda.graph(g, pool=self._pool):
                 self._decode_step()
             self.graphs[key] = (g, F2.launch_count() - n0)
-            self.tok.copy_(save[0]); self.pos.copy_(save[1]); self.out_tokens.copy_(save[2])
+            self._restore(save)
         return self.graphs[key]
+
+    def _restore(self, save):
+        self.tok.copy_(save[0]); self.pos.copy_(save[1]); self.out_tokens.copy_(save[2])
+        self.state.corrected.copy_(save[3]); self.state.nonfinite.copy_(save[4])
 
     def _prefill_graph(self, mode):
         """CUDA graph of the whole first-token pass (embedding, 24 blocks with
         the FT2 bound sweeps on the critical layers, LM head, first token) on
         the static prompt buffer; one per mode."""
-        key = ("prefill", mode)
+        key = ("prefill", mode, self.sites is not None)
         if key not in self.graphs:
             self.mode = mode
             self._site_step = None
@@ -384,7 +415,7 @@ class Runner:
                 body()   # warm-up (allocations, cuBLAS/cuDNN plans)
             torch.cuda.current_stream().wait_stream(s)
             g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g):
+            with torch.cuda.graph(g, pool=self._pool):
                 body()
             self.graphs[key] = g
         return self.graphs[key]
@@ -398,18 +429,21 @@ class Runner:
         return per_prefill + per_step * (self.G - 1)
 
     def generate(self, prompt_ids, mode="fused", use_graph=True):
-        """Greedy generation of G tokens (1 first token + G-1 decode steps)."""
-        if self.sites is not None and use_graph:
-            raise ValueError("fault sites need eager decode (use_graph=False): the step index changes per token")
+        """Greedy generation of G tokens (1 first token + G-1 decode steps).
+        With fault sites armed (set_sites / make_sites) and use_graph, every
+        decode step t replays its own captured graph (captured on first use)."""
         self.mode = mode
         self._site_step = None
+        faulty = self.sites is not None
+        if use_graph and self.graph_prefill:
+            pg = self._prefill_graph(mode)   # capture (and its warm-up) before the counters reset
         self.state.reset_counters()
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)] if self.time_phases else None
         if ev:
             ev[0].record()
         if use_graph and self.graph_prefill:
             self.prompt_static.copy_(prompt_ids, non_blocking=True)
-            self._prefill_graph(mode).replay()
+            pg.replay()
         else:
             first = self.prefill(prompt_ids)
             self.out_tokens[:, 0] = first
@@ -417,7 +451,12 @@ class Runner:
             self.pos.fill_(self.T)
         if ev:
             ev[1].record()
-        if use_graph:
+        if use_graph and faulty:
+            for t in range(1, self.G):
+                g, _ = self._graph(mode, t)   # decode step t (0 = prefill / first token)
+                g.replay()
+            self.mode = mode
+        elif use_graph:
             g, _ = self._graph(mode, None)
             self.mode = mode
             for _ in range(self.G - 1):

@@ -96,3 +96,32 @@ def test_nan_vulnerable_profile_matches_oracle(tiny):
     want = oracle.nan_vulnerable_count(yh, seq_offsets=np.arange(0, 17 * 8, 8))
     assert counts[0, 0].numpy().astype(np.uint32).tolist() == want.tolist()
     assert int(elems[0]) == 8 * tiny.cfg.hidden
+
+
+def test_graphed_faulty_runs_equal_eager(tiny):
+    """Per-step CUDA graphs of the faulty generations (captured once, sites
+    rewritten in place per batch) give the same tokens and the same FT2
+    counters as eager decode, batch after batch."""
+    p = torch.randint(0, 512, (16, 8), generator=torch.Generator().manual_seed(8)).cuda()
+    for trial0 in (0, 16, 32):
+        for mode in ("off", "fused"):
+            tiny.make_sites(5, trial0, 2)
+            e = tiny.generate(p, mode, use_graph=False).clone()
+            ec = (tiny.state.corrected.clone(), tiny.state.nonfinite.clone())
+            tiny.make_sites(5, trial0, 2)
+            g = tiny.generate(p, mode, use_graph=True).clone()
+            assert torch.equal(e, g), (trial0, mode)
+            assert torch.equal(ec[0], tiny.state.corrected) and torch.equal(ec[1], tiny.state.nonfinite)
+    tiny.set_sites(None)
+
+
+def test_partial_batch_counts_only_its_rows(tiny):
+    from paper_conf_hpdc_sunzmg00y25_b200 import campaign
+    prompts = campaign.campaign_prompts(tiny)
+    gold = campaign.golden_runs(tiny, prompts)
+    full = campaign.run_batch(tiny, prompts, 3, 0, 2, golden=gold)
+    part = campaign.run_batch(tiny, prompts, 3, 0, 2, golden=gold, take=5)
+    assert part.trials == 5 and full.trials == 16
+    assert part.sdc_off <= full.sdc_off and part.detected_on <= full.detected_on
+    eager = campaign.run_batch(tiny, prompts, 3, 0, 2, golden=gold, use_graph=False)
+    assert eager == full
