@@ -58,8 +58,17 @@ typedef enum {
 } ft2_status;
 
 /* Activation dtype.  BF16 and FP16 (the paper's main precision, L282) are
- * implemented by every entry point; FP32 (the paper's FP32 study, L334)
- * returns FT2_ERR_UNSUPPORTED in this release. */
+ * implemented by every entry point.  FP32 (the paper's FP32 study, L334;
+ * SURVEY.md 8(f) NEXT(3)) is implemented by ft2_bounds_from_prefill,
+ * ft2_bounds_finalize, ft2_protect, ft2_inject_faults and
+ * ft2_make_fault_sites, on 32-bit order keys
+ *     key32(b) = b & 0x80000000 ? ~b : b | 0x80000000
+ * with bounds stored as fp32 pairs, R3's product/quotient formed in fp64 from
+ * the fp32 value and scale and rounded outward to fp32, and keys_out in the
+ * MAX-combinable encoding (int32)(~key32(lo_raw) ^ 0x80000000),
+ * (int32)(key32(hi_raw) ^ 0x80000000), INT32_MIN = no finite value.  The
+ * fused GEMMs (bf16/fp16 tensor-core contractions) return
+ * FT2_ERR_UNSUPPORTED for FP32: use a library GEMM + ft2_protect. */
 typedef enum { FT2_BF16 = 0, FT2_FP16 = 1, FT2_FP32 = 2 } ft2_dtype;
 
 /* Fault models, PAPER.md L84 (Sec. 2.2): single-bit flip, double-bit flip,
@@ -79,8 +88,9 @@ typedef enum {
 typedef struct {
     void* data;       /* device pointer, 16-byte aligned */
     int64_t rows;     /* number of rows (tokens) */
-    int64_t n;        /* elements per row (output neurons); multiple of 8 for bf16 */
-    int64_t ld;       /* row stride in elements, >= n, multiple of 8 for bf16 */
+    int64_t n;        /* elements per row (output neurons); multiple of 8 (bf16/fp16) or 4 (fp32):
+                         one 16-byte vector */
+    int64_t ld;       /* row stride in elements, >= n, same multiple as n */
     ft2_dtype dtype;
 } ft2_tensor;
 
@@ -141,12 +151,14 @@ size_t ft2_workspace_bytes(int32_t num_seqs);
  *              a tensor-parallel MAX all-reduce, then ft2_bounds_finalize).
  * correct_nonfinite  1 (requires finalize = 1): after the bounds are known,
  *              NaN -> clamp(+0, lo, hi), +Inf -> hi, -Inf -> lo (readings A3-A6).
- * bounds_out   [num_seqs x 2] bf16 (lo, hi) per sequence, or NULL if finalize = 0.
+ * bounds_out   [num_seqs x 2] (lo, hi) per sequence in y.dtype (4-byte aligned; 8 for
+ *              fp32), or NULL if finalize = 0.
  *              A sequence without finite values gets lo = hi = +0 (reading A9).
  * keys_out     NULL or int32 [num_seqs x 2]: keys_out[2s] = 0xFFFF - key(lo_raw),
  *              keys_out[2s+1] = key(hi_raw), -1 where the sequence has no finite
  *              value; element-wise MAX of these over shards gives the keys of
- *              the unsharded tensor (min/max are exact and associative).
+ *              the unsharded tensor (min/max are exact and associative).  For
+ *              FT2_FP32 the encoding is the 32-bit one given at ft2_dtype.
  * nan_vulnerable_count  NULL or uint32 [num_seqs]: WRITTEN with the number of
  *              NaN-vulnerable values, those in (-2,-1) U (1,2) whose exponent-MSB
  *              flip gives NaN (Fig. 7; L202 reports their share per
@@ -155,7 +167,7 @@ size_t ft2_workspace_bytes(int32_t num_seqs);
  * nonfinite_count  NULL or uint32 [num_seqs]: WRITTEN with the number of
  *              non-finite elements of each sequence.
  * workspace    ft2_workspace_bytes(num_seqs) bytes, see above.
- * Limits: num_seqs <= FT2_MAX_SEQS, rows * n / 8 < 2^31. */
+ * Limits: num_seqs <= FT2_MAX_SEQS, rows * n / (8, fp32: 4) < 2^31. */
 ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int32_t num_seqs,
                                    float scale, int32_t finalize, int32_t correct_nonfinite,
                                    void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
@@ -164,7 +176,7 @@ ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int
 /* Bounds from (all-reduced) keys in the ft2_bounds_from_prefill keys_out
  * encoding: the second half of the tensor-parallel path. */
 ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scale,
-                               ft2_dtype dtype, void* bounds_out, void* stream);  /* dtype: BF16 / FP16 */
+                               ft2_dtype dtype, void* bounds_out, void* stream);  /* dtype: BF16 / FP16 / FP32 */
 
 /* Online range restriction of one protected layer's output: PAPER.md L151,
  * L259-L261 (Sec. 4.3: check every neuron after each critical layer), L261/L270
@@ -175,7 +187,8 @@ ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scal
  *              r when num_seqs == rows, every row -> sequence 0 when num_seqs
  *              == 1 (otherwise FT2_ERR_INVALID_ARG).  Rows mapped outside
  *              [0, num_seqs) are left untouched.
- * bounds       [num_seqs x 2] bf16 (lo, hi) with key(lo) <= key(hi), finite.
+ * bounds       [num_seqs x 2] (lo, hi) in y.dtype with key(lo) <= key(hi), finite
+ *              (4-byte aligned; 8 for fp32).
  * corrected_count  NULL or uint32 [num_seqs]: += number of elements whose bits
  *              changed (= NaN, +-Inf or out of bounds).
  * Only vectors containing a corrected element are written back. */

@@ -88,6 +88,13 @@ def lib():
             ("ft2o_linear_f64_dt", None, [P, i64, P, i64, P, i32, i32, i32, P, P, i64, ctypes.c_int]),
             ("ft2o_protected_linear_dt", None, [P, i64, P, i64, P, i32, i32, i32, P, i64, P, P, i32, P,
                                                 P, i32, i32, i32, P, ctypes.c_int]),
+            ("ft2o_isnan32", ctypes.c_int, [u32]), ("ft2o_isfinite32", ctypes.c_int, [u32]),
+            ("ft2o_key32", u32, [u32]), ("ft2o_unkey32", u32, [u32]),
+            ("ft2o_scale_bound32", u32, [u32, ctypes.c_float, ctypes.c_int]),
+            ("ft2o_clip_value32", u32, [u32, u32, u32]),
+            ("ft2o_protect32", None, [P, i64, i64, i64, P, P, i32, P]),
+            ("ft2o_bounds32", None, [P, i64, i64, i64, P, i32, ctypes.c_float, i32, P, P, P, P]),
+            ("ft2o_inject32", None, [P, i64, i64, i64, P, i32, i32, i32, P]),
         ]:
             f = getattr(L, name)
             f.restype = res
@@ -231,3 +238,57 @@ def protected_linear(x, w, bias, bounds_, row_to_seq=None, sites=None, cur_layer
     lib().ft2o_protected_linear_dt(_p(x), K, _p(w), K, _p(b), M, N, K, _p(y), N, _p(r2s), _p(bd), S,
                                    _p(cnt), _p(s), ns, cur_layer, cur_step, _p(br), dtype)
     return y, cnt
+
+
+# ------------------------------------------------------------------- FP32 --
+# The paper's FP32 study: the same method on binary32
+# activations, handled as uint32 bit patterns with a 32-bit order key.
+def key32(b: int) -> int: return lib().ft2o_key32(b)
+def unkey32(k: int) -> int: return lib().ft2o_unkey32(k)
+def isnan32(b: int) -> bool: return bool(lib().ft2o_isnan32(b))
+def scale_bound32(raw: int, c: float, is_hi: bool) -> int: return lib().ft2o_scale_bound32(raw, c, int(is_hi))
+def clip_value32(y: int, lo: int, hi: int) -> int: return lib().ft2o_clip_value32(y, lo, hi)
+
+
+def _u32(a):
+    a = np.ascontiguousarray(a)
+    if a.dtype != np.uint32:
+        a = a.view(np.uint32) if a.dtype.itemsize == 4 else a.astype(np.uint32)
+    return a
+
+
+def bounds32(y, seq_offsets=None, scale: float = 2.0, correct_nonfinite: bool = False):
+    """R2-R4 on binary32 bits y (uint32 [rows, n], modified in place iff
+    correct_nonfinite).  Returns (bounds uint32 [S,2], raw keys uint32 [S,2],
+    have int32 [S], nonfinite uint32 [S])."""
+    assert y.dtype == np.uint32 and y.ndim == 2 and y.flags.c_contiguous
+    rows, n = y.shape
+    so = None if seq_offsets is None else np.ascontiguousarray(seq_offsets, dtype=np.int32)
+    S = 1 if so is None else so.size - 1
+    b = np.zeros((S, 2), np.uint32)
+    k = np.zeros((S, 2), np.uint32)
+    have = np.zeros(S, np.int32)
+    nf = np.zeros(S, np.uint32)
+    lib().ft2o_bounds32(_p(y), rows, n, n, _p(so), S, scale, int(correct_nonfinite), _p(b), _p(k), _p(have), _p(nf))
+    return b, k, have, nf
+
+
+def protect32(y, bounds_, row_to_seq=None, count=None):
+    """R5 in place on binary32 bits y (uint32 [rows, n]); bounds_ uint32 [S, 2]."""
+    assert y.dtype == np.uint32 and y.ndim == 2 and y.flags.c_contiguous
+    rows, n = y.shape
+    b = _u32(bounds_).reshape(-1, 2)
+    S = b.shape[0]
+    cnt = np.zeros(S, np.uint32) if count is None else count
+    r2s = None if row_to_seq is None else np.ascontiguousarray(row_to_seq, dtype=np.int32)
+    lib().ft2o_protect32(_p(y), rows, n, n, _p(r2s), _p(b), S, _p(cnt))
+    return cnt
+
+
+def inject32(y, sites, cur_layer, cur_step, base_row=None):
+    assert y.dtype == np.uint32 and y.ndim == 2 and y.flags.c_contiguous
+    rows, n = y.shape
+    s = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
+    br = None if base_row is None else np.ascontiguousarray(base_row, dtype=np.int32)
+    lib().ft2o_inject32(_p(y), rows, n, n, _p(s), s.size, cur_layer, cur_step, _p(br))
+    return y

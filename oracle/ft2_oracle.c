@@ -440,4 +440,118 @@ EXPORT void ft2o_protected_linear_dt(const uint16_t* x, int64_t ldx, const uint1
     if (bounds) ft2o_protect_dt(y, M, N, ldy, row_to_seq, bounds, num_seqs, count, dtype);
 }
 
+
+/* ------------------------------------------------------------ FP32 --- */
+/* The paper's FP32 study (Sec. 6: FT2 "also applies to FP32
+ * models") runs the same method on 32-bit activations.  R0 for binary32:
+ * values are uint32 bit patterns, ordered by the 32-bit key
+ *     key32(b) = (b & 0x80000000) ? ~b : (b | 0x80000000)
+ * (total order on non-NaN values: -Inf = 0x007FFFFF < ... < -0 = 0x7FFFFFFF
+ * < +0 = 0x80000000 < ... < +Inf = 0xFF800000; NaN keys lie outside).
+ * Readings A2-A10 carry over unchanged; R3's product / quotient is formed in
+ * fp64 from the fp32 value and the fp32 scale (the product is exact; the
+ * quotient is one IEEE division), then rounded outward to fp32 and saturated
+ * to +-FLT_MAX. */
+EXPORT int ft2o_isnan32(uint32_t b) { return (b & 0x7FFFFFFFu) > 0x7F800000u; }
+EXPORT int ft2o_isfinite32(uint32_t b) { return (b & 0x7F800000u) != 0x7F800000u; }
+EXPORT uint32_t ft2o_key32(uint32_t b) { return (b & 0x80000000u) ? ~b : (b | 0x80000000u); }
+EXPORT uint32_t ft2o_unkey32(uint32_t k) { return (k & 0x80000000u) ? (k & 0x7FFFFFFFu) : ~k; }
+
+static float f32_of(uint32_t b) { float f; memcpy(&f, &b, 4); return f; }
+static uint32_t bits_of(float f) { uint32_t b; memcpy(&b, &f, 4); return b; }
+
+/* Outward rounding of a double to fp32 (dir -1 toward -Inf, +1 toward +Inf):
+ * the nearest fp32 (the C conversion, round-to-nearest-even), then one step
+ * outward in key order if it lies on the wrong side of d. */
+static uint32_t f64_to_f32_dir(double d, int dir) {
+    uint32_t r = bits_of((float)d);
+    double rv = (double)f32_of(r);
+    if (dir < 0 && rv > d) r = ft2o_unkey32(ft2o_key32(r) - 1u);
+    if (dir > 0 && rv < d) r = ft2o_unkey32(ft2o_key32(r) + 1u);
+    return r;
+}
+
+EXPORT uint32_t ft2o_scale_bound32(uint32_t raw, float c32, int is_hi) {
+    double x = (double)f32_of(raw), c = (double)c32;   /* the ABI's fp32 scale, exact in fp64 */
+    volatile double s;
+    if (is_hi) s = (x >= 0.0) ? x * c : x / c;
+    else       s = (x <= 0.0) ? x * c : x / c;
+    uint32_t r = f64_to_f32_dir((double)s, is_hi ? +1 : -1);
+    if (r == 0x7F800000u) r = 0x7F7FFFFFu;   /* +Inf -> +FLT_MAX (A8) */
+    if (r == 0xFF800000u) r = 0xFF7FFFFFu;   /* -Inf -> -FLT_MAX */
+    return r;
+}
+
+/* R5 for binary32 (A5-A7 as for the 16-bit formats). */
+EXPORT uint32_t ft2o_clip_value32(uint32_t y, uint32_t lo, uint32_t hi) {
+    uint32_t x = ft2o_isnan32(y) ? 0u : y;
+    uint32_t k = ft2o_key32(x);
+    if (k < ft2o_key32(lo)) return lo;
+    if (k > ft2o_key32(hi)) return hi;
+    return x;
+}
+
+EXPORT void ft2o_protect32(uint32_t* y, int64_t rows, int64_t n, int64_t ld, const int32_t* row_to_seq,
+                           const uint32_t* bounds, int32_t num_seqs, uint32_t* count) {
+    for (int64_t r = 0; r < rows; ++r) {
+        int32_t s = row_to_seq ? row_to_seq[r] : (num_seqs == 1 ? 0 : (int32_t)r);
+        if (s < 0 || s >= num_seqs) continue;
+        for (int64_t j = 0; j < n; ++j) {
+            uint32_t v = y[r * ld + j];
+            uint32_t w = ft2o_clip_value32(v, bounds[2 * s], bounds[2 * s + 1]);
+            if (w != v) {
+                y[r * ld + j] = w;
+                if (count) count[s] += 1;
+            }
+        }
+    }
+}
+
+/* R2-R4 for binary32.  raw_keys[2s], raw_keys[2s+1] = key32 of the finite
+ * min / max as uint32, have[s] = 0 when the sequence has no finite value (A9). */
+EXPORT void ft2o_bounds32(uint32_t* y, int64_t rows, int64_t n, int64_t ld, const int32_t* seq_offsets,
+                          int32_t num_seqs, float scale, int32_t correct_nonfinite, uint32_t* bounds,
+                          uint32_t* raw_keys, int32_t* have_out, uint32_t* nonfinite) {
+    for (int32_t s = 0; s < num_seqs; ++s) {
+        int64_t r0 = seq_offsets ? seq_offsets[s] : 0;
+        int64_t r1 = seq_offsets ? seq_offsets[s + 1] : rows;
+        int have = 0;
+        uint32_t kmin = 0, kmax = 0, nf = 0;
+        for (int64_t r = r0; r < r1; ++r)
+            for (int64_t j = 0; j < n; ++j) {
+                uint32_t v = y[r * ld + j];
+                if (!ft2o_isfinite32(v)) { nf++; continue; }
+                uint32_t k = ft2o_key32(v);
+                if (!have || k < kmin) kmin = k;
+                if (!have || k > kmax) kmax = k;
+                have = 1;
+            }
+        uint32_t lo = 0u, hi = 0u;
+        if (have) {
+            lo = ft2o_scale_bound32(ft2o_unkey32(kmin), scale, 0);
+            hi = ft2o_scale_bound32(ft2o_unkey32(kmax), scale, 1);
+        }
+        if (raw_keys) { raw_keys[2 * s] = kmin; raw_keys[2 * s + 1] = kmax; }
+        if (have_out) have_out[s] = have;
+        if (bounds) { bounds[2 * s] = lo; bounds[2 * s + 1] = hi; }
+        if (nonfinite) nonfinite[s] = nf;
+        if (correct_nonfinite)
+            for (int64_t r = r0; r < r1; ++r)
+                for (int64_t j = 0; j < n; ++j)
+                    y[r * ld + j] = ft2o_clip_value32(y[r * ld + j], lo, hi);
+    }
+}
+
+/* R7 for binary32: the 32-bit mask of the site (dtype 2 in ft2o_make_sites). */
+EXPORT void ft2o_inject32(uint32_t* y, int64_t rows, int64_t n, int64_t ld, const ft2o_site* sites,
+                          int32_t n_sites, int32_t cur_layer, int32_t cur_step, const int32_t* base_row) {
+    for (int32_t i = 0; i < n_sites; ++i) {
+        const ft2o_site* s = &sites[i];
+        if ((int32_t)s->step != cur_step || (int32_t)s->layer != cur_layer) continue;
+        int64_t row = (base_row ? base_row[i] : i) + (cur_step == 0 ? (int64_t)s->token : 0);
+        if (row < 0 || row >= rows || (int64_t)s->col >= n) continue;
+        y[row * ld + s->col] ^= s->xor_mask;
+    }
+}
+
 EXPORT int32_t ft2o_site_size(void) { return (int32_t)sizeof(ft2o_site); }

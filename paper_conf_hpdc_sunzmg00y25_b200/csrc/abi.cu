@@ -31,12 +31,16 @@ static std::atomic<uint64_t> g_launches{0};
 
 static inline bool al16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
+// elements per 16-byte vector: 8 for the 16-bit formats, 4 for binary32
+static inline int64_t vec_elems(int32_t dtype) { return dtype == FT2_FP32 ? 4 : 8; }
+
 static ft2_status check_tensor(const ft2_tensor& t, bool allow_null_if_empty = true) {
     if (t.rows < 0 || t.n < 0 || t.ld < t.n) return FT2_ERR_INVALID_ARG;
-    if (t.dtype != FT2_BF16 && t.dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
+    if (t.dtype != FT2_BF16 && t.dtype != FT2_FP16 && t.dtype != FT2_FP32) return FT2_ERR_UNSUPPORTED;
     if (t.rows == 0 || t.n == 0) return FT2_OK;
     if (t.data == nullptr) return FT2_ERR_INVALID_ARG;
-    if (!al16(t.data) || (t.n % 8) != 0 || (t.ld % 8) != 0) return FT2_ERR_MISALIGNED;
+    const int64_t ve = vec_elems(t.dtype);
+    if (!al16(t.data) || (t.n % ve) != 0 || (t.ld % ve) != 0) return FT2_ERR_MISALIGNED;
     (void)allow_null_if_empty;
     return FT2_OK;
 }
@@ -70,9 +74,9 @@ ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int
     if (!finalize && keys_out == nullptr) return FT2_ERR_INVALID_ARG;
     if (correct_nonfinite && !finalize) return FT2_ERR_INVALID_ARG;
     if (seq_offsets == nullptr && num_seqs != 1) return FT2_ERR_INVALID_ARG;
-    if (((uintptr_t)workspace & 7u) != 0 || (bounds_out && ((uintptr_t)bounds_out & 3u) != 0))
+    if (((uintptr_t)workspace & 7u) != 0 || (bounds_out && ((uintptr_t)bounds_out & (y.dtype == FT2_FP32 ? 7u : 3u)) != 0))
         return FT2_ERR_MISALIGNED;
-    if ((y.rows * (y.n / 8)) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
+    if ((y.rows * (y.n / vec_elems(y.dtype))) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
     if (y.rows == 0 || y.n == 0) {
         // nothing to reduce: every sequence is empty (reading A9) -- still a
         // well-defined result, produced by the finalize kernel on "no value" keys
@@ -96,7 +100,8 @@ ft2_status ft2_bounds_from_prefill(ft2_tensor y, const int32_t* seq_offsets, int
     a.ws = static_cast<uint32_t*>(workspace);
     a.dtype = y.dtype;
     int nl = 0;
-    cudaError_t e = launch_bounds(a, static_cast<cudaStream_t>(stream), &nl);
+    cudaError_t e = y.dtype == FT2_FP32 ? launch_bounds32(a, static_cast<cudaStream_t>(stream), &nl)
+                                        : launch_bounds(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
 }
 
@@ -104,10 +109,13 @@ ft2_status ft2_bounds_finalize(const int32_t* keys, int32_t num_seqs, float scal
                                void* bounds_out, void* stream) {
     if (keys == nullptr || bounds_out == nullptr || num_seqs < 1) return FT2_ERR_INVALID_ARG;
     if (!(std::isfinite(scale)) || scale < 1.0f) return FT2_ERR_INVALID_ARG;
-    if (dtype != FT2_BF16 && dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
+    if (dtype != FT2_BF16 && dtype != FT2_FP16 && dtype != FT2_FP32) return FT2_ERR_UNSUPPORTED;
+    if (((uintptr_t)bounds_out & (dtype == FT2_FP32 ? 7u : 3u)) != 0) return FT2_ERR_MISALIGNED;
     int nl = 0;
-    cudaError_t e = launch_finalize(keys, num_seqs, scale, static_cast<uint16_t*>(bounds_out), (int)dtype,
-                                    static_cast<cudaStream_t>(stream), &nl);
+    cudaError_t e = dtype == FT2_FP32
+                        ? launch_finalize32(keys, num_seqs, scale, bounds_out, static_cast<cudaStream_t>(stream), &nl)
+                        : launch_finalize(keys, num_seqs, scale, static_cast<uint16_t*>(bounds_out), (int)dtype,
+                                          static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
 }
 
@@ -117,8 +125,8 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
     if (s != FT2_OK) return s;
     if (num_seqs < 1 || bounds == nullptr) return FT2_ERR_INVALID_ARG;
     if (row_to_seq == nullptr && num_seqs != 1 && (int64_t)num_seqs != y.rows) return FT2_ERR_INVALID_ARG;
-    if (((uintptr_t)bounds & 3u) != 0) return FT2_ERR_MISALIGNED;
-    if ((y.rows * (y.n / 8)) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
+    if (((uintptr_t)bounds & (y.dtype == FT2_FP32 ? 7u : 3u)) != 0) return FT2_ERR_MISALIGNED;
+    if ((y.rows * (y.n / vec_elems(y.dtype))) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
     if (y.rows == 0 || y.n == 0) return FT2_OK;
     ProtectArgs a;
     a.y = static_cast<uint16_t*>(y.data);
@@ -131,7 +139,8 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
     a.counts = corrected_count;
     a.dtype = y.dtype;
     int nl = 0;
-    cudaError_t e = launch_protect(a, static_cast<cudaStream_t>(stream), &nl);
+    cudaError_t e = y.dtype == FT2_FP32 ? launch_protect32(a, static_cast<cudaStream_t>(stream), &nl)
+                                        : launch_protect(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
 }
 
@@ -274,11 +283,16 @@ ft2_status ft2_make_fault_sites(uint64_t seed, uint64_t trial0, int32_t n_trials
 ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
                              int32_t cur_step, const int32_t* base_row, void* stream) {
     if (y.rows < 0 || y.n < 0 || y.ld < y.n) return FT2_ERR_INVALID_ARG;
-    if (y.dtype != FT2_BF16 && y.dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
+    if (y.dtype != FT2_BF16 && y.dtype != FT2_FP16 && y.dtype != FT2_FP32) return FT2_ERR_UNSUPPORTED;
     if (n_sites < 0) return FT2_ERR_INVALID_ARG;
     if (n_sites == 0 || y.rows == 0 || y.n == 0) return FT2_OK;
     if (sites == nullptr || y.data == nullptr) return FT2_ERR_INVALID_ARG;
     int nl = 0;
+    if (y.dtype == FT2_FP32) {
+        cudaError_t e = launch_inject32(y.data, y.rows, y.n, y.ld, sites, n_sites, cur_layer, cur_step, base_row,
+                                        static_cast<cudaStream_t>(stream), &nl);
+        return finish(e, nl);
+    }
     cudaError_t e = launch_inject(static_cast<uint16_t*>(y.data), y.rows, y.n, y.ld, sites, n_sites, cur_layer,
                                   cur_step, base_row, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);

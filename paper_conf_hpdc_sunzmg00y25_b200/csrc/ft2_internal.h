@@ -29,7 +29,7 @@ struct BoundsArgs {
     uint32_t* nonfinite_out;
     uint32_t* nv_out;  // NaN-vulnerable counts or NULL
     uint32_t* ws;
-    int32_t dtype;  // FT2_BF16 or FT2_FP16
+    int32_t dtype;  // FT2_BF16, FT2_FP16 (bounds.cu) or FT2_FP32 (f32.cu)
 };
 cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch);
 cudaError_t launch_finalize(const int32_t* keys, int32_t S, float scale, uint16_t* out, int dtype,
@@ -89,6 +89,16 @@ struct PrefillDerive {
 };
 // Persistent 128x256-tile tcgen05 GEMM for M > 128 (PLAIN / CHECK, or DERIVE when d != NULL)
 cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaStream_t st, int* n_launch);
+
+// binary32 variants (f32.cu; the paper's FP32 study).  The
+// 16-bit argument structs are reused: y / bounds point at 32-bit elements.
+cudaError_t launch_bounds32(const BoundsArgs& a, cudaStream_t st, int* n_launch);
+cudaError_t launch_finalize32(const int32_t* keys, int32_t S, float scale, void* out, cudaStream_t st,
+                              int* n_launch);
+cudaError_t launch_protect32(const ProtectArgs& a, cudaStream_t st, int* n_launch);
+cudaError_t launch_inject32(void* y, int64_t rows, int64_t n, int64_t ld, const ft2_fault_site* sites,
+                            int32_t n_sites, int32_t layer, int32_t step, const int32_t* base_row,
+                            cudaStream_t st, int* n_launch);
 
 int num_sms();
 

@@ -10,15 +10,15 @@ import ctypes
 import torch
 
 from . import _lib
-from ._lib import (FT2_BF16, FT2_FP16, FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FaultSite, SiteGeometry, Tensor, check,
+from ._lib import (FT2_BF16, FT2_FP16, FT2_FP32, FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FaultSite, SiteGeometry, Tensor, check,
                    load)
 
-_DTYPES = {torch.bfloat16: FT2_BF16, torch.float16: FT2_FP16}
+_DTYPES = {torch.bfloat16: FT2_BF16, torch.float16: FT2_FP16, torch.float32: FT2_FP32}
 
 
 def _dtype_of(t: torch.Tensor) -> int:
     if t.dtype not in _DTYPES:
-        raise TypeError(f"ft2: unsupported activation dtype {t.dtype} (bfloat16 / float16)")
+        raise TypeError(f"ft2: unsupported activation dtype {t.dtype} (bfloat16 / float16 / float32)")
     return _DTYPES[t.dtype]
 
 SITE_BYTES = ctypes.sizeof(FaultSite)

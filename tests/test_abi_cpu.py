@@ -58,8 +58,13 @@ def test_validation_without_gpu(L):
     # misaligned base, n % 8
     assert L.ft2_protect(Tensor(0x1002, 4, 16, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
     assert L.ft2_protect(Tensor(0x1000, 4, 12, 16, 0), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
-    # dtype not implemented (FP32); FP16 passes validation
-    assert L.ft2_protect(Tensor(0x1000, 4, 16, 16, 2), None, P(0x2000), 1, None, None) == FT2_ERR_UNSUPPORTED
+    # unknown dtype; FP32 (16-byte vectors of 4): n % 4, fp32 bounds 8-byte aligned
+    assert L.ft2_protect(Tensor(0x1000, 4, 16, 16, 3), None, P(0x2000), 1, None, None) == FT2_ERR_UNSUPPORTED
+    assert L.ft2_protect(Tensor(0x1000, 4, 6, 8, 2), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
+    assert L.ft2_protect(Tensor(0x1000, 4, 8, 10, 2), None, P(0x2000), 1, None, None) == FT2_ERR_MISALIGNED
+    assert L.ft2_protect(Tensor(0x1000, 4, 8, 8, 2), None, P(0x2004), 1, None, None) == FT2_ERR_MISALIGNED
+    assert L.ft2_bounds_finalize(P(0x1000), 1, 2.0, 3, P(0x2000), None) == FT2_ERR_UNSUPPORTED
+    # the fused GEMMs are bf16/fp16 tensor-core contractions: FP32 is unsupported
     assert L.ft2_protect_fused_gemm(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, 4, 16, 16, 0, 2, 0, 16,
                                     None, None, 0, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_UNSUPPORTED
     # zero-size -> OK with no launch
