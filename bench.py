@@ -411,6 +411,8 @@ def main():
         dec_us = 1000.0 * phases["fused"]["decode_ms_per_step"]
         # the kernel's share of a decode step (compare with the ncu launch list in profiles/)
         rf["share_of_decode_step"] = rf["launches_per_graph"] * rf["avg_launch_us"] / dec_us
+    if not args.no_extras:
+        res["coverage_overhead_pct"] = coverage_costs(cfg, B, T, G, dev, prompt, stream, runner, ms_off)
     if rank == 0 and world == 1 and not args.no_extras:
         cb = oracle_sample(args.model, B, T, G)
         res["cpu_baseline"] = {"value": cb["tokens_per_s"], "unit": "tokens/s", "cores": cb["cores"],
@@ -420,6 +422,44 @@ def main():
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def coverage_costs(cfg, B, T, G, dev, prompt, stream, runner_ft2, ms_off_ft2, rounds=5):
+    """FT2 overhead under the protection coverages of PAPER.md Table 1
+    (L164-L177): FT2's critical layers, MaxiMals' (out_proj, fc2),
+    Global Clipper's (v_proj, out_proj), and every linear layer (the "nearly
+    2x" cost of protecting all layers, L160).  Each coverage runs its own
+    runner (same seeded weights); fused vs off medians of interleaved requests."""
+    import torch
+
+    from paper_conf_hpdc_sunzmg00y25_b200.runner import Runner
+
+    def one(r, mode):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        r.generate(prompt, mode)
+        b.record(stream)
+        return a, b
+
+    out = {}
+    for cov in ("ft2", "maximals", "globalclipper", "all"):
+        r = runner_ft2 if cov == "ft2" else Runner(cfg, B, T, G, seed=1, device=dev, coverage=cov)
+        for m in ("fused", "off"):
+            for _ in range(4):
+                r.generate(prompt, m)
+        samples = {"fused": [], "off": []}
+        for _ in range(rounds):
+            evs = [(m, one(r, m)) for m in ("fused", "off")]
+            torch.cuda.synchronize()
+            for m, (a, b) in evs:
+                samples[m].append(a.elapsed_time(b))
+        f, o = statistics.median(samples["fused"]), statistics.median(samples["off"])
+        out[cov] = {"protected_layers": r.n_crit, "overhead_pct": 100.0 * (1 - o / f), "ms_fused": f, "ms_off": o}
+        if r is not runner_ft2:
+            del r
+            torch.cuda.empty_cache()
+    out["note"] = "Table 1 coverages (MaxiMals: out_proj+fc2; Global Clipper: v_proj+out_proj; all linear layers)"
+    return out
 
 
 def kernel_rooflines(runner, dev, ft2):
@@ -614,6 +654,7 @@ def c4_tp_bounds(args, dev, rank, world, B=32, T=128, blocks=40, R=20):
         dist.all_reduce(f, op=dist.ReduceOp.MAX)
         exact = int(f.item()) == 0
     shard_bytes = sum(rows * (e - b) * 2 for _, b, e in col_layers) + sum(y.numel() * 2 for y in row_layers)
+    row_parallel = c4_row_parallel_decode(dev, world, B, blocks, dev_time)
     return {"leg": "c4", "metric": "TP first-token bounds phase per prefill (us, max over ranks)", "value": us_phase,
             "unit": "us", "higher_is_better": False, "n_gpus": world, "scaling": "strong",
             "config": {"workload": "llama-2-13b-shaped critical layers, TP over the ranks (configs[3]): "
@@ -623,7 +664,70 @@ def c4_tp_bounds(args, dev, rank, world, B=32, T=128, blocks=40, R=20):
             "allreduce_us": us_ar, "allreduce_bytes": keys.numel() * 4,
             "bounds_bitexact_vs_unsharded": exact,
             "per_rank_bytes_swept": shard_bytes, "l2": "4 distinct tensors per layer class rotated (> L2)",
-            "per_rank_GBps": shard_bytes / (us_phase * 1e-6) / 1e9}
+            "per_rank_GBps": shard_bytes / (us_phase * 1e-6) / 1e9,
+            "row_parallel_decode": row_parallel}
+
+
+def c4_row_parallel_decode(dev, world, B, blocks, dev_time, n=5120, R=20):
+    """Decode-time check of the 2*blocks row-parallel critical layers (o_proj,
+    down_proj; [B, 5120] outputs) after their sum all-reduce (reading A17):
+    NCCL all_reduce + ft2_protect (two launches per layer) against the fused
+    one-shot ft2_allreduce_protect over CUDA IPC peer memory (NEXT(2)).  One
+    CUDA graph of 2*blocks layers per variant; us per decode step, max over
+    ranks."""
+    import torch
+    import torch.distributed as dist
+
+    import ft2_synth
+    import paper_conf_hpdc_sunzmg00y25_b200 as ft2
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+
+    if world > 1:
+        rpc = tp.RowParallelCheck(B, n)
+    else:
+        import socket
+        if not dist.is_initialized():
+            s = socket.socket()
+            s.bind(("127.0.0.1", 0))
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ["MASTER_PORT"] = str(s.getsockname()[1])
+            s.close()
+            dist.init_process_group("gloo", rank=0, world_size=1)
+        rpc = tp.RowParallelCheck(B, n)
+    L = 2 * blocks
+    part = ft2_synth.gen_bf16_torch((B, n), 970, 5, device=dev)
+    rpc.partials[0].copy_(part)
+    rpc.partials[1].copy_(part)
+    bias = ft2_synth.gen_bf16_torch((n,), 971, 5, device=dev)
+    bnd = torch.tensor([[-3.0e38, 3.0e38]], dtype=torch.bfloat16, device=dev).repeat(B, 1)
+    cnt = torch.zeros(B, dtype=torch.int32, device=dev)
+    ys = [torch.empty((B, n), dtype=torch.bfloat16, device=dev) for _ in range(L)]
+    bufs = [part.clone() for _ in range(L)]
+
+    def nccl_protect():
+        for i in range(L):
+            if world > 1:
+                dist.all_reduce(bufs[i])
+            ft2.protect(bufs[i], bnd, num_seqs=B, corrected_count=cnt)
+
+    def fused():
+        for i in range(L):
+            rpc(i, ys[i], bias=bias, mode=1, bounds=bnd, num_seqs=B, corrected_count=cnt)
+
+    out = {"layers": L, "shape": [B, n], "tp": world}
+    for name, fn in (("nccl_allreduce_plus_protect", nccl_protect), ("fused_allreduce_protect", fused)):
+        s_ = torch.cuda.Stream()
+        s_.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s_):
+            fn()
+        torch.cuda.current_stream().wait_stream(s_)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            fn()
+        out[name + "_us_per_step"] = dev_time(g.replay, R)
+    out["status"] = rpc.status()
+    return out
 
 
 def c5_campaign(args, dev, rank, world, model="llama-2-7b", B=256, T=16, S=32):

@@ -282,6 +282,46 @@ ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t 
                              int32_t cur_layer, int32_t cur_step, const int32_t* base_row,
                              void* stream);
 
+/* Tensor-parallel row-parallel critical layer (o_proj / down_proj / out_proj /
+ * fc2 under Megatron TP): its sum all-reduce fused with the check
+ * (reading A17: row-parallel outputs are checked
+ * after their sum all-reduce, PAPER.md L259-L272 for the check).  One-shot,
+ * over peer memory (NVLink / NVSwitch through CUDA IPC mappings, ft2_ipc_*):
+ *   y[r, c] = check(inject(rne(((p_0 + p_1) + ... + p_{P-1}) + bias[c])))
+ * summed in fp32 in rank order 0..P-1 (reading A22), so every rank computes
+ * the same bits; the check is ft2_protect's (FT2_GEMM_CHECK) or none
+ * (FT2_GEMM_PLAIN: a plain one-shot all-reduce).
+ * partials     device array [P] of device pointers: rank t's partial output
+ *              [rows x n] (16-bit, row stride ldp) as mapped in THIS process
+ *              (this rank's own buffer at index rank).  Double-buffer them:
+ *              alternate two buffers per call.
+ * flags        device array [P] of device pointers: rank t's flag array of P
+ *              uint32 (zero-filled once, before the first call of any rank).
+ * epoch, done, status  this rank's device uint32 words (zero-filled once):
+ *              the call counter, a self-cleaning CTA counter, and an error
+ *              word set to 1 if a peer did not arrive within 2^24 polls
+ *              (the kernel then returns without writing y).
+ * y            this rank's output [rows x n] (ld), 16-bit (bf16 / fp16).
+ * bias, row_to_seq, bounds, num_seqs, corrected_count, sites, n_sites,
+ * cur_layer, cur_step, base_row: as in ft2_protect_fused_gemm / ft2_protect.
+ * Every rank must make the same sequence of calls with the same shapes.
+ * Asynchronous on stream; graph-capturable (the epoch lives in device memory). */
+ft2_status ft2_allreduce_protect(const void* const* partials, int64_t ldp, int32_t P, int32_t rank,
+                                 uint32_t* const* flags, uint32_t* epoch, uint32_t* done, uint32_t* status,
+                                 ft2_tensor y, const void* bias, ft2_gemm_mode mode,
+                                 const int32_t* row_to_seq, const void* bounds, int32_t num_seqs,
+                                 uint32_t* corrected_count, const ft2_fault_site* sites, int32_t n_sites,
+                                 int32_t cur_layer, int32_t cur_step, const int32_t* base_row, void* stream);
+
+/* CUDA IPC plumbing for ft2_allreduce_protect's buffers (setup time, not
+ * the hot path): export the device allocation holding dev_ptr as a 64-byte
+ * handle (host buffer) plus dev_ptr's byte offset inside it; map a peer's
+ * handle into this process (the allocation's base; add the offset; peer
+ * access is enabled lazily) and unmap it again with ft2_ipc_close(base). */
+ft2_status ft2_ipc_get_handle(void* dev_ptr, void* handle_out, uint64_t* offset_out);
+ft2_status ft2_ipc_open_handle(const void* handle, void** dev_ptr_out);
+ft2_status ft2_ipc_close(void* dev_ptr);
+
 /* Human-readable status. */
 const char* ft2_status_string(ft2_status s);
 

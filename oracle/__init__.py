@@ -95,6 +95,8 @@ def lib():
             ("ft2o_protect32", None, [P, i64, i64, i64, P, P, i32, P]),
             ("ft2o_bounds32", None, [P, i64, i64, i64, P, i32, ctypes.c_float, i32, P, P, P, P]),
             ("ft2o_inject32", None, [P, i64, i64, i64, P, i32, i32, i32, P]),
+            ("ft2o_allreduce_protect", None, [P, i32, i64, i64, P, i32, P, P, i32, P, P, i32, i32, i32, P, P,
+                                              ctypes.c_int]),
         ]:
             f = getattr(L, name)
             f.restype = res
@@ -292,3 +294,21 @@ def inject32(y, sites, cur_layer, cur_step, base_row=None):
     br = None if base_row is None else np.ascontiguousarray(base_row, dtype=np.int32)
     lib().ft2o_inject32(_p(y), rows, n, n, _p(s), s.size, cur_layer, cur_step, _p(br))
     return y
+
+
+def allreduce_protect(partials, bias=None, bounds_=None, row_to_seq=None, sites=None, cur_layer=0, cur_step=0,
+                      base_row=None, dtype=DT_BF16):
+    """Reading A22 + A17: partials uint16 [P, rows, n] -> (y uint16 [rows, n], count [S])."""
+    pp = np.ascontiguousarray(partials, dtype=np.uint16)
+    P, rows, n = pp.shape
+    y = np.zeros((rows, n), np.uint16)
+    b = None if bias is None else np.ascontiguousarray(bias, dtype=np.uint16)
+    bd = None if bounds_ is None else np.ascontiguousarray(bounds_, dtype=np.uint16).reshape(-1, 2)
+    S = 0 if bd is None else bd.shape[0]
+    cnt = np.zeros(max(S, 1), np.uint32)
+    r2s = None if row_to_seq is None else np.ascontiguousarray(row_to_seq, dtype=np.int32)
+    s = None if sites is None else np.ascontiguousarray(sites, dtype=SITE_DTYPE)
+    br = None if base_row is None else np.ascontiguousarray(base_row, dtype=np.int32)
+    lib().ft2o_allreduce_protect(_p(pp), P, rows, n, _p(b), int(bd is not None), _p(r2s), _p(bd), S, _p(cnt),
+                                 _p(s), 0 if s is None else s.size, cur_layer, cur_step, _p(br), _p(y), dtype)
+    return y, cnt[:S]

@@ -554,4 +554,31 @@ EXPORT void ft2o_inject32(uint32_t* y, int64_t rows, int64_t n, int64_t ld, cons
     }
 }
 
+
+/* ------------------------------------------------------ NEXT(2) / A22 --- */
+/* Row-parallel critical layer under tensor parallelism: the sum all-reduce of
+ * the P ranks' partial outputs followed by the check (reading A17: check after
+ * the sum all-reduce).  Reading A22 fixes the reduction:
+ * the partials (16-bit) are summed in fp32 in rank order,
+ *     acc = f32(p_0); acc = fl32(acc + f32(p_t)) for t = 1..P-1;
+ *     acc = fl32(acc + f32(bias[c]))  (if bias),
+ * then rounded once to the 16-bit format (RNE), then R7 (inject), then R5.
+ * partials: [P][rows][n] contiguous. */
+EXPORT void ft2o_allreduce_protect(const uint16_t* partials, int32_t P, int64_t rows, int64_t n,
+                                   const uint16_t* bias, int32_t check, const int32_t* row_to_seq,
+                                   const uint16_t* bounds, int32_t num_seqs, uint32_t* count,
+                                   const ft2o_site* sites, int32_t n_sites, int32_t cur_layer, int32_t cur_step,
+                                   const int32_t* base_row, uint16_t* y, int dtype) {
+    for (int64_t r = 0; r < rows; ++r)
+        for (int64_t c = 0; c < n; ++c) {
+            volatile float acc = (float)ft2o_to_f64_dt(partials[r * n + c], dtype);
+            for (int32_t t = 1; t < P; ++t)
+                acc = acc + (float)ft2o_to_f64_dt(partials[((int64_t)t * rows + r) * n + c], dtype);
+            if (bias) acc = acc + (float)ft2o_to_f64_dt(bias[c], dtype);
+            y[r * n + c] = ft2o_f64_to_dt_rne((double)acc, dtype);
+        }
+    if (sites && n_sites > 0) ft2o_inject(y, rows, n, n, sites, n_sites, cur_layer, cur_step, base_row);
+    if (check) ft2o_protect_dt(y, rows, n, n, row_to_seq, bounds, num_seqs, count, dtype);
+}
+
 EXPORT int32_t ft2o_site_size(void) { return (int32_t)sizeof(ft2o_site); }

@@ -41,7 +41,7 @@ assert ctypes.sizeof(FaultSite) == 24
 EXPORTS = [
     "ft2_workspace_bytes", "ft2_bounds_from_prefill", "ft2_bounds_finalize", "ft2_protect",
     "ft2_gemm_workspace_bytes", "ft2_protect_fused_gemm", "ft2_prefill_fused_gemm", "ft2_make_fault_sites",
-    "ft2_inject_faults",
+    "ft2_inject_faults", "ft2_allreduce_protect", "ft2_ipc_get_handle", "ft2_ipc_open_handle", "ft2_ipc_close",
     "ft2_status_string", "ft2_launch_count", "ft2_version",
 ]
 
@@ -71,6 +71,11 @@ def load(path: str = LIB):
         "ft2_make_fault_sites": (st, [u64, u64, i32, ctypes.c_int, ctypes.c_int, ctypes.POINTER(SiteGeometry),
                                       P, P]),
         "ft2_inject_faults": (st, [Tensor, P, i32, i32, i32, P, P]),
+        "ft2_allreduce_protect": (st, [P, i64, i32, i32, P, P, P, P, Tensor, P, ctypes.c_int, P, P, i32, P, P, i32,
+                                       i32, i32, P, P]),
+        "ft2_ipc_get_handle": (st, [P, P, ctypes.POINTER(ctypes.c_uint64)]),
+        "ft2_ipc_open_handle": (st, [P, ctypes.POINTER(ctypes.c_void_p)]),
+        "ft2_ipc_close": (st, [P]),
         "ft2_status_string": (ctypes.c_char_p, [ctypes.c_int]),
         "ft2_launch_count": (ctypes.c_uint64, []),
         "ft2_version": (ctypes.c_char_p, []),

@@ -1,10 +1,12 @@
 // abi.cu -- the C ABI of libft2.so (include/ft2.h): argument validation,
 // status codes, launch bookkeeping.  All compute happens in the kernels of
 // bounds.cu, protect.cu, faults.cu and gemm_sm100.cu.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <atomic>
 #include <cmath>
+#include <cstring>
 
 #include "ft2_internal.h"
 
@@ -296,6 +298,100 @@ ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t 
     cudaError_t e = launch_inject(static_cast<uint16_t*>(y.data), y.rows, y.n, y.ld, sites, n_sites, cur_layer,
                                   cur_step, base_row, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);
+}
+
+ft2_status ft2_allreduce_protect(const void* const* partials, int64_t ldp, int32_t P, int32_t rank,
+                                 uint32_t* const* flags, uint32_t* epoch, uint32_t* done, uint32_t* status,
+                                 ft2_tensor y, const void* bias, ft2_gemm_mode mode, const int32_t* row_to_seq,
+                                 const void* bounds, int32_t num_seqs, uint32_t* corrected_count,
+                                 const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer, int32_t cur_step,
+                                 const int32_t* base_row, void* stream) {
+    ft2_status s = check_tensor(y);
+    if (s != FT2_OK) return s;
+    if (y.dtype == FT2_FP32) return FT2_ERR_UNSUPPORTED;
+    if (P < 1 || P > 64 || rank < 0 || rank >= P) return FT2_ERR_INVALID_ARG;
+    if (partials == nullptr || flags == nullptr || epoch == nullptr || done == nullptr || status == nullptr)
+        return FT2_ERR_INVALID_ARG;
+    const int32_t m = (int32_t)mode & ~FT2_GEMM_W_STATIC;
+    if (m != FT2_GEMM_PLAIN && m != FT2_GEMM_CHECK) return FT2_ERR_INVALID_ARG;
+    if (m == FT2_GEMM_CHECK && (bounds == nullptr || num_seqs < 1)) return FT2_ERR_INVALID_ARG;
+    if (m == FT2_GEMM_CHECK && row_to_seq == nullptr && num_seqs != 1 && (int64_t)num_seqs != y.rows)
+        return FT2_ERR_INVALID_ARG;
+    if (ldp < y.n || (ldp % 8) != 0) return ldp < y.n ? FT2_ERR_INVALID_ARG : FT2_ERR_MISALIGNED;
+    if ((bias && !al16(bias)) || (bounds && ((uintptr_t)bounds & 3u) != 0)) return FT2_ERR_MISALIGNED;
+    if (n_sites < 0 || (n_sites > 0 && sites == nullptr)) return FT2_ERR_INVALID_ARG;
+    if ((y.rows * (y.n / 8)) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
+    if (y.rows == 0 || y.n == 0) return FT2_OK;   // identical on every rank: nobody waits
+    AllreduceProtectArgs a;
+    a.partials = reinterpret_cast<const uint16_t* const*>(partials);
+    a.ldp = ldp;
+    a.P = P;
+    a.rank = rank;
+    a.flags = flags;
+    a.epoch = epoch;
+    a.done = done;
+    a.status = status;
+    a.y = static_cast<uint16_t*>(y.data);
+    a.ldy = y.ld;
+    a.rows = y.rows;
+    a.n = y.n;
+    a.bias = static_cast<const uint16_t*>(bias);
+    a.mode = m;
+    a.row_to_seq = row_to_seq;
+    a.bounds = static_cast<const uint16_t*>(bounds);
+    a.S = num_seqs;
+    a.counts = corrected_count;
+    a.sites = sites;
+    a.n_sites = sites ? n_sites : 0;
+    a.cur_layer = cur_layer;
+    a.cur_step = cur_step;
+    a.base_row = base_row;
+    a.dtype = y.dtype;
+    int nl = 0;
+    cudaError_t e = launch_allreduce_protect(a, static_cast<cudaStream_t>(stream), &nl);
+    return finish(e, nl);
+}
+
+ft2_status ft2_ipc_get_handle(void* dev_ptr, void* handle_out, uint64_t* offset_out) {
+    if (dev_ptr == nullptr || handle_out == nullptr || offset_out == nullptr) return FT2_ERR_INVALID_ARG;
+    // IPC handles name whole allocations: find the allocation holding dev_ptr
+    // (a caching allocator hands out sub-ranges) and report the offset into it
+    typedef CUresult (*GetRange)(CUdeviceptr*, size_t*, CUdeviceptr);
+    static GetRange get_range = [] {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            fn = nullptr;
+        return reinterpret_cast<GetRange>(fn);
+    }();
+    if (get_range == nullptr) return FT2_ERR_CUDA;
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (get_range(&base, &size, (CUdeviceptr)dev_ptr) != CUDA_SUCCESS) return FT2_ERR_CUDA;
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, (void*)base) != cudaSuccess) { cudaGetLastError(); return FT2_ERR_CUDA; }
+    static_assert(sizeof(h) == 64, "cudaIpcMemHandle_t is 64 bytes");
+    memcpy(handle_out, &h, sizeof(h));
+    *offset_out = (uint64_t)((CUdeviceptr)dev_ptr - base);
+    return FT2_OK;
+}
+
+ft2_status ft2_ipc_open_handle(const void* handle, void** dev_ptr_out) {
+    if (handle == nullptr || dev_ptr_out == nullptr) return FT2_ERR_INVALID_ARG;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    if (cudaIpcOpenMemHandle(dev_ptr_out, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        return FT2_ERR_CUDA;
+    }
+    return FT2_OK;
+}
+
+ft2_status ft2_ipc_close(void* dev_ptr) {
+    if (dev_ptr == nullptr) return FT2_ERR_INVALID_ARG;
+    if (cudaIpcCloseMemHandle(dev_ptr) != cudaSuccess) { cudaGetLastError(); return FT2_ERR_CUDA; }
+    return FT2_OK;
 }
 
 const char* ft2_status_string(ft2_status s) {

@@ -1,0 +1,178 @@
+// allreduce_protect.cu -- a tensor-parallel row-parallel critical layer's sum
+// all-reduce fused with FT2's check (reading A17:
+// row-parallel outputs are checked after their sum all-reduce).
+//
+// Each of the P ranks holds a partial output [rows x n] of the layer (its
+// K-slice of the GEMM, 16-bit, no bias) in a buffer every peer can address
+// (CUDA IPC mappings over NVLink/NVSwitch; ft2_ipc_*).  One kernel per rank:
+//
+//   1. signal: CTA 0 publishes this call's epoch into every peer's flag slot
+//      for this rank (fence.sc.sys, then st.release.sys);
+//   2. wait: every CTA polls its own P flag slots (ld.acquire.sys) until all
+//      ranks reached the epoch -- every partial of this call is complete;
+//   3. one-shot reduce of this CTA's contiguous chunk of 16-byte vectors:
+//      the P partials are summed in fp32 in rank order 0..P-1 (identical
+//      arithmetic on every rank, so every rank ends with the same bits),
+//      + bias, rounded to the 16-bit format (RNE), fault XOR, key-space
+//      check-and-clip (readings A5-A7, A19, A20),
+//      stored to this rank's own output;
+//   4. the last CTA bumps the rank's epoch counter (device memory, so the
+//      kernel is CUDA-graph replayable).
+//
+// The partial buffers must be double-buffered by the caller (alternate per
+// call): a rank reaches call e+1's signal only after its call e finished
+// reading, so a buffer written at call e+2 is never read by a late peer.
+// Polling is bounded: after 2^24 polls (seconds) the kernel records FT2 status 1 in
+// `status` and returns (a dead peer cannot hang the GPU).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "ft2_device.cuh"
+#include "ft2_internal.h"
+#include "sm100_ptx.cuh"
+
+namespace ft2impl {
+using namespace ft2dev;
+
+namespace {
+
+constexpr int kARThreads = 256;
+constexpr int kARSites = 64;
+
+__device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+// peer data written during this kernel's lifetime: strong (sys-scope) loads,
+// never the non-coherent path
+__device__ __forceinline__ uint4 ld_relaxed_sys_v4(const void* p) {
+    uint4 r;
+    asm volatile("ld.relaxed.sys.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
+    return r;
+}
+
+template <int DT>
+__device__ __forceinline__ void add8(float (&acc)[8], uint4 v, bool first) {
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        const float f = to_f32<DT>((uint16_t)(w[j >> 1] >> ((j & 1) * 16)));
+        acc[j] = first ? f : __fadd_rn(acc[j], f);
+    }
+}
+
+template <int DT>
+__global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const AllreduceProtectArgs p, uint32_t chunk,
+                                                                       uint32_t n8, uint32_t total_vec, FastDiv div_n8,
+                                                                       int row_mode) {
+    __shared__ uint32_t sh_e, sh_ok, sh_last, sh_ns;
+    __shared__ uint32_t sh_site_e[kARSites], sh_site_m[kARSites];
+    const int tid = threadIdx.x;
+    const uint32_t v0 = blockIdx.x * chunk, v1 = min(v0 + chunk, total_vec);
+    if (tid == 0) {
+        sh_e = *reinterpret_cast<volatile uint32_t*>(p.epoch) + 1u;
+        sh_ok = 1u;
+        sh_ns = 0u;
+    }
+    __syncthreads();
+    const uint32_t e = sh_e;
+    // ---- 1. signal: my partial (written by the preceding kernel) is ready
+    if (blockIdx.x == 0 && tid < p.P) {
+        __threadfence_system();
+        st_release_sys(p.flags[tid] + p.rank, e);
+    }
+    // ---- 2. wait for every rank's partial of this call
+    if (tid < p.P) {
+        const uint32_t* f = p.flags[p.rank] + tid;
+        uint32_t polls = 0;
+        while ((int32_t)(ld_acquire_sys(f) - e) < 0) {
+            if (++polls > (1u << 24)) { atomicExch(p.status, 1u); sh_ok = 0u; break; }
+        }
+    }
+    // fault sites landing in this CTA's chunk (rare; campaign runs only)
+    if (p.sites != nullptr) {
+        for (int i = tid; i < p.n_sites; i += kARThreads) {
+            const ft2_fault_site s = p.sites[i];
+            if ((int)s.step != p.cur_step || (int)s.layer != p.cur_layer) continue;
+            const int64_t row = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
+                                (p.cur_step == 0 ? (int64_t)s.token : 0);
+            if (row < 0 || row >= p.rows || (int64_t)s.col >= p.n) continue;
+            const uint64_t el = (uint64_t)row * (uint64_t)p.n + s.col;
+            const uint64_t vv = el >> 3;
+            if (vv < v0 || vv >= v1) continue;
+            const uint32_t k = atomicAdd(&sh_ns, 1u);
+            if (k < (uint32_t)kARSites) { sh_site_e[k] = (uint32_t)(el - (uint64_t)v0 * 8u); sh_site_m[k] = s.xor_mask; }
+        }
+    }
+    __syncthreads();
+    if (sh_ok) {
+        const uint32_t nsite = min(sh_ns, (uint32_t)kARSites);
+        for (uint32_t v = v0 + tid; v < v1; v += kARThreads) {
+            const uint32_t row = fdiv(v, div_n8), c8 = v - row * n8;
+            float acc[8];
+            for (int t = 0; t < p.P; ++t)
+                add8<DT>(acc, ld_relaxed_sys_v4(p.partials[t] + (int64_t)row * p.ldp + c8 * 8), t == 0);
+            if (p.bias) {
+                const uint4 b = *reinterpret_cast<const uint4*>(p.bias + c8 * 8);
+                const uint32_t bw[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+                for (int j = 0; j < 8; ++j)
+                    acc[j] = __fadd_rn(acc[j], to_f32<DT>((uint16_t)(bw[j >> 1] >> ((j & 1) * 16))));
+            }
+            uint32_t w[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                w[j] = (uint32_t)rne16<DT>(acc[2 * j]) | ((uint32_t)rne16<DT>(acc[2 * j + 1]) << 16);
+            for (uint32_t i = 0; i < nsite; ++i) {
+                const uint32_t d = sh_site_e[i] - (v - v0) * 8u;
+                if (d < 8u) w[d >> 1] ^= (sh_site_m[i] & 0xFFFFu) << ((d & 1) * 16);
+            }
+            if (p.mode == FT2_GEMM_CHECK) {
+                const int s = row_mode == 2 ? 0 : (row_mode == 1 ? (int)row : p.row_to_seq[row]);
+                if (s >= 0 && s < p.S) {
+                    const uint32_t k = key2(*reinterpret_cast<const uint32_t*>(p.bounds + 2 * s));
+                    const uint32_t kL2 = (k & 0xFFFFu) * 0x10001u, kH2 = (k >> 16) * 0x10001u;
+                    uint32_t cnt = 0, c;
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) { w[j] = clip2<DT>(w[j], kL2, kH2, &c); cnt += c; }
+                    if (cnt && p.counts) atomicAdd(&p.counts[s], cnt);
+                }
+            }
+            *reinterpret_cast<uint4*>(p.y + (int64_t)row * p.ldy + c8 * 8) = make_uint4(w[0], w[1], w[2], w[3]);
+        }
+    }
+    // ---- 4. last CTA: this rank's call is complete; advance the epoch
+    __syncthreads();
+    if (tid == 0) sh_last = atom_add_acq_rel_gpu(p.done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (sh_last && tid == 0) {
+        *p.done = 0u;
+        *reinterpret_cast<volatile uint32_t*>(p.epoch) = e;
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_allreduce_protect(const AllreduceProtectArgs& a, cudaStream_t st, int* n_launch) {
+    const uint32_t n8 = (uint32_t)(a.n / 8), total = (uint32_t)(a.rows * (a.n / 8));
+    // one vector per thread per pass; at most 2 CTAs per SM (every CTA polls)
+    uint32_t grid = (total + kARThreads - 1) / kARThreads;
+    const uint32_t cap = (uint32_t)(2 * num_sms());
+    grid = grid < 1 ? 1 : (grid > cap ? cap : grid);
+    uint32_t chunk = (total + grid - 1) / grid;
+    grid = (total + chunk - 1) / chunk;
+    const int row_mode = a.row_to_seq ? 0 : (a.S == 1 ? 2 : 1);
+    if (a.dtype == FT2_FP16)
+        allreduce_protect_kernel<1><<<grid, kARThreads, 0, st>>>(a, chunk, n8, total, make_fastdiv(n8), row_mode);
+    else
+        allreduce_protect_kernel<0><<<grid, kARThreads, 0, st>>>(a, chunk, n8, total, make_fastdiv(n8), row_mode);
+    ++*n_launch;
+    return cudaGetLastError();
+}
+
+}  // namespace ft2impl

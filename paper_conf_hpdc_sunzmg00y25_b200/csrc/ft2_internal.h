@@ -100,6 +100,30 @@ cudaError_t launch_inject32(void* y, int64_t rows, int64_t n, int64_t ld, const 
                             int32_t n_sites, int32_t layer, int32_t step, const int32_t* base_row,
                             cudaStream_t st, int* n_launch);
 
+// Row-parallel sum all-reduce fused with the check (allreduce_protect.cu).
+struct AllreduceProtectArgs {
+    const uint16_t* const* partials;  // device array [P] of (peer-mapped) partial outputs
+    int64_t ldp;
+    int32_t P, rank;
+    uint32_t* const* flags;           // device array [P]: rank t's flag array [P]
+    uint32_t* epoch;                  // this rank's call counter (device)
+    uint32_t* done;                   // this rank's CTA completion counter (device, self-cleaning)
+    uint32_t* status;                 // this rank's error word (1 = peer timeout)
+    uint16_t* y;
+    int64_t ldy, rows, n;
+    const uint16_t* bias;
+    int32_t mode;
+    const int32_t* row_to_seq;
+    const uint16_t* bounds;
+    int32_t S;
+    uint32_t* counts;
+    const ft2_fault_site* sites;
+    int32_t n_sites, cur_layer, cur_step;
+    const int32_t* base_row;
+    int32_t dtype;
+};
+cudaError_t launch_allreduce_protect(const AllreduceProtectArgs& a, cudaStream_t st, int* n_launch);
+
 int num_sms();
 
 }  // namespace ft2impl

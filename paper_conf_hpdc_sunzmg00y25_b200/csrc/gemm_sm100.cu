@@ -580,9 +580,16 @@ struct GemmPlan {
     int swap, bn, tilesA, tilesB, splitk, nkb, deep;
 };
 
+// Largest token count that runs swap-AB on this kernel (BN = 128 token tiles
+// above 64); larger M goes to the persistent prefill kernel.
+static int swap_max_m() {
+    static const int v = [] { const char* e = getenv("FT2_GEMM_SWAP_MAX"); return e ? atoi(e) : 128; }();
+    return v;
+}
+
 static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     GemmPlan g;
-    g.swap = M <= 128 ? 1 : 0;
+    g.swap = M <= swap_max_m() ? 1 : 0;
     g.bn = g.swap ? (M <= 16 ? 16 : (M <= 32 ? 32 : (M <= 64 ? 64 : 128))) : 128;
     const int rowsA = g.swap ? N : M, rowsB = g.swap ? M : N;
     g.tilesA = (rowsA + kBlockA - 1) / kBlockA;
@@ -699,7 +706,7 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     // prefill shapes (M > 128 tokens): the persistent 128x256 kernel (gemm_prefill_sm100.cu)
-    if (a.M > 128) return launch_prefill_gemm(a, nullptr, st, n_launch);
+    if (a.M > swap_max_m()) return launch_prefill_gemm(a, nullptr, st, n_launch);
     const GemmPlan g = plan_gemm(a.M, a.N, a.K);
     GemmK p = {};
     p.M = a.M;

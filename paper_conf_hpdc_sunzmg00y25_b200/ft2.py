@@ -169,3 +169,40 @@ def launch_count() -> int:
 
 def version() -> str:
     return load().ft2_version().decode()
+
+
+def allreduce_protect(partial_ptrs, ldp, P, rank, flag_ptrs, words, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None,
+                      row_to_seq=None, num_seqs=None, corrected_count=None, sites=None, n_sites=None, cur_layer=0,
+                      cur_step=0, base_row=None, stream=None):
+    """ft2_allreduce_protect.  partial_ptrs / flag_ptrs: device int64 [P]
+    tensors of (peer-mapped) pointers; words: device int32 [3] (epoch, done,
+    status) of this rank; y: this rank's output."""
+    t = _as_ft2_tensor(y)
+    S = num_seqs if num_seqs is not None else (bounds.numel() // 2 if bounds is not None else 0)
+    ns = 0 if sites is None else (n_sites if n_sites is not None else sites.numel() // SITE_BYTES)
+    wp = words.data_ptr()
+    st = load().ft2_allreduce_protect(_ptr(partial_ptrs), int(ldp), int(P), int(rank), _ptr(flag_ptrs),
+                                      ctypes.c_void_p(wp), ctypes.c_void_p(wp + 4), ctypes.c_void_p(wp + 8), t,
+                                      _ptr(bias), int(mode), _ptr(row_to_seq), _ptr(bounds), S,
+                                      _ptr(corrected_count), _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),
+                                      _stream(stream))
+    check("ft2_allreduce_protect", st)
+
+
+def ipc_get_handle(t: torch.Tensor):
+    """(64-byte handle, byte offset) of the allocation holding t (CUDA IPC)."""
+    h = ctypes.create_string_buffer(64)
+    off = ctypes.c_uint64(0)
+    check("ft2_ipc_get_handle", load().ft2_ipc_get_handle(ctypes.c_void_p(t.data_ptr()), h, ctypes.byref(off)))
+    return h.raw, int(off.value)
+
+
+def ipc_open_handle(handle: bytes) -> int:
+    """Map a peer allocation's handle; returns its base device address."""
+    p = ctypes.c_void_p(0)
+    check("ft2_ipc_open_handle", load().ft2_ipc_open_handle(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)))
+    return int(p.value)
+
+
+def ipc_close(base: int):
+    check("ft2_ipc_close", load().ft2_ipc_close(ctypes.c_void_p(base)))

@@ -27,7 +27,6 @@ replayed: one prefill replay and G-1 decode replays per request.
 from __future__ import annotations
 
 import dataclasses
-import math
 
 import torch
 import torch.nn.functional as F
@@ -38,6 +37,7 @@ from . import ft2 as F2
 from ._lib import FT2_GEMM_CHECK, FT2_GEMM_PLAIN, FT2_GEMM_W_STATIC
 
 MODES = ("off", "standalone", "fused", "fused_plain")
+FUSED_MAX_M = 128
 
 
 @dataclasses.dataclass(frozen=True)
@@ -204,8 +204,7 @@ class Runner:
     def _norm(self, x, w, b):
         if self.cfg.arch == "opt":
             return F.layer_norm(x, (x.shape[-1],), w, b, 1e-5)
-        xf = x.float()
-        return (xf * torch.rsqrt(xf.pow(2).mean(-1, keepdim=True) + 1e-6)).to(x.dtype) * w
+        return F.rms_norm(x, (x.shape[-1],), w, 1e-6)
 
     def _rope(self, x, pos_idx):
         cos = self.rope_cos[pos_idx].unsqueeze(1)
@@ -226,7 +225,7 @@ class Runner:
 
         phase "prefill": bounds from the first-token output (+ NaN/Inf correction).
         phase "decode":  check-and-clip according to self.mode.
-        With self.sites set (fault-injection campaign, eager mode only), the
+        With self.sites set (fault-injection campaign; eager or per-step graphs), the
         site of each trial row is applied to the layer's bf16 output before the
         check (order GEMM -> bias -> bf16 -> inject -> check, readings A19/A20).
         """
@@ -251,8 +250,21 @@ class Runner:
                 F2.bounds_from_prefill(y, st.bounds[cid], st.ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
                                        scale=self.scale, correct_nonfinite=True, nonfinite_count=st.nonfinite[cid])
             return y
-        # decode
-        if not crit or self.mode in ("off", "standalone"):
+        # decode.  The fused tcgen05 GEMM serves decode batches of up to
+        # FUSED_MAX_M tokens (swap-AB, cluster split-K); larger decode batches
+        # (the 256-trial campaign) would land on the persistent prefill kernel,
+        # which has no split-K and starves the grid at M = 256 (measured 1.4-2.5x
+        # slower than cuBLAS, profiles/r1_m256_probe.txt), so there "fused" runs
+        # cuBLAS + ft2_protect and "fused_plain" plain cuBLAS.
+        fused_ok = x2.shape[0] <= FUSED_MAX_M
+        if not crit or self.mode in ("off", "standalone") or not fused_ok:
+            if crit and not fused_ok and self.mode == "fused":
+                y = F.linear(x2, w, b)
+                if sites is not None:
+                    F2.inject_faults(y, sites, lid, step, n_sites=self.B)
+                cid = self._crit_id(blk.idx, name)
+                F2.protect(y, self.state.bounds[cid], num_seqs=self.B, corrected_count=self.state.corrected[cid])
+                return y
             y = F.linear(x2, w, b)
             if sites is not None:
                 F2.inject_faults(y, sites, lid, step, n_sites=self.B)
@@ -295,9 +307,8 @@ class Runner:
         else:
             kc.index_copy_(2, self.pos, k)
             vc.index_copy_(2, self.pos, v)
-            s = torch.matmul(q, kc.transpose(2, 3)) * (1.0 / math.sqrt(D))
-            s = s + self._mask
-            a = torch.matmul(torch.softmax(s.float(), -1).to(q.dtype), vc)
+            # one fused attention kernel over the whole (masked) cache
+            a = F.scaled_dot_product_attention(q, kc, vc, attn_mask=self._mask)
         a = a.transpose(1, 2).reshape(-1, cfg.hidden)
         o_name = "out_proj" if cfg.arch == "opt" else "o_proj"
         x = x + self._linear(a, blk, o_name, phase, step).view(B, T, -1)

@@ -65,3 +65,62 @@ def column_shard(n: int, world: int, rank: int):
     per = (n + world - 1) // world
     b = min(n, rank * per)
     return b, min(n, b + per)
+
+
+class RowParallelCheck:
+    """A row-parallel critical layer's sum all-reduce fused with FT2's check
+    (ft2_allreduce_protect, reading A17).
+
+    Owns this rank's double-buffered partial outputs [2, rows, n], its flag
+    array [P] and its (epoch, done, status) words; exchanges CUDA IPC handles
+    once over `group` (any backend: the handles are host bytes) and maps every
+    peer's buffers.  Call i writes its GEMM partial into partial(i) and then
+    calls __call__(i, ...); consecutive calls must alternate i's parity."""
+
+    def __init__(self, rows: int, n: int, dtype=torch.bfloat16, group=None, device=None):
+        from . import ft2 as F2
+        self.F2 = F2
+        self.P = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.rows, self.n = rows, n
+        self.partials = torch.zeros((2, rows, n), dtype=dtype, device=dev)
+        self.flags = torch.zeros(self.P, dtype=torch.int32, device=dev)
+        self.words = torch.zeros(3, dtype=torch.int32, device=dev)
+        mine = (F2.ipc_get_handle(self.partials), F2.ipc_get_handle(self.flags))
+        allh = [None] * self.P
+        dist.all_gather_object(allh, mine, group=group)
+        self._opened = []
+        pptr, fptr = [], []
+        elt = self.partials.element_size()
+        for t, ((hp, op), (hf, of)) in enumerate(allh):
+            if t == self.rank:
+                bp, bf = self.partials.data_ptr(), self.flags.data_ptr()
+            else:
+                basep = F2.ipc_open_handle(hp)
+                basef = F2.ipc_open_handle(hf) if hf != hp else basep
+                self._opened += [basep] + ([basef] if basef != basep else [])
+                bp, bf = basep + op, basef + of
+            pptr.append((bp, bp + rows * n * elt))
+            fptr.append(bf)
+        self.partial_ptrs = [torch.tensor([p[b] for p in pptr], dtype=torch.int64, device=dev) for b in (0, 1)]
+        self.flag_ptrs = torch.tensor(fptr, dtype=torch.int64, device=dev)
+        dist.barrier(group=group)   # every rank mapped everything before any call
+
+    def partial(self, i: int) -> torch.Tensor:
+        return self.partials[i & 1]
+
+    def __call__(self, i: int, y: torch.Tensor, bias=None, mode=1, bounds=None, row_to_seq=None, num_seqs=None,
+                 corrected_count=None, sites=None, n_sites=None, cur_layer=0, cur_step=0, base_row=None):
+        self.F2.allreduce_protect(self.partial_ptrs[i & 1], self.n, self.P, self.rank, self.flag_ptrs, self.words, y,
+                                  bias=bias, mode=mode, bounds=bounds, row_to_seq=row_to_seq, num_seqs=num_seqs,
+                                  corrected_count=corrected_count, sites=sites, n_sites=n_sites,
+                                  cur_layer=cur_layer, cur_step=cur_step, base_row=base_row)
+
+    def status(self) -> int:
+        return int(self.words[2].item())
+
+    def close(self):
+        for b in self._opened:
+            self.F2.ipc_close(b)
+        self._opened = []

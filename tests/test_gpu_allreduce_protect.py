@@ -1,0 +1,133 @@
+"""ft2_allreduce_protect: a row-parallel critical
+layer's one-shot sum all-reduce over CUDA IPC peer memory fused with the check,
+bit-exact against the oracle (reading A22 + R7 + R5), identical on every rank.
+World size 2 runs as two processes sharing the one GPU (IPC mappings of the
+same device; gloo exchanges the handles); P = 1 runs in-process."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import ft2_synth
+import oracle
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROWS, N, CALLS = 32, 5120, 5
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _inputs(i, world):
+    parts = np.stack([ft2_synth.gen_bf16((ROWS, N), 300 + 16 * i + t, 9) for t in range(world)])
+    bias = ft2_synth.gen_bf16((N,), 299, 9)
+    rng = np.random.default_rng(i)
+    bounds = np.stack([[oracle.f64_to_bf16(-abs(rng.normal(1.0, 0.3)) - 0.1),
+                        oracle.f64_to_bf16(abs(rng.normal(1.0, 0.3)) + 0.1)] for _ in range(ROWS)]).astype(np.uint16)
+    sites = oracle.make_sites(11, 64 * i, ROWS, oracle.FAULT_EXP, [N], n_steps=1, prompt_len=1, step_policy=1)
+    return parts, bias, bounds, sites
+
+
+def _worker(rank, world, port, q):
+    import sys
+    sys.path[:0] = [ROOT, os.path.join(ROOT, "tests")]
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    from gpu_util import dev, host, sites_to_dev
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+    rpc = tp.RowParallelCheck(ROWS, N)
+    out = []
+    for i in range(CALLS):
+        parts, bias, bounds, sites = _inputs(i, world)
+        rpc.partial(i).copy_(dev(parts[rank]))
+        y = torch.empty((ROWS, N), dtype=torch.bfloat16, device="cuda")
+        cnt = torch.zeros(ROWS, dtype=torch.int32, device="cuda")
+        torch.cuda.synchronize()
+        rpc(i, y, bias=dev(bias), mode=1, bounds=dev(bounds), num_seqs=ROWS, corrected_count=cnt,
+            sites=sites_to_dev(sites), n_sites=ROWS, cur_layer=0, cur_step=1)
+        torch.cuda.synchronize()
+        out.append((host(y).tobytes(), cnt.cpu().numpy().tolist()))
+    q.put((rank, out, rpc.status()))
+    dist.barrier()
+    rpc.close()
+    dist.destroy_process_group()
+
+
+def _check(results, world):
+    for i in range(CALLS):
+        parts, bias, bounds, sites = _inputs(i, world)
+        want, wcnt = oracle.allreduce_protect(parts, bias=bias, bounds_=bounds, sites=sites, cur_layer=0, cur_step=1)
+        for rank, out, status in results:
+            assert status == 0
+            y = np.frombuffer(out[i][0], np.uint16).reshape(ROWS, N)
+            assert np.array_equal(y, want), (rank, i)
+            assert np.array_equal(np.array(out[i][1], np.uint32), wcnt), (rank, i)
+        assert int(wcnt.sum()) > 0   # the EXP faults were corrected
+
+
+def test_allreduce_protect_world2_ipc():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(2)]
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    _check(res, 2)
+
+
+def test_allreduce_protect_p1_in_process():
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+    port = _port()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        from gpu_util import dev, host, sites_to_dev
+        rpc = tp.RowParallelCheck(ROWS, N)
+        out = []
+        for i in range(CALLS):
+            parts, bias, bounds, sites = _inputs(i, 1)
+            rpc.partial(i).copy_(dev(parts[0]))
+            y = torch.empty((ROWS, N), dtype=torch.bfloat16, device="cuda")
+            cnt = torch.zeros(ROWS, dtype=torch.int32, device="cuda")
+            rpc(i, y, bias=dev(bias), mode=1, bounds=dev(bounds), num_seqs=ROWS, corrected_count=cnt,
+                sites=sites_to_dev(sites), n_sites=ROWS, cur_layer=0, cur_step=1)
+            torch.cuda.synchronize()
+            out.append((host(y).tobytes(), cnt.cpu().numpy().tolist()))
+        _check([(0, out, rpc.status())], 1)
+        # CUDA-graph replay: the epoch lives in device memory
+        g = torch.cuda.CUDAGraph()
+        parts, bias, bounds, sites = _inputs(0, 1)
+        rpc.partial(0).copy_(dev(parts[0]))
+        rpc.partial(1).copy_(dev(parts[0]))
+        y = torch.empty((ROWS, N), dtype=torch.bfloat16, device="cuda")
+        cnt = torch.zeros(ROWS, dtype=torch.int32, device="cuda")
+        bd, bs = dev(bounds), dev(bias)
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            with torch.cuda.graph(g):
+                rpc(0, y, bias=bs, mode=1, bounds=bd, num_seqs=ROWS, corrected_count=cnt)
+                rpc(1, y, bias=bs, mode=1, bounds=bd, num_seqs=ROWS, corrected_count=cnt)
+        for _ in range(3):
+            g.replay()
+        torch.cuda.synchronize()
+        want, wcnt = oracle.allreduce_protect(parts[:1], bias=bias, bounds_=bounds)
+        assert np.array_equal(host(y), want) and rpc.status() == 0
+        assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), 6 * wcnt)
+        assert int(rpc.words[0].item()) == CALLS + 6     # epoch advanced once per call
+    finally:
+        dist.destroy_process_group()
