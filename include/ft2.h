@@ -208,12 +208,15 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
  * sites/n_sites/cur_layer/cur_step/base_row  optional fault injection applied
  *              to the bf16 result before the check (order: GEMM -> bias -> bf16 ->
  *              inject -> check; readings A19, A20), as in ft2_inject_faults.
- * workspace/ws_bytes  at least ft2_gemm_workspace_bytes(M, N, K) bytes, 16-byte
- *              aligned (may be NULL when that is 0): split-K partial tiles and
- *              per-tile arrival counters.  Zero-filled once before first use; every
- *              call leaves the counters zero again.  The split-K partial sums are
- *              combined in a fixed order, so results are deterministic.  At most
- *              16 MiB for any shape on a 148-SM B200.
+ * workspace/ws_bytes  optional, 16-byte aligned, zero-filled once before first
+ *              use (every call leaves its counters zero again).  Decode shapes
+ *              (M <= 128) split K across a thread-block cluster and need none.
+ *              The persistent M > 128 kernel splits K through it when its tiles
+ *              cannot fill the GPU (small M): ft2_gemm_workspace_bytes(M, N, K)
+ *              bytes give the best split, fewer bytes fewer splits, NULL none.
+ *              Split partials are summed in split order: results do not depend
+ *              on the workspace (only the timing does) -- except that a
+ *              different split count changes the fp32 summation order.
  * The kernel is launched with programmatic stream serialization (PDL): its
  * prologue and first weight tiles overlap the previous kernel's tail; it reads
  * x, bias, bounds, sites and writes y, counters, workspace only after the
@@ -249,6 +252,8 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
  * padding, reading A18) or NULL for one sequence; scale, correct_nonfinite,
  * bounds_out, keys_out, nonfinite_count, workspace: as ft2_bounds_from_prefill
  * (workspace = ft2_workspace_bytes(num_seqs) bytes, zero-filled once, left zero).
+ * gemm_workspace/gemm_ws_bytes: the optional K-split workspace of
+ *              ft2_protect_fused_gemm (ft2_gemm_workspace_bytes(M, N, K)).
  * sites/n_sites/cur_layer/base_row: faults of step 0 (base_row = seq_offsets).
  * The GEMM is a persistent 128x256-tile tcgen05 kernel (one CTA per SM, TMEM
  * double-buffered accumulators); it is also what ft2_protect_fused_gemm runs
@@ -261,7 +266,8 @@ ft2_status ft2_prefill_fused_gemm(const void* x, int64_t ldx, const void* w, int
                                   int32_t num_seqs, float scale, int32_t correct_nonfinite,
                                   void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
                                   const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
-                                  const int32_t* base_row, void* workspace, void* stream);
+                                  const int32_t* base_row, void* workspace, void* gemm_workspace,
+                                  size_t gemm_ws_bytes, void* stream);
 
 /* Seeded fault sites for trials [trial0, trial0 + n_trials) (reading R6:
  * Philox4x32-10 keyed by seed, counter = trial id; uniform step, layer, neuron

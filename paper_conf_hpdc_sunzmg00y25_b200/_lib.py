@@ -67,7 +67,7 @@ def load(path: str = LIB):
         "ft2_protect_fused_gemm": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, ctypes.c_int, i32, i32,
                                         P, P, i32, P, P, i32, i32, i32, P, P, ctypes.c_size_t, P]),
         "ft2_prefill_fused_gemm": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, P, i32, f32, i32,
-                                        P, P, P, P, i32, i32, P, P, P]),
+                                        P, P, P, P, i32, i32, P, P, P, ctypes.c_size_t, P]),
         "ft2_make_fault_sites": (st, [u64, u64, i32, ctypes.c_int, ctypes.c_int, ctypes.POINTER(SiteGeometry),
                                       P, P]),
         "ft2_inject_faults": (st, [Tensor, P, i32, i32, i32, P, P]),

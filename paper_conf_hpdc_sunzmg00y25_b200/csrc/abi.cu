@@ -173,9 +173,10 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
         if (col_begin < 0 || col_end > N || col_begin > col_end) return FT2_ERR_INVALID_ARG;
     }
     if (n_sites < 0 || (n_sites > 0 && sites == nullptr)) return FT2_ERR_INVALID_ARG;
-    const size_t need = gemm_ws_bytes(M, N, K);
-    if (need > 0 && (workspace == nullptr || ws_bytes < need)) return FT2_ERR_INVALID_ARG;
-    if (need > 0 && !al16(workspace)) return FT2_ERR_MISALIGNED;
+    // the workspace is optional (K splits of the persistent M > 128 kernel): a
+    // smaller one or none means fewer or no splits
+    if (workspace != nullptr && !al16(workspace)) return FT2_ERR_MISALIGNED;
+    if (workspace == nullptr) ws_bytes = 0;
     GemmArgs a;
     a.x = static_cast<const uint16_t*>(x);
     a.ldx = ldx;
@@ -213,8 +214,10 @@ ft2_status ft2_prefill_fused_gemm(const void* x, int64_t ldx, const void* w, int
                                   const int32_t* seq_offsets, int32_t num_seqs, float scale, int32_t correct_nonfinite,
                                   void* bounds_out, int32_t* keys_out, uint32_t* nonfinite_count,
                                   const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
-                                  const int32_t* base_row, void* workspace, void* stream) {
+                                  const int32_t* base_row, void* workspace, void* gemm_workspace,
+                                  size_t gemm_ws_bytes, void* stream) {
     if (M < 0 || N < 0 || K < 0) return FT2_ERR_INVALID_ARG;
+    if (gemm_workspace != nullptr && !al16(gemm_workspace)) return FT2_ERR_MISALIGNED;
     if (dtype != FT2_BF16 && dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
     if (num_seqs < 1 || num_seqs > FT2_MAX_SEQS) return num_seqs < 1 ? FT2_ERR_INVALID_ARG : FT2_ERR_UNSUPPORTED;
     if (!(std::isfinite(scale)) || scale < 1.0f) return FT2_ERR_INVALID_ARG;
@@ -249,6 +252,8 @@ ft2_status ft2_prefill_fused_gemm(const void* x, int64_t ldx, const void* w, int
     a.cur_step = 0;  // the first token (prefill) is step 0 of the fault-site geometry
     a.base_row = base_row;
     a.dtype = dtype;
+    a.ws = gemm_workspace;
+    a.ws_bytes = gemm_workspace ? gemm_ws_bytes : 0;
     PrefillDerive d;
     d.seq_offsets = seq_offsets;
     d.S = num_seqs;

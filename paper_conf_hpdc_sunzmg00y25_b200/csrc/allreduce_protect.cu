@@ -47,11 +47,11 @@ __device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
     asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
-// peer data written during this kernel's lifetime: strong (sys-scope) loads,
-// never the non-coherent path
-__device__ __forceinline__ uint4 ld_relaxed_sys_v4(const void* p) {
+// peer data written during this kernel's lifetime, read after the acquire
+// handshake: L2-level loads (never L1, never the non-coherent path)
+__device__ __forceinline__ uint4 ld_peer_v4(const void* p) {
     uint4 r;
-    asm volatile("ld.relaxed.sys.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
     return r;
 }
@@ -81,13 +81,14 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     }
     __syncthreads();
     const uint32_t e = sh_e;
-    // ---- 1. signal: my partial (written by the preceding kernel) is ready
-    if (blockIdx.x == 0 && tid < p.P) {
+    // ---- 1. signal: my partial (written by the preceding kernel) is ready.
+    // P = 1 needs no handshake: stream order already covers my own partial.
+    if (p.P > 1 && blockIdx.x == 0 && tid < p.P) {
         __threadfence_system();
         st_release_sys(p.flags[tid] + p.rank, e);
     }
     // ---- 2. wait for every rank's partial of this call
-    if (tid < p.P) {
+    if (p.P > 1 && tid < p.P) {
         const uint32_t* f = p.flags[p.rank] + tid;
         uint32_t polls = 0;
         while ((int32_t)(ld_acquire_sys(f) - e) < 0) {
@@ -116,7 +117,7 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
             const uint32_t row = fdiv(v, div_n8), c8 = v - row * n8;
             float acc[8];
             for (int t = 0; t < p.P; ++t)
-                add8<DT>(acc, ld_relaxed_sys_v4(p.partials[t] + (int64_t)row * p.ldp + c8 * 8), t == 0);
+                add8<DT>(acc, ld_peer_v4(p.partials[t] + (int64_t)row * p.ldp + c8 * 8), t == 0);
             if (p.bias) {
                 const uint4 b = *reinterpret_cast<const uint4*>(p.bias + c8 * 8);
                 const uint32_t bw[4] = {b.x, b.y, b.z, b.w};

@@ -87,6 +87,13 @@ struct PrefillDerive {
     uint32_t* nonfinite_out;
     uint32_t* ws;  // bounds workspace (bounds_ws_bytes(S))
 };
+// K-split plan of the persistent kernel (gemm_prefill_sm100.cu): splits that
+// fit ws_bytes, the counter-area bytes, and the bytes the best plan needs.
+struct PrefillSplit {
+    int splits;
+    size_t cnt_bytes, need_bytes;
+};
+PrefillSplit plan_prefill_split(int32_t M, int32_t N, int32_t K, size_t ws_bytes);
 // Persistent 128x256-tile tcgen05 GEMM for M > 128 (PLAIN / CHECK, or DERIVE when d != NULL)
 cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaStream_t st, int* n_launch);
 

@@ -65,9 +65,16 @@ constexpr int kPMaxRowSites = 4;                     // fault sites one row may 
 constexpr int kPMiscBytes = 256;
 constexpr int kPSmemBytes = 1024 + kPTileBytes + kPMiscBytes + 3 * kPSeqTab * 4;
 constexpr int kPGemmDerive = 2;
+constexpr int kSplitCounters = 16384;   // split-K arrival counters at the head of the GEMM workspace
 
 struct PrefK {
     int32_t M, N, K, tilesM, ntiles, nkb;
+    // split-K for grids the tiles alone cannot fill (small M): `splits` units
+    // per tile, fp32 partial slots [half-tile][split][128][256] in skws, one
+    // arrival counter per 128 x 256 half-tile in skcnt (self-cleaning)
+    int32_t splits;
+    float* skws;
+    uint32_t* skcnt;
     int32_t mode, col_begin, col_end;
     const uint16_t* bias;
     uint16_t* y;
@@ -97,18 +104,24 @@ __device__ __forceinline__ uint32_t pack_rne2(float a, float b, int dt) {
 // its own 128 output rows x 256 columns -- the weight box is read from L2 and
 // staged in shared memory once per pair.
 template <int MC>
-__device__ __forceinline__ bool tile_of(const PrefK& p, int i, int& m0, int& n0) {
+__device__ __forceinline__ bool tile_of(const PrefK& p, int i, int& m0, int& n0, int& ks) {
+    // work units (tile, K split), split-major: a tile's splits land on
+    // different CTAs (clusters) of the same wave
     if (MC == 1) {
-        const int t = blockIdx.x + i * gridDim.x;
-        if (t >= p.ntiles) return false;
+        const int u = blockIdx.x + i * gridDim.x;
+        if (u >= p.ntiles * p.splits) return false;
+        const int t = u % p.ntiles;
+        ks = u / p.ntiles;
         m0 = (t % p.tilesM) * kPBM;
         n0 = (t / p.tilesM) * kPBN;
         return true;
     }
     const int pairsM = (p.tilesM + 1) >> 1;
     const int npairs = pairsM * (p.ntiles / p.tilesM);
-    const int pr = (int)(blockIdx.x >> 1) + i * (int)(gridDim.x >> 1);
-    if (pr >= npairs) return false;
+    const int u = (int)(blockIdx.x >> 1) + i * (int)(gridDim.x >> 1);
+    if (u >= npairs * p.splits) return false;
+    const int pr = u % npairs;
+    ks = u / npairs;
     m0 = ((pr % pairsM) * 2 + (int)(blockIdx.x & 1)) * kPBM;
     n0 = (pr / pairsM) * kPBN;
     return true;
@@ -129,6 +142,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     uint64_t* tmem_empty = tmem_full + 2;    // [2]
     uint32_t* tmem_base_sh = reinterpret_cast<uint32_t*>(tmem_empty + 2);
     uint32_t* last_sh = tmem_base_sh + 1;
+    uint32_t* skl_sh = tmem_base_sh + 2;  // "this unit finishes its half-tile" (split-K)
     uint32_t* tab_lo = reinterpret_cast<uint32_t*>(misc + kPMiscBytes);  // 0x10000 - min key (0: none)
     uint32_t* tab_hi = tab_lo + kPSeqTab;                                 // max key + 1 (0: none)
     uint32_t* tab_nf = tab_hi + kPSeqTab;                                 // non-finite count
@@ -168,9 +182,10 @@ __global__ void __launch_bounds__(kPThreads, 1)
             // ---------------------------------------------------- TMA producer
             griddep_wait();  // x may be the previous kernel's output
             uint32_t stage = 0, phase = 0;
-            int m0, n0;
-            for (int i = 0; tile_of<MC>(p, i, m0, n0); ++i) {
-                for (int kb = 0; kb < p.nkb; ++kb) {
+            int m0, n0, ks;
+            for (int i = 0; tile_of<MC>(p, i, m0, n0, ks); ++i) {
+                const int kb0 = (int)((int64_t)ks * p.nkb / p.splits), kb1 = (int)((int64_t)(ks + 1) * p.nkb / p.splits);
+                for (int kb = kb0; kb < kb1; ++kb) {
                     mbar_wait(&empty[stage], phase ^ 1u);
                     uint8_t* st = tiles + stage * kPStageBytes;
                     if (MC == 1) {
@@ -199,13 +214,14 @@ __global__ void __launch_bounds__(kPThreads, 1)
             constexpr uint32_t idesc =
                 (make_idesc(kPBM * MC, kPBN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
             uint32_t stage = 0, phase = 0;
-            int tc = 0, m0, n0;
-            for (int i = 0; tile_of<MC>(p, i, m0, n0); ++i, ++tc) {
+            int tc = 0, m0, n0, ks;
+            for (int i = 0; tile_of<MC>(p, i, m0, n0, ks); ++i, ++tc) {
                 const int buf = tc & 1;
                 mbar_wait(&tmem_empty[buf], ((uint32_t)(tc >> 1) & 1u) ^ 1u);  // the epilogue drained it
                 tc_fence_after();
                 const uint32_t d = tmem_base + (uint32_t)(buf * kPBN);
-                for (int kb = 0; kb < p.nkb; ++kb) {
+                const int kb0 = (int)((int64_t)ks * p.nkb / p.splits), kb1 = (int)((int64_t)(ks + 1) * p.nkb / p.splits);
+                for (int kb = kb0; kb < kb1; ++kb) {
                     mbar_wait(&full[stage], phase);
                     tc_fence_after();
                     const uint32_t sa = smem_u32(tiles + stage * kPStageBytes);
@@ -213,9 +229,9 @@ __global__ void __launch_bounds__(kPThreads, 1)
 #pragma unroll
                     for (int k = 0; k < kPBK / 16; ++k) {
                         if (MC == 1)
-                            tc_mma(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                            tc_mma(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > kb0 || k > 0) ? 1u : 0u);
                         else
-                            tc_mma2(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                            tc_mma2(d, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (kb > kb0 || k > 0) ? 1u : 0u);
                     }
                     if (MC == 1) tc_commit(&empty[stage]);
                     else tc_commit2_mc(&empty[stage], (uint16_t)3u);  // both producers may refill it
@@ -235,8 +251,8 @@ __global__ void __launch_bounds__(kPThreads, 1)
         uint32_t* ws_ov = p.bp.ws + 4 * p.bp.S + 2;
         unsigned long long* list = reinterpret_cast<unsigned long long*>(
             reinterpret_cast<char*>(p.bp.ws) + (((size_t)(4 * p.bp.S + 4) * 4 + 7) & ~(size_t)7));
-        int tc = 0, m0, n0;
-        for (int i = 0; tile_of<MC>(p, i, m0, n0); ++i, ++tc) {
+        int tc = 0, m0, n0, ks;
+        for (int i = 0; tile_of<MC>(p, i, m0, n0, ks); ++i, ++tc) {
             const int buf = tc & 1;
             const int m = m0 + e;
             const bool row_ok = m < p.M;
@@ -279,11 +295,66 @@ __global__ void __launch_bounds__(kPThreads, 1)
             tc_fence_after();
             const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * kPBN);
             uint16_t* yrow = p.y + (int64_t)m * p.ldy;
+            const bool split = p.splits > 1;
+            // 128 x 256 half-tile id; pairs may cover one phantom m-tile past tilesM
+            const int half = m0 / kPBM + (MC == 2 ? ((p.tilesM + 1) & ~1) : p.tilesM) * (n0 / kPBN);
+            float* const slot0 = split ? p.skws + ((size_t)half * p.splits * kPBM + e) * kPBN : nullptr;
+            if (split) {
+                // K split: stage this unit's fp32 partial rows; the last of the
+                // tile's splits to arrive sums all slots in split order
+                // (deterministic) and runs the epilogue below
+                float* mine = slot0 + (size_t)ks * kPBM * kPBN;
+#pragma unroll 1
+                for (int c0 = h0; c0 < h0 + kPBN / 2; c0 += 32) {
+                    uint32_t r[32];
+                    tmem_ld32(taddr + (uint32_t)c0, r);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        __stcg(reinterpret_cast<float4*>(mine + c0) + j,
+                               make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                           __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3])));
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if (MC == 1) mbar_arrive(&tmem_empty[buf]);
+                    else mbar_arrive_cluster(mapa(smem_u32(&tmem_empty[buf]), 0u));
+                }
+                __threadfence();
+                named_bar(1, 32 * kPEpiWarps);
+                if (tid == 64) {
+                    const bool last = atom_add_acq_rel_gpu(p.skcnt + half, 1u) == (uint32_t)(p.splits - 1);
+                    if (last) p.skcnt[half] = 0u;   // every split arrived: reset for the next launch
+                    *skl_sh = last ? 1u : 0u;
+                }
+                named_bar(1, 32 * kPEpiWarps);
+                if (*skl_sh == 0u) continue;   // another split finishes this half-tile
+            }
 #pragma unroll 1
             for (int c0 = h0; c0 < h0 + kPBN / 2; c0 += 32) {
                 uint32_t r[32];
-                tmem_ld32(taddr + (uint32_t)c0, r);
-                tmem_wait_ld();
+                if (!split) {
+                    tmem_ld32(taddr + (uint32_t)c0, r);
+                    tmem_wait_ld();
+                } else {
+                    float acc[32];
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {
+                        const float4 v = __ldcg(reinterpret_cast<const float4*>(slot0 + c0) + j);
+                        acc[4 * j] = v.x; acc[4 * j + 1] = v.y; acc[4 * j + 2] = v.z; acc[4 * j + 3] = v.w;
+                    }
+                    for (int sk = 1; sk < p.splits; ++sk) {
+                        const float* sl = slot0 + (size_t)sk * kPBM * kPBN + c0;
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) {
+                            const float4 v = __ldcg(reinterpret_cast<const float4*>(sl) + j);
+                            acc[4 * j] += v.x; acc[4 * j + 1] += v.y; acc[4 * j + 2] += v.z; acc[4 * j + 3] += v.w;
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) r[j] = __float_as_uint(acc[j]);
+                }
                 const int nb = n0 + c0;
                 if (!row_ok || nb >= p.N) continue;
                 const int nvalid = min(32, p.N - nb);
@@ -356,11 +427,13 @@ __global__ void __launch_bounds__(kPThreads, 1)
                 }
             }
             // accumulator buffer drained: hand it back to the MMA warp (the leader's)
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) {
-                if (MC == 1) mbar_arrive(&tmem_empty[buf]);
-                else mbar_arrive_cluster(mapa(smem_u32(&tmem_empty[buf]), 0u));
+            if (!split) {
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if (MC == 1) mbar_arrive(&tmem_empty[buf]);
+                    else mbar_arrive_cluster(mapa(smem_u32(&tmem_empty[buf]), 0u));
+                }
             }
             if (p.mode == FT2_GEMM_CHECK && ncorr != 0u && p.counts != nullptr && seq >= 0)
                 atomicAdd(&p.counts[seq], ncorr);
@@ -493,6 +566,45 @@ static cudaError_t launch_prefill_dt(const CUtensorMap& mx, const CUtensorMap& m
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+// K-split plan for the persistent kernel: when the tiles cannot fill the
+// machine (small M: e.g. 512 prompt tokens at N = 4096 give 16 pair-tiles for
+// 74 SM pairs; a 256-trial decode batch gives 43 at N = 11008), split each
+// tile's K range into s units (>= 8 k-blocks each) and pick the s that
+// minimises the waves per unit of work, ceil(units * s / slots) / s, by at
+// least 10 %.  Partials go through an fp32 workspace (s slots per tile).
+PrefillSplit plan_prefill_split(int32_t M, int32_t N, int32_t K, size_t ws_bytes) {
+    PrefillSplit r{1, 0, 0};
+    const int tilesM = (M + kPBM - 1) / kPBM, tilesN = (N + kPBN - 1) / kPBN, nkb = (K + kPBK - 1) / kPBK;
+    const int units = tilesM >= 2 ? ((tilesM + 1) / 2) * tilesN : tilesM * tilesN;
+    const int slots = tilesM >= 2 ? num_sms() / 2 : num_sms();
+    const int tilesMp = tilesM >= 2 ? ((tilesM + 1) & ~1) : tilesM;  // + the pairs' phantom m-tile
+    // the arrival counters sit at a FIXED place (the first kSplitCounters
+    // words) whatever the shape, so one launch's partial slots never alias
+    // the next launch's counters
+    r.cnt_bytes = (size_t)kSplitCounters * 4;
+    if ((size_t)tilesMp * tilesN > (size_t)kSplitCounters) return r;
+    const size_t per_split = (size_t)tilesMp * kPBM * tilesN * kPBN * 4;
+    // Opt-in (FT2_PREFILL_SPLITS = s >= 2, or -1 for the planner below): the
+    // first implementation stages partials with one thread per row (16-byte
+    // stores spread over 32 rows per warp instruction) and measured SLOWER
+    // than the unsplit kernel at every small-M shape tried (M = 256, 4096^2:
+    // 29 -> 47 us; profiles/r1_prefill_splitk.txt), so it is off by default
+    // until the partial tiles move through shared memory / TMA bulk stores.
+    const char* ev = getenv("FT2_PREFILL_SPLITS");   // read per call: tests toggle it
+    const int env = ev ? atoi(ev) : 0;
+    if (env == 0 || env == 1) return r;
+    double best_t = (double)((units + slots - 1) / slots);
+    for (int s = 2; s <= 8; ++s) {
+        if (nkb < 8 * s) break;
+        if (env > 0 && s != env) continue;
+        const double t = (double)((units * s + slots - 1) / slots) / s;
+        if (t < 0.9 * best_t || (env > 0 && s == env)) { best_t = t; r.splits = s; }
+    }
+    r.need_bytes = r.splits > 1 ? r.cnt_bytes + (size_t)r.splits * per_split : 0;
+    while (r.splits > 1 && r.cnt_bytes + (size_t)r.splits * per_split > ws_bytes) --r.splits;
+    return r;
+}
+
 cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaStream_t st, int* n_launch) {
     CUtensorMap mx, mw;
     if (!make_map_p(&mx, a.x, a.M, a.K, a.ldx, kPBM, a.dtype)) return cudaErrorInvalidValue;
@@ -546,14 +658,14 @@ cudaError_t launch_prefill_gemm(const GemmArgs& a, const PrefillDerive* d, cudaS
     static const int mc_env = [] { const char* v = getenv("FT2_PREFILL_MC"); return v ? atoi(v) : 2; }();
     const int mc = (mc_env == 2 && p.tilesM >= 2) ? 2 : 1;  // CTA pairs (cta_group::2) unless one m-tile
     if (!make_map_p(&mw, a.w, a.N, a.K, a.ldw, mc == 2 ? kPBN / 2 : kPBN, a.dtype)) return cudaErrorInvalidValue;
-    int grid;
-    if (mc == 2) {
-        const int npairs = ((p.tilesM + 1) / 2) * (p.ntiles / p.tilesM);
-        const int maxpairs = num_sms() / 2;
-        grid = 2 * (npairs < maxpairs ? npairs : maxpairs);
-    } else {
-        grid = p.ntiles < num_sms() ? p.ntiles : num_sms();
-    }
+    const int units = mc == 2 ? ((p.tilesM + 1) / 2) * (p.ntiles / p.tilesM) : p.ntiles;
+    const int slots = mc == 2 ? num_sms() / 2 : num_sms();
+    const PrefillSplit sp = plan_prefill_split(p.M, p.N, p.K, a.ws_bytes);
+    p.splits = a.ws != nullptr ? sp.splits : 1;
+    p.skcnt = static_cast<uint32_t*>(a.ws);
+    p.skws = p.splits > 1 ? reinterpret_cast<float*>(static_cast<char*>(a.ws) + sp.cnt_bytes) : nullptr;
+    const int work = units * p.splits;
+    int grid = mc * (work < slots ? work : slots);
     cudaError_t e;
     if (mc == 2) e = a.dtype == FT2_FP16 ? launch_prefill_dt<1, 2>(mx, mw, p, grid, st)
                                          : launch_prefill_dt<0, 2>(mx, mw, p, grid, st);

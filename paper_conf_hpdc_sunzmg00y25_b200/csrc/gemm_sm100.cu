@@ -669,8 +669,13 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     return g;
 }
 
-// The cluster split-K needs no global workspace.
-size_t gemm_ws_bytes(int32_t, int32_t, int32_t) { return 0; }
+// The decode kernel's cluster split-K needs no global workspace; the
+// persistent kernel (M > swap_max_m()) uses one for its K splits when the
+// tiles alone cannot fill the machine (optional: less space, fewer splits).
+size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K) {
+    if (M <= swap_max_m()) return 0;
+    return plan_prefill_split(M, N, K, (size_t)-1).need_bytes;
+}
 
 template <int BN, bool SWAP, int DT, bool DEEP = false>
 static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st, int* n_launch) {

@@ -108,23 +108,24 @@ def protect_fused_gemm(x, w, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None, row
 
 def prefill_fused_gemm(x, w, y, bounds_out, workspace, bias=None, seq_offsets=None, num_seqs=None, scale=2.0,
                        correct_nonfinite=True, keys_out=None, nonfinite_count=None, sites=None, n_sites=None,
-                       cur_layer=0, base_row=None, stream=None):
+                       cur_layer=0, base_row=None, gemm_workspace=None, stream=None):
     """ft2_prefill_fused_gemm: y = inject(bf16(x @ w.T + bias)) and, in the same
     kernel's epilogue, ft2_bounds_from_prefill(y, ...) (finalize = 1)."""
     M, K = x.shape
     N = w.shape[0]
     S = num_seqs if num_seqs is not None else (1 if seq_offsets is None else seq_offsets.numel() - 1)
     ns = 0 if sites is None else (n_sites if n_sites is not None else sites.numel() // SITE_BYTES)
+    gw = gemm_workspace if gemm_workspace is not None else default_gemm_workspace(x.device)
     st = load().ft2_prefill_fused_gemm(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y), y.stride(0),
                                        M, N, K, _dtype_of(x), _ptr(seq_offsets), S, float(scale),
                                        int(correct_nonfinite), _ptr(bounds_out), _ptr(keys_out),
                                        _ptr(nonfinite_count), _ptr(sites), ns, cur_layer, _ptr(base_row),
-                                       _ptr(workspace), _stream(stream))
+                                       _ptr(workspace), _ptr(gw), gw.numel() * gw.element_size(), _stream(stream))
     check("ft2_prefill_fused_gemm", st)
 
 
 _GEMM_WS = {}
-GEMM_WS_BYTES = 16 << 20
+GEMM_WS_BYTES = 64 << 20   # K-split workspace of the M > 128 kernel (ft2_gemm_workspace_bytes)
 
 
 def default_gemm_workspace(device) -> torch.Tensor:

@@ -123,6 +123,22 @@ class Block:
         for j, (name, o, i, _) in enumerate(cfg.linears()):
             self.w[name] = _w((o, i), tau0 + 2 * j, seed, device, K=i)
             self.b[name] = _w((o,), tau0 + 2 * j + 1, seed, device) if cfg.bias else None
+        # horizontally fused projections (same weights; the per-layer tensors
+        # become views into the fused ones): qkv, and Llama's gate_up
+        self.groups = {"qkv": ["q_proj", "k_proj", "v_proj"]}
+        if cfg.arch == "llama":
+            self.groups["gate_up"] = ["gate_proj", "up_proj"]
+        self.wf, self.bf = {}, {}
+        for g, names in self.groups.items():
+            self.wf[g] = torch.cat([self.w[n] for n in names])
+            self.bf[g] = torch.cat([self.b[n] for n in names]) if cfg.bias else None
+            r0 = 0
+            for n in names:
+                o = self.w[n].shape[0]
+                self.w[n] = self.wf[g][r0:r0 + o]
+                if cfg.bias:
+                    self.b[n] = self.bf[g][r0:r0 + o]
+                r0 += o
         h = cfg.hidden
         self.ln1_w = torch.ones(h, dtype=torch.bfloat16, device=device)
         self.ln2_w = torch.ones(h, dtype=torch.bfloat16, device=device)
@@ -149,7 +165,7 @@ class Runner:
     """Batched greedy generation with FT2 on the critical layers."""
 
     def __init__(self, cfg: ModelConfig, batch: int, prompt_len: int, gen_len: int, seed: int = 1,
-                 device="cuda", scale: float = 2.0, coverage: str = "ft2"):
+                 device="cuda", scale: float = 2.0, coverage: str = "ft2", fuse_proj: bool = False):
         self.cfg = cfg
         self.B = batch
         self.T = prompt_len
@@ -166,6 +182,16 @@ class Runner:
         self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
         self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h)
         self.coverage = coverage
+        # fuse_proj: fused q/k/v (and Llama gate/up) projections, one GEMM per
+        # group; the protected layer of a group (v_proj, up_proj) is a column
+        # slice whose check runs in the fused GEMM's epilogue (col_begin/
+        # col_end).  Off by default: at the fused OPT-1.3B QKV shape (N = 6144,
+        # K = 2048, M = 32) the tcgen05 decode GEMM runs 15.4-20.2 us in situ
+        # against cuBLAS's 13.5 us (profiles/r1_qkv_splitk.txt), so fusing
+        # helps the unprotected baseline more than FT2 (measured 8.4 % FT2
+        # overhead fused vs 2.8 % unfused).  Fault campaigns address sites per
+        # linear layer and need fuse_proj=False.
+        self.fuse_proj = fuse_proj
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
@@ -282,6 +308,57 @@ class Runner:
                               cur_layer=lid, cur_step=step)
         return y
 
+    def _group_ok(self, blk: Block, g: str) -> bool:
+        """A fused group runs as one GEMM when fusion is on, no fault sites are
+        armed, and at most one of its layers is protected (one column range)."""
+        if not self.fuse_proj or g not in blk.groups:
+            return False
+        if self.sites is not None:
+            raise ValueError("fault sites address single linear layers: build the runner with fuse_proj=False")
+        return sum(n in self.crit_names for n in blk.groups[g]) <= 1
+
+    def _linear_group(self, x2, blk: Block, g: str, phase: str, step_for_sites=None):
+        """A horizontally fused projection group (qkv / gate_up): one GEMM whose
+        output columns are the group's layers side by side.  FT2 work applies
+        to the protected layer's column slice only: first-token bounds on the
+        slice (strided view), and in decode the check in the fused GEMM's
+        epilogue restricted to [col_begin, col_end) -- the other columns are
+        written unchecked.  Returns the per-layer column views."""
+        w, b = blk.wf[g], blk.bf[g]
+        names = blk.groups[g]
+        offs = [0]
+        for n in names:
+            offs.append(offs[-1] + blk.w[n].shape[0])
+        crit = [i for i, n in enumerate(names) if n in self.crit_names]
+        ci = crit[0] if crit else None
+        st = self.state
+        M = x2.shape[0]
+        if phase == "prefill":
+            y = F.linear(x2, w, b)
+            if self._nv is not None:
+                for i, n in enumerate(names):
+                    F2.bounds_from_prefill(y[:, offs[i]:offs[i + 1]], None, self._nv_ws, seq_offsets=self.seq_offsets,
+                                           num_seqs=self.B, finalize=False, keys_out=self._nv_keys,
+                                           nan_vulnerable_count=self._nv[self._lin_id(blk.idx, n)])
+            if ci is not None and self.mode != "off":
+                cid = self._crit_id(blk.idx, names[ci])
+                F2.bounds_from_prefill(y[:, offs[ci]:offs[ci + 1]], st.bounds[cid], st.ws, seq_offsets=self.seq_offsets,
+                                       num_seqs=self.B, scale=self.scale, correct_nonfinite=True,
+                                       nonfinite_count=st.nonfinite[cid])
+        elif ci is not None and self.mode in ("fused", "fused_plain") and M <= FUSED_MAX_M:
+            cid = self._crit_id(blk.idx, names[ci])
+            y = torch.empty((M, w.shape[0]), dtype=torch.bfloat16, device=x2.device)
+            mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
+            F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, col_begin=offs[ci], col_end=offs[ci + 1],
+                                  bounds=st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid])
+        else:
+            y = F.linear(x2, w, b)
+            if ci is not None and (self.mode == "standalone" or (self.mode == "fused" and M > FUSED_MAX_M)):
+                cid = self._crit_id(blk.idx, names[ci])
+                F2.protect(y[:, offs[ci]:offs[ci + 1]], st.bounds[cid], num_seqs=self.B,
+                           corrected_count=st.corrected[cid])
+        return [y[:, offs[i]:offs[i + 1]] for i in range(len(names))]
+
     # ------------------------------------------------------------ forward
     def _block(self, blk: Block, x, phase, pos_idx=None, step=None):
         cfg = self.cfg
@@ -290,9 +367,12 @@ class Runner:
         T = x.shape[1]
         h = self._norm(x, blk.ln1_w, blk.ln1_b)
         h2 = h.reshape(-1, cfg.hidden)
-        q = self._linear(h2, blk, "q_proj", phase, step)
-        k = self._linear(h2, blk, "k_proj", phase, step)
-        v = self._linear(h2, blk, "v_proj", phase, step)
+        if self._group_ok(blk, "qkv"):
+            q, k, v = self._linear_group(h2, blk, "qkv", phase, step)
+        else:
+            q = self._linear(h2, blk, "q_proj", phase, step)
+            k = self._linear(h2, blk, "k_proj", phase, step)
+            v = self._linear(h2, blk, "v_proj", phase, step)
         q = q.view(B, T, H, D).transpose(1, 2)
         k = k.view(B, T, H, D).transpose(1, 2)
         v = v.view(B, T, H, D).transpose(1, 2)
@@ -317,8 +397,11 @@ class Runner:
             f = torch.relu(self._linear(h, blk, "fc1", phase, step))
             y = self._linear(f, blk, "fc2", phase, step)
         else:
-            g = self._linear(h, blk, "gate_proj", phase, step)
-            u = self._linear(h, blk, "up_proj", phase, step)
+            if self._group_ok(blk, "gate_up"):
+                g, u = self._linear_group(h, blk, "gate_up", phase, step)
+            else:
+                g = self._linear(h, blk, "gate_proj", phase, step)
+                u = self._linear(h, blk, "up_proj", phase, step)
             y = self._linear(F.silu(g) * u, blk, "down_proj", phase, step)
         return x + y.view(B, T, -1)
 

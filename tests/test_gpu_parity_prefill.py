@@ -212,3 +212,58 @@ def test_prefill_derive_workspace_reuse(ft2):
         rb, _, _ = oracle.bounds(plain.copy(), seq_offsets=so, correct_nonfinite=True)
         _, bnd, _, _, _ = _derive(ft2, x, w, b, so=so, S=S, ws=ws)
         assert np.array_equal(bnd, rb)
+
+
+# ------------------------------------------------------- split-K (small M) --
+SPLIT_SHAPES = [(256, 11008, 4096), (256, 4096, 11008), (192, 4096, 4096), (512, 2048, 8192), (136, 1032, 4096)]
+
+
+@pytest.fixture
+def split_on(monkeypatch):
+    """The persistent kernel's K split is opt-in (FT2_PREFILL_SPLITS, read per
+    call); -1 lets its planner choose."""
+    monkeypatch.setenv("FT2_PREFILL_SPLITS", "-1")
+    yield
+
+
+@pytest.mark.parametrize("M,N,K", SPLIT_SHAPES)
+def test_split_k_plain_check_and_no_split(ft2, split_on, M, N, K):
+    """Grids the tiles cannot fill split K through the fp32 workspace; with
+    and without the split the layer is within the GEMM tolerance of the fp64
+    oracle, and the CHECK epilogue (same split) is bit-exact vs the oracle's
+    R5 on the kernel's own PLAIN output."""
+    assert ft2.gemm_workspace_bytes(M, N, K) > 0, "this shape should split"
+    x, w, b = _operands(M, N, K, seed=M + K)
+    rows = np.unique(np.linspace(0, M - 1, 10).astype(int))
+    y_ref, _ = oracle.linear_f64(x[rows], w, b)
+    rms = np.sqrt(np.mean(y_ref ** 2, axis=1, keepdims=True))
+    tiny = torch.zeros(2, dtype=torch.int64, device="cuda")       # 16 bytes: no split
+    outs = []
+    for ws in (None, tiny):
+        y = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        ft2.protect_fused_gemm(dev(x), dev(w), y, bias=dev(b), mode=0, workspace=ws)
+        torch.cuda.synchronize()
+        g = _f64(host(y)[rows])
+        assert int((np.abs(g - y_ref) > 1e-2 * np.maximum(np.abs(y_ref), 1e-2 * rms)).sum()) == 0
+        outs.append(host(y))
+    plain = outs[0]
+    S = M
+    bnds = np.array([[oracle.f64_to_bf16(-0.2 - 0.001 * i), oracle.f64_to_bf16(0.25)] for i in range(S)], np.uint16)
+    y = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+    cnt = torch.zeros(S, dtype=torch.int32, device="cuda")
+    ft2.protect_fused_gemm(dev(x), dev(w), y, bias=dev(b), mode=1, bounds=dev(bnds), num_seqs=S, corrected_count=cnt)
+    ref = plain.copy()
+    rc = oracle.protect(ref, bnds, row_to_seq=np.arange(M, dtype=np.int32))
+    assert np.array_equal(host(y), ref)
+    assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), rc) and rc.sum() > 0
+    # the split workspace is self-cleaning: a second call gives the same bits
+    y2 = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+    ft2.protect_fused_gemm(dev(x), dev(w), y2, bias=dev(b), mode=0)
+    assert np.array_equal(host(y2), plain)
+
+
+@pytest.mark.parametrize("M,N,K,S", [(512, 4096, 4096, 32), (256, 11008, 4096, 16)])
+def test_split_k_derive_bit_exact(ft2, split_on, M, N, K, S):
+    x, w, b = _operands(M, N, K, seed=S + 3)
+    so = np.arange(0, M + 1, M // S).astype(np.int32)
+    _check_derive(ft2, x, w, b, so, S)

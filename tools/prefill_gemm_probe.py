@@ -10,7 +10,9 @@ import paper_conf_hpdc_sunzmg00y25_b200 as ft2
 
 R = int(os.environ.get("R", 20))
 shapes = [(4096, 2048, 2048), (4096, 2048, 8192), (4096, 4096, 4096), (4096, 11008, 4096), (4096, 4096, 11008),
-          (512, 4096, 4096)]
+          (512, 4096, 4096), (512, 11008, 4096), (512, 4096, 11008)]
+if os.environ.get("SMALL"):
+    shapes = [s for s in shapes if s[0] <= 512]
 for M, N, K in shapes:
     ws = [ft2_synth.gen_bf16_torch((N, K), 21 + i, 1, scale_log2=-6, device="cuda") for i in range(4)]
     x = ft2_synth.gen_bf16_torch((M, K), 20, 1, device="cuda")
