@@ -561,6 +561,20 @@ def kernel_rooflines(runner, dev, ft2):
     }
     del y
     torch.cuda.empty_cache()
+    # the FP32 variants (the paper's FP32 study, L334) on the same 1.44 GB:
+    # [65536, 5504] fp32; the values are the bf16 tensor's first half widened
+    y32 = ft2_synth.gen_bf16_torch((rows, n // 2), 11, 5, device=dev).float()
+    b32 = torch.zeros((1, 2), dtype=torch.float32, device=dev)
+    wide32 = torch.tensor([[-3.0e38, 3.0e38]], dtype=torch.float32, device=dev)
+    ms_b32 = time_it(lambda: ft2.bounds_from_prefill(y32, b32, ws))
+    ms_p32 = time_it(lambda: ft2.protect(y32, wide32, corrected_count=cnt))
+    for name, ms in (("bounds_fp32", ms_b32), ("protect_fp32", ms_p32)):
+        ach = nb / (ms / 1e3) / 1e9
+        prot[name] = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+                      "traffic": None, "us": 1000 * ms, "shape": [rows, n // 2],
+                      "algorithmic_bytes": "4 B read per element"}
+    del y32
+    torch.cuda.empty_cache()
     return {"roofline": gemm, "protect_kernels_roofline": prot, "prefill_derive_roofline": prefill_derive_roofline(
         dev, ft2, peaks, time_it), "c3_llama7b_decode_gemm": c3_decode_gemm(dev, ft2, peaks)}
 
