@@ -370,9 +370,13 @@ class Runner:
         if self._group_ok(blk, "qkv"):
             q, k, v = self._linear_group(h2, blk, "qkv", phase, step)
         else:
+            # v first: the protected projection then follows a torch kernel
+            # (layer norm) instead of a cuBLAS GEMM, after which the tcgen05
+            # GEMM's launch measured 1.3 us slower (tools/after_cublas_probe.py);
+            # the three projections are independent, so the order is free
+            v = self._linear(h2, blk, "v_proj", phase, step)
             q = self._linear(h2, blk, "q_proj", phase, step)
             k = self._linear(h2, blk, "k_proj", phase, step)
-            v = self._linear(h2, blk, "v_proj", phase, step)
         q = q.view(B, T, H, D).transpose(1, 2)
         k = k.view(B, T, H, D).transpose(1, 2)
         v = v.view(B, T, H, D).transpose(1, 2)

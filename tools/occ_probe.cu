@@ -23,7 +23,7 @@ int main() {
     cudaDeviceGetAttribute(&smem_blk_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev);
     printf("smem/SM %d, optin/block %d, reserved/block %d\n", smem_sm, smem_blk_optin, reserved);
-    for (int d : {80000, 100000, 107904, 110000, 113000, 115000}) {
+    for (int d : {0, 16384, 50000, 80000, 100000, 107904, 110000, 113000, 115000}) {
         for (int which = 0; which < 3; ++which) {
             void* f = which == 2 ? (void*)k3 : which ? (void*)k2 : (void*)k1;
             cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, d);
