@@ -424,7 +424,7 @@ def main():
     return 0
 
 
-def coverage_costs(cfg, B, T, G, dev, prompt, stream, runner_ft2, ms_off_ft2, rounds=5):
+def coverage_costs(cfg, B, T, G, dev, prompt, stream, runner_ft2, ms_off_ft2, rounds=9):
     """FT2 overhead under the protection coverages of PAPER.md Table 1
     (L164-L177): FT2's critical layers, MaxiMals' (out_proj, fc2),
     Global Clipper's (v_proj, out_proj), and every linear layer (the "nearly

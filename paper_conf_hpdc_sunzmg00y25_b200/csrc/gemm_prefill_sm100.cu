@@ -63,7 +63,11 @@ struct PCfg {
 constexpr int kPSeqTab = 512;                        // sequences kept in the per-CTA table
 constexpr int kPMaxRowSites = 4;                     // fault sites one row may hold per tile
 constexpr int kPMiscBytes = 256;
-constexpr int kPSmemBytes = 1024 + kPTileBytes + kPMiscBytes + 3 * kPSeqTab * 4;
+// split-K staging: per epilogue column half, 128 rows x 16 fp32 (+4 pad: the
+// per-row float4 writes of a quarter-warp hit disjoint banks)
+constexpr int kSkStride = 20;
+constexpr int kSkStageBytes = 2 * kPBM * kSkStride * 4;
+constexpr int kPSmemBytes = 1024 + kPTileBytes + kPMiscBytes + 3 * kPSeqTab * 4 + kSkStageBytes;
 constexpr int kPGemmDerive = 2;
 constexpr int kSplitCounters = 16384;   // split-K arrival counters at the head of the GEMM workspace
 
@@ -146,6 +150,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     uint32_t* tab_lo = reinterpret_cast<uint32_t*>(misc + kPMiscBytes);  // 0x10000 - min key (0: none)
     uint32_t* tab_hi = tab_lo + kPSeqTab;                                 // max key + 1 (0: none)
     uint32_t* tab_nf = tab_hi + kPSeqTab;                                 // non-finite count
+    float* sk_stage = reinterpret_cast<float*>(tab_nf + kPSeqTab);        // [2][128][kSkStride] (split-K)
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const bool derive = p.mode == kPGemmDerive;
@@ -298,11 +303,16 @@ __global__ void __launch_bounds__(kPThreads, 1)
             const bool split = p.splits > 1;
             // 128 x 256 half-tile id; pairs may cover one phantom m-tile past tilesM
             const int half = m0 / kPBM + (MC == 2 ? ((p.tilesM + 1) & ~1) : p.tilesM) * (n0 / kPBN);
-            float* const slot0 = split ? p.skws + ((size_t)half * p.splits * kPBM + e) * kPBN : nullptr;
+            // split-K slots: [half-tile][split][16 column chunks][128 rows][16],
+            // so a chunk is one contiguous 8 KB block (coalesced copies)
+            float* const slot0 = split ? p.skws + (size_t)half * p.splits * kPBM * kPBN : nullptr;
+            const int grp = (warp - 2) >> 2;  // column half = staging group (4 warps, rows 0..127)
+            float* const stg = sk_stage + grp * kPBM * kSkStride;
             if (split) {
-                // K split: stage this unit's fp32 partial rows; the last of the
-                // tile's splits to arrive sums all slots in split order
-                // (deterministic) and runs the epilogue below
+                // K split: stage this unit's fp32 partial tile through shared
+                // memory into its slot (chunk-major, 16-byte coalesced stores);
+                // the last of the tile's splits to arrive sums all slots in
+                // split order (deterministic) and runs the epilogue below
                 float* mine = slot0 + (size_t)ks * kPBM * kPBN;
 #pragma unroll 1
                 for (int c0 = h0; c0 < h0 + kPBN / 2; c0 += 32) {
@@ -310,10 +320,22 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     tmem_ld32(taddr + (uint32_t)c0, r);
                     tmem_wait_ld();
 #pragma unroll
-                    for (int j = 0; j < 8; ++j)
-                        __stcg(reinterpret_cast<float4*>(mine + c0) + j,
-                               make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
-                                           __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3])));
+                    for (int sub = 0; sub < 2; ++sub) {
+#pragma unroll
+                        for (int j = 0; j < 4; ++j)
+                            *reinterpret_cast<float4*>(stg + e * kSkStride + 4 * j) =
+                                make_float4(__uint_as_float(r[16 * sub + 4 * j]), __uint_as_float(r[16 * sub + 4 * j + 1]),
+                                            __uint_as_float(r[16 * sub + 4 * j + 2]), __uint_as_float(r[16 * sub + 4 * j + 3]));
+                        named_bar(2 + grp, 128);
+                        float* chunk = mine + (size_t)((c0 + 16 * sub) >> 4) * (kPBM * 16);
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            const int i = e + 128 * k;   // float4 index within the chunk
+                            __stcg(reinterpret_cast<float4*>(chunk) + i,
+                                   *reinterpret_cast<const float4*>(stg + (i >> 2) * kSkStride + 4 * (i & 3)));
+                        }
+                        named_bar(2 + grp, 128);
+                    }
                 }
                 tc_fence_before();
                 __syncwarp();
@@ -338,22 +360,39 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     tmem_ld32(taddr + (uint32_t)c0, r);
                     tmem_wait_ld();
                 } else {
-                    float acc[32];
+                    // coalesced chunk sums (split order 0..S-1 per element),
+                    // transposed back to one row per thread through shared memory
 #pragma unroll
-                    for (int j = 0; j < 8; ++j) {
-                        const float4 v = __ldcg(reinterpret_cast<const float4*>(slot0 + c0) + j);
-                        acc[4 * j] = v.x; acc[4 * j + 1] = v.y; acc[4 * j + 2] = v.z; acc[4 * j + 3] = v.w;
-                    }
-                    for (int sk = 1; sk < p.splits; ++sk) {
-                        const float* sl = slot0 + (size_t)sk * kPBM * kPBN + c0;
+                    for (int sub = 0; sub < 2; ++sub) {
+                        const size_t coff = (size_t)((c0 + 16 * sub) >> 4) * (kPBM * 16);
+                        float4 acc[4];
 #pragma unroll
-                        for (int j = 0; j < 8; ++j) {
-                            const float4 v = __ldcg(reinterpret_cast<const float4*>(sl) + j);
-                            acc[4 * j] += v.x; acc[4 * j + 1] += v.y; acc[4 * j + 2] += v.z; acc[4 * j + 3] += v.w;
+                        for (int k = 0; k < 4; ++k)
+                            acc[k] = __ldcg(reinterpret_cast<const float4*>(slot0 + coff) + e + 128 * k);
+                        for (int sk = 1; sk < p.splits; ++sk) {
+                            const float4* sl = reinterpret_cast<const float4*>(slot0 + (size_t)sk * kPBM * kPBN + coff);
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) {
+                                const float4 v = __ldcg(sl + e + 128 * k);
+                                acc[k].x += v.x; acc[k].y += v.y; acc[k].z += v.z; acc[k].w += v.w;
+                            }
                         }
-                    }
 #pragma unroll
-                    for (int j = 0; j < 32; ++j) r[j] = __float_as_uint(acc[j]);
+                        for (int k = 0; k < 4; ++k) {
+                            const int i = e + 128 * k;
+                            *reinterpret_cast<float4*>(stg + (i >> 2) * kSkStride + 4 * (i & 3)) = acc[k];
+                        }
+                        named_bar(2 + grp, 128);
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const float4 v = *reinterpret_cast<const float4*>(stg + e * kSkStride + 4 * j);
+                            r[16 * sub + 4 * j] = __float_as_uint(v.x);
+                            r[16 * sub + 4 * j + 1] = __float_as_uint(v.y);
+                            r[16 * sub + 4 * j + 2] = __float_as_uint(v.z);
+                            r[16 * sub + 4 * j + 3] = __float_as_uint(v.w);
+                        }
+                        named_bar(2 + grp, 128);
+                    }
                 }
                 const int nb = n0 + c0;
                 if (!row_ok || nb >= p.N) continue;
