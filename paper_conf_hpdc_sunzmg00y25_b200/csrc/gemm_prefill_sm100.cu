@@ -623,12 +623,12 @@ PrefillSplit plan_prefill_split(int32_t M, int32_t N, int32_t K, size_t ws_bytes
     r.cnt_bytes = (size_t)kSplitCounters * 4;
     if ((size_t)tilesMp * tilesN > (size_t)kSplitCounters) return r;
     const size_t per_split = (size_t)tilesMp * kPBM * tilesN * kPBN * 4;
-    // Opt-in (FT2_PREFILL_SPLITS = s >= 2, or -1 for the planner below): the
-    // first implementation stages partials with one thread per row (16-byte
-    // stores spread over 32 rows per warp instruction) and measured SLOWER
-    // than the unsplit kernel at every small-M shape tried (M = 256, 4096^2:
-    // 29 -> 47 us; profiles/r1_prefill_splitk.txt), so it is off by default
-    // until the partial tiles move through shared memory / TMA bulk stores.
+    // Opt-in (FT2_PREFILL_SPLITS = s >= 2, or -1 for the planner below).
+    // Measured (profiles/r1_prefill_splitk.txt): with per-row partial stores
+    // the split was 1.6x SLOWER; with the shared-memory-staged coalesced
+    // slots it is at par (M = 256, 4096^2: 28.7 us unsplit, 28.9 at s = 4),
+    // because the mainloop is latency-bound at ~0.45 us per k-block per CTA
+    // pair either way -- so it stays off until that is fixed.
     const char* ev = getenv("FT2_PREFILL_SPLITS");   // read per call: tests toggle it
     const int env = ev ? atoi(ev) : 0;
     if (env == 0 || env == 1) return r;
