@@ -145,10 +145,12 @@ __device__ __forceinline__ uint16_t bf16_rne(float f) {
     u += 0x7FFFu + ((u >> 16) & 1u);
     return (uint16_t)(u >> 16);
 }
-// fp32 -> activation format, round-to-nearest-even.
+// fp32 -> activation format, round-to-nearest-even; NaN -> the canonical
+// quiet NaN of the format (bf16 0x7FC0, fp16 0x7E00), as the oracle's R0.
 template <int DT = 0>
 __device__ __forceinline__ uint16_t rne16(float f) {
     if (DT == 0) return bf16_rne(f);
+    if (f != f) return 0x7E00;
     return __half_as_ushort(__float2half_rn(f));
 }
 

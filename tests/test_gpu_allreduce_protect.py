@@ -131,3 +131,42 @@ def test_allreduce_protect_p1_in_process():
         assert int(rpc.words[0].item()) == CALLS + 6     # epoch advanced once per call
     finally:
         dist.destroy_process_group()
+
+
+def test_allreduce_protect_fp16_plain_and_row_map_p1():
+    """FP16 (the paper's precision), PLAIN mode (a plain one-shot all-reduce),
+    a row -> sequence map with unmapped (-1) rows, no bias; P = 1."""
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+    port = _port()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        rows, n = 24, 1024
+        rpc = tp.RowParallelCheck(rows, n, dtype=torch.float16)
+        rng = np.random.default_rng(4)
+        p16 = (rng.standard_normal((rows, n)) * 0.8).astype(np.float16)
+        p16.reshape(-1)[::97] = np.float16(np.nan)
+        bits = p16.view(np.uint16)
+        rpc.partial(0).copy_(torch.from_numpy(bits.view(np.int16).copy()).view(torch.float16).cuda())
+        y = torch.empty((rows, n), dtype=torch.float16, device="cuda")
+        rpc(0, y, mode=0)                                   # PLAIN: sum (+ no bias), round, no check
+        torch.cuda.synchronize()
+        want, _ = oracle.allreduce_protect(bits[None], dtype=oracle.DT_FP16)
+        got = y.cpu().view(torch.int16).numpy().view(np.uint16)
+        assert np.array_equal(got, want)
+        S = 3
+        r2s = (np.arange(rows) % 4).astype(np.int32) - 1     # rows with -1 are left unchecked
+        bnd = np.array([[oracle.f64_to(-0.5, oracle.DT_FP16), oracle.f64_to(0.5, oracle.DT_FP16)],
+                        [oracle.f64_to(-1.0, oracle.DT_FP16), oracle.f64_to(0.25, oracle.DT_FP16)],
+                        [oracle.f64_to(-0.1, oracle.DT_FP16), oracle.f64_to(2.0, oracle.DT_FP16)]], np.uint16)
+        cnt = torch.zeros(S, dtype=torch.int32, device="cuda")
+        rpc.partial(1).copy_(rpc.partial(0))
+        rpc(1, y, mode=1, bounds=torch.from_numpy(bnd.view(np.int16)).view(torch.float16).cuda(),
+            row_to_seq=torch.from_numpy(r2s).cuda(), num_seqs=S, corrected_count=cnt)
+        torch.cuda.synchronize()
+        want, wcnt = oracle.allreduce_protect(bits[None], bounds_=bnd, row_to_seq=r2s, dtype=oracle.DT_FP16)
+        got = y.cpu().view(torch.int16).numpy().view(np.uint16)
+        assert np.array_equal(got, want) and np.array_equal(cnt.cpu().numpy().astype(np.uint32), wcnt)
+        assert int(wcnt.sum()) > 0 and rpc.status() == 0
+    finally:
+        dist.destroy_process_group()
