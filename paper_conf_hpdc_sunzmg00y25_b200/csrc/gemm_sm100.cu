@@ -89,6 +89,7 @@ struct GemmK {
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
     int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
+    int32_t trigger;   // issue griddepcontrol.launch_dependents early (FT2_GEMM_TRIGGER, default 1)
     int32_t rows_per_slot;  // ceil(128 / splitk): rows of one split-K receive slot
     uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
 };
@@ -286,7 +287,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     // peers may push into my receive buffer once my barrier is initialised
     if (splitk > 1) cluster_arrive_relaxed();
     const uint32_t tmem_base = *tmem_base_sh;
-    griddep_launch();  // the next kernel in the stream may start its prologue (PDL)
+    if (p.trigger) griddep_launch();  // the next kernel in the stream may start its prologue (PDL)
 
     if (warp == 0) {
         if (lane == 0) {
@@ -740,6 +741,8 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cur_step = a.cur_step;
     p.base_row = a.base_row;
     p.w_static = a.w_static;
+    static const int trig = env_int("FT2_GEMM_TRIGGER", 1);
+    p.trigger = trig;
     p.rows_per_slot = (kBlockA + g.splitk - 1) / g.splitk;
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
     if (g.deep) {
