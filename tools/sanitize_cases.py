@@ -35,5 +35,35 @@ for (M, N, K) in [(8, 384, 512), (32, 256, 128), (1, 200, 72), (160, 256, 192)]:
     ft2.protect_fused_gemm(x, w, out, bias=bias, mode=1, bounds=bb, num_seqs=1, corrected_count=c, sites=sites,
                            cur_layer=0, cur_step=1)
     ft2.protect_fused_gemm(x, w, out, bias=bias, mode=0)
+# FP32 variants (bounds with correction, protect, inject)
+y32 = torch.randn((48, 260), device=dev)
+y32.view(-1)[::37] = float("nan")
+y32.view(-1)[5::53] = float("inf")
+b32 = torch.zeros((4, 2), dtype=torch.float32, device=dev)
+so32 = torch.tensor([0, 10, 10, 30, 48], dtype=torch.int32, device=dev)
+ft2.bounds_from_prefill(y32, b32, ft2.make_workspace(4), seq_offsets=so32, num_seqs=4, correct_nonfinite=True,
+                        keys_out=k)
+ft2.bounds_finalize(k, b32)
+ft2.protect(y32, b32, row_to_seq=(torch.arange(48, device=dev) % 4).to(torch.int32), num_seqs=4, corrected_count=cnt)
+s32 = ft2.make_fault_sites(1, 0, 48, 0, [260], 4, 8, dtype=2)
+ft2.inject_faults(y32, s32, 0, 2)
+# persistent kernel with the (opt-in) K split, and DERIVE
+os.environ["FT2_PREFILL_SPLITS"] = "2"
+for (M, N, K) in [(256, 512, 1024), (136, 264, 1024)]:
+    x = ft2_synth.gen_bf16_torch((M, K), 6, 1, device=dev)
+    w = ft2_synth.gen_bf16_torch((N, K), 7, 1, scale_log2=-5, device=dev)
+    out = torch.empty((M, N), dtype=torch.bfloat16, device=dev)
+    ft2.protect_fused_gemm(x, w, out, mode=0)
+    sq = torch.tensor([0, M // 2, M], dtype=torch.int32, device=dev)
+    bd = torch.zeros((2, 2), dtype=torch.bfloat16, device=dev)
+    ft2.prefill_fused_gemm(x, w, out, bd, ft2.make_workspace(2), seq_offsets=sq, num_seqs=2)
+os.environ.pop("FT2_PREFILL_SPLITS")
+# fused row-parallel all-reduce + check at P = 1 (handshake skipped) through the C ABI directly
+pp = torch.tensor([yd.data_ptr()], dtype=torch.int64, device=dev)
+fl = torch.zeros(1, dtype=torch.int32, device=dev)
+fp = torch.tensor([fl.data_ptr()], dtype=torch.int64, device=dev)
+words = torch.zeros(3, dtype=torch.int32, device=dev)
+yo = torch.empty_like(yd)
+ft2.allreduce_protect(pp, 520, 1, 0, fp, words, yo, mode=1, bounds=b[:1].clone(), num_seqs=1, corrected_count=cnt)
 torch.cuda.synchronize()
 print("sanitize cases: done")
