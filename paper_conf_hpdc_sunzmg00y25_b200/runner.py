@@ -192,6 +192,10 @@ class Runner:
         # overhead fused vs 2.8 % unfused).  Fault campaigns address sites per
         # linear layer and need fuse_proj=False.
         self.fuse_proj = fuse_proj
+        # critical layers whose decode check runs as cuBLAS + ft2_protect even
+        # in "fused" mode (FT2_STANDALONE_LAYERS="v_proj,out_proj", experiments)
+        import os
+        self.standalone_layers = set(filter(None, os.environ.get("FT2_STANDALONE_LAYERS", "").split(",")))
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
@@ -282,7 +286,7 @@ class Runner:
         # which has no split-K and starves the grid at M = 256 (measured 1.4-2.5x
         # slower than cuBLAS, profiles/r1_m256_probe.txt), so there "fused" runs
         # cuBLAS + ft2_protect and "fused_plain" plain cuBLAS.
-        fused_ok = x2.shape[0] <= FUSED_MAX_M
+        fused_ok = x2.shape[0] <= FUSED_MAX_M and name not in self.standalone_layers
         if not crit or self.mode in ("off", "standalone") or not fused_ok:
             if crit and not fused_ok and self.mode == "fused":
                 y = F.linear(x2, w, b)
