@@ -90,6 +90,15 @@ struct GemmK {
     const int32_t* base_row;
     int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
     int32_t trigger;   // issue griddepcontrol.launch_dependents early (FT2_GEMM_TRIGGER, default 1)
+    // K split through global memory instead of the cluster (no cluster launch:
+    // every CTA starts at once; the last split of a tile to arrive sums the
+    // tile's fp32 slots in split order and finishes all 128 rows).  Opt-in
+    // experiment (FT2_GEMM_GSPLIT=1): parity-clean but measured 3-4x slower
+    // than the cluster/DSMEM split (2048x2048, M = 32: 21.3 vs 5.7 us back to
+    // back), so the late-starting 16th cluster of 8 is the cheaper evil.
+    int32_t gsplit;
+    float* gws;        // [tiles][splitk][128][BN] fp32 partial slots
+    uint32_t* gcnt;    // [tiles] arrival counters (self-cleaning)
     int32_t rows_per_slot;  // ceil(128 / splitk): rows of one split-K receive slot
     uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
 };
@@ -253,6 +262,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     uint32_t* site_n = tmem_base_sh + 1;
     uint32_t* site_e = site_n + 1;                // [kMaxSitesPerCta] local element a * BN + b
     uint32_t* site_m = site_e + kMaxSitesPerCta;  // [kMaxSitesPerCta] xor mask
+    uint32_t* gs_last = site_m + kMaxSitesPerCta;  // global split: this CTA finishes its tile
     TabE* row_tab = reinterpret_cast<TabE*>(misc + C::kMiscBytes);  // [128]
     TabE* col_tab = row_tab + kBlockA;                                // [BN]
     uint32_t* row_cnt = reinterpret_cast<uint32_t*>(col_tab + BN);    // [128]
@@ -265,8 +275,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     const int kb1 = (int)((int64_t)(split + 1) * p.nkb / splitk);
     const int nk = kb1 - kb0;
     // rows of the tile this CTA finishes: all of them, or its split-K slice
-    const int r0 = (int)(((uint32_t)(split * kBlockA) * p.sk_magic) >> 24);
-    const int r1 = (int)(((uint32_t)((split + 1) * kBlockA) * p.sk_magic) >> 24);
+    const bool gs = splitk > 1 && p.gsplit;    // split through global memory
+    const bool cs = splitk > 1 && !p.gsplit;   // split across the cluster (DSMEM)
+    const int r0 = gs ? 0 : (int)(((uint32_t)(split * kBlockA) * p.sk_magic) >> 24);
+    const int r1 = gs ? kBlockA : (int)(((uint32_t)((split + 1) * kBlockA) * p.sk_magic) >> 24);
+    const int tile_id = tileA + p.tilesA * tileB;
 
     if (warp == 0 && lane == 0) {
         FT2_TRACE(0);
@@ -275,7 +288,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
         mbar_init(tmem_full, 1);
         mbar_init(recv_bar, 1);
-        if (splitk > 1)  // bytes the other splits will push into my slice
+        if (cs)  // bytes the other splits will push into my slice
             mbar_expect_tx(recv_bar, (uint32_t)((splitk - 1) * (r1 - r0) * BN * 4));
         fence_mbar_init();
         *site_n = 0;
@@ -285,7 +298,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     __syncthreads();
     tc_fence_after();
     // peers may push into my receive buffer once my barrier is initialised
-    if (splitk > 1) cluster_arrive_relaxed();
+    if (cs) cluster_arrive_relaxed();
     const uint32_t tmem_base = *tmem_base_sh;
     if (p.trigger) griddep_launch();  // the next kernel in the stream may start its prologue (PDL)
 
@@ -387,7 +400,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const int nrow = r1 - r0;
         const int nvec = nrow * (BN / 4);
         const uint32_t inv = (uint32_t)((1u << 20) + nrow - 1) / (uint32_t)nrow;  // v / nrow == (v * inv) >> 20
-        if (splitk > 1) cluster_wait();  // every peer's receive barrier is initialised
+        if (cs) cluster_wait();  // every peer's receive barrier is initialised
         mbar_wait(tmem_full, 0);
         if (a == 0) FT2_TRACE(5);
         tc_fence_after();
@@ -401,10 +414,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
                 for (int j = 0; j < 32; ++j) r[j] = 0u;
             }
+            if (gs) {
+                float4* g = reinterpret_cast<float4*>(p.gws + ((size_t)(tile_id * splitk + split) * kBlockA + a) * BN);
 #pragma unroll
-            for (int j = 0; j < 32; j += 4) {
-                if (local) st_shared_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
-                else st_async_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
+                for (int j = 0; j < 32; j += 4)
+                    __stcg(g + j / 4, make_float4(__uint_as_float(r[j]), __uint_as_float(r[j + 1]),
+                                                  __uint_as_float(r[j + 2]), __uint_as_float(r[j + 3])));
+            } else {
+#pragma unroll
+                for (int j = 0; j < 32; j += 4) {
+                    if (local) st_shared_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
+                    else st_async_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
+                }
             }
         } else
 #pragma unroll 1
@@ -416,30 +437,56 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
                 for (int j = 0; j < 16; ++j) r[j] = 0u;
             }
+            if (gs) {
+                float4* g = reinterpret_cast<float4*>(p.gws + ((size_t)(tile_id * splitk + split) * kBlockA + a) * BN + c0);
 #pragma unroll
-            for (int j = 0; j < 16; j += 4) {
-                if (local) st_shared_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
-                else st_async_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
+                for (int j = 0; j < 16; j += 4)
+                    __stcg(g + j / 4, make_float4(__uint_as_float(r[j]), __uint_as_float(r[j + 1]),
+                                                  __uint_as_float(r[j + 2]), __uint_as_float(r[j + 3])));
+            } else {
+#pragma unroll
+                for (int j = 0; j < 16; j += 4) {
+                    if (local) st_shared_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
+                    else st_async_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3], dbar);
+                }
             }
         }
         if (tid == 64) FT2_TRACE(8);
         // ------------------------------------ finish the slice (epilogue warps)
+        if (gs) __threadfence();   // my slot before my arrival
         named_bar(2, 128);  // tables, site list and my own rows are in shared memory
         if (tid == 64) FT2_TRACE(9);
-        if (splitk > 1) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
+        if (cs) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
+        bool finisher = true;
+        if (gs) {   // the last split of the tile to arrive finishes it
+            if (tid == 64) {
+                const bool last = atom_add_acq_rel_gpu(p.gcnt + tile_id, 1u) == (uint32_t)(splitk - 1);
+                if (last) p.gcnt[tile_id] = 0u;
+                *gs_last = last ? 1u : 0u;
+            }
+            named_bar(2, 128);
+            finisher = *gs_last != 0u;
+        }
         if (tid == 64) FT2_TRACE(6);
         const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
         uint16_t* const y = p.y;
         const int64_t ldy = p.ldy;
 #pragma unroll 1
-        for (int v = e; v < nvec; v += 128) {
+        for (int v = e; v < (finisher ? nvec : 0); v += 128) {
             // consecutive threads take consecutive rows (coalesced stores in swap-AB mode)
             const int c4 = (int)(((uint32_t)v * inv) >> 20), lr = v - c4 * nrow, la = r0 + lr;
-            const float* src = recv + lr * C::kRecvStride + c4 * 4;
             float4 part[kMaxSplitK];
+            if (gs) {   // the tile's slots in split order, from L2
+                const float* g = p.gws + ((size_t)tile_id * splitk * kBlockA + la) * BN + c4 * 4;
 #pragma unroll
-            for (int rr = 0; rr < kMaxSplitK; ++rr)
-                if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
+                for (int rr = 0; rr < kMaxSplitK; ++rr)
+                    if (rr < splitk) part[rr] = __ldcg(reinterpret_cast<const float4*>(g + (size_t)rr * kBlockA * BN));
+            } else {
+                const float* src = recv + lr * C::kRecvStride + c4 * 4;
+#pragma unroll
+                for (int rr = 0; rr < kMaxSplitK; ++rr)
+                    if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
+            }
             float4 acc = part[0];
 #pragma unroll
             for (int rr = 1; rr < kMaxSplitK; ++rr)
@@ -449,7 +496,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                               (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4);
         }
         if (tid == 64) FT2_TRACE(7);
-        if (p.counts != nullptr && p.mode == FT2_GEMM_CHECK) {
+        if (p.counts != nullptr && p.mode == FT2_GEMM_CHECK && finisher) {
             named_bar(3, 128);  // every finish4 of this CTA has counted
             if (!SWAP && row_cnt[e] != 0u) atomicAdd(&p.counts[row_tab[e].seq], row_cnt[e]);
             for (int c = e; SWAP && c < BN; c += 128)
@@ -457,7 +504,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         }
     }
     // warps 0 and 1 pair their prologue cluster arrive (no finish work for them)
-    if (splitk > 1 && warp < 2) cluster_wait();
+    if (cs && warp < 2) cluster_wait();
     tc_fence_before();
     __syncthreads();
     if (warp == 1) {
@@ -649,7 +696,7 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     if (dbg) {
         fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d bn=%d tiles=%dx%d nkb=%d splitk=%d deep=%d clusters(sk)=", M,
                 N, K, g.swap, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk, g.deep);
-        for (int sk = 2; sk <= 8 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
+        for (int sk = 2; sk <= 16 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
         int occ = -1;
         if (g.bn == 32) {
             set_attrs<32, true, 0, false>();
@@ -670,11 +717,22 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     return g;
 }
 
+// Global-memory K split of the decode kernel: counters at the workspace head,
+// then [tiles][splitk][128][bn] fp32 slots.
+constexpr size_t kDecodeCounterBytes = 65536;
+static size_t decode_gsplit_bytes(const GemmPlan& g) {
+    return kDecodeCounterBytes + (size_t)g.tilesA * g.tilesB * g.splitk * kBlockA * g.bn * 4;
+}
+
 // The decode kernel's cluster split-K needs no global workspace; the
 // persistent kernel (M > swap_max_m()) uses one for its K splits when the
 // tiles alone cannot fill the machine (optional: less space, fewer splits).
 size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K) {
-    if (M <= swap_max_m()) return 0;
+    if (M <= swap_max_m()) {
+        if (!env_int("FT2_GEMM_GSPLIT", 0)) return 0;
+        const GemmPlan g = plan_gemm(M, N, K);
+        return g.splitk > 1 ? decode_gsplit_bytes(g) : 0;
+    }
     return plan_prefill_split(M, N, K, (size_t)-1).need_bytes;
 }
 
@@ -704,7 +762,7 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     attr[2].id = cudaLaunchAttributeClusterSchedulingPolicyPreference;
     attr[2].val.clusterSchedulingPolicyPreference = cudaClusterSchedulingPolicySpread;
     cfg.attrs = attr;
-    cfg.numAttrs = p.splitk > 1 ? (spread_policy() ? 3 : 2) : 1;
+    cfg.numAttrs = (p.splitk > 1 && !p.gsplit) ? (spread_policy() ? 3 : 2) : 1;
     e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP, DT, DEEP>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
@@ -743,6 +801,17 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.w_static = a.w_static;
     static const int trig = env_int("FT2_GEMM_TRIGGER", 1);
     p.trigger = trig;
+    // K split through global memory (FT2_GEMM_GSPLIT=1; needs the workspace)
+    static const int gsplit_env = env_int("FT2_GEMM_GSPLIT", 0);
+    p.gsplit = 0;
+    if (gsplit_env && g.splitk > 1 && !g.deep) {
+        const size_t need = decode_gsplit_bytes(g);
+        if (a.ws != nullptr && a.ws_bytes >= need) {
+            p.gsplit = 1;
+            p.gcnt = static_cast<uint32_t*>(a.ws);
+            p.gws = reinterpret_cast<float*>(static_cast<char*>(a.ws) + kDecodeCounterBytes);
+        }
+    }
     p.rows_per_slot = (kBlockA + g.splitk - 1) / g.splitk;
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
     if (g.deep) {
