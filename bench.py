@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--prompt", type=int, default=128)
     ap.add_argument("--gen", type=int, default=60)
     ap.add_argument("--no-extras", action="store_true", help="skip the kernel roofline / cpu baseline legs")
-    ap.add_argument("--leg", default=None, choices=["c3", "c4", "c5"],
+    ap.add_argument("--leg", default=None, choices=["c3", "c4", "c5", "models"],
                     help="run one measurement leg alone and print its JSON (c3: Llama-2-7B decode GEMMs; "
                          "c4: Llama-2-13B tensor-parallel bounds over the ranks (NCCL MAX all-reduce); "
                          "c5: SDC fault-injection campaign, trials sharded over ranks)")
@@ -278,6 +278,10 @@ def main():
     if args.leg == "c3":
         if rank == 0:
             print(json.dumps({"leg": "c3", **c3_decode_gemm(dev, ft2, load_peaks())}), flush=True)
+        return 0
+    if args.leg == "models":
+        if rank == 0:
+            print(json.dumps({"leg": "models", **paper_models_leg(dev, ft2, load_peaks())}), flush=True)
         return 0
     if args.leg == "c4":
         res = c4_tp_bounds(args, dev, rank, world)
@@ -616,7 +620,113 @@ def kernel_rooflines(runner, dev, ft2):
     del y32
     torch.cuda.empty_cache()
     return {"roofline": gemm, "protect_kernels_roofline": prot, "prefill_derive_roofline": prefill_derive_roofline(
-        dev, ft2, peaks, time_it), "c3_llama7b_decode_gemm": c3_decode_gemm(dev, ft2, peaks)}
+        dev, ft2, peaks, time_it), "c3_llama7b_decode_gemm": c3_decode_gemm(dev, ft2, peaks),
+        "paper_models": paper_models_leg(dev, ft2, peaks)}
+
+
+# The paper's seven LLMs (Table 2; public model-card
+# shapes): (arch, hidden, ffn, layers, kv width).  Critical layers per Table 1:
+# OPT / GPT-J v, out, fc2; Llama / Vicuna / Qwen2 v, o, up, down (Qwen2's v is
+# GQA-narrow: kv heads x 128).
+PAPER_MODELS = {
+    "opt-6.7b": ("opt", 4096, 16384, 32, 4096), "opt-2.7b": ("opt", 2560, 10240, 32, 2560),
+    "gptj-6b": ("opt", 4096, 16384, 28, 4096), "llama2-7b": ("llama", 4096, 11008, 32, 4096),
+    "vicuna-7b": ("llama", 4096, 11008, 32, 4096), "qwen2-7b": ("llama", 3584, 18944, 28, 512),
+    "qwen2-1.5b": ("llama", 1536, 8960, 28, 256),
+}
+
+
+def paper_models_leg(dev, ft2, peaks, B=32, T=128, nb=4, R=5):
+    """FT2's per-request work on activations shaped like the paper's seven
+    LLMs (north star; Table 2), one GPU, B = 32: per decode step the critical
+    layers' fused GEMM (CHECK) vs cuBLAS and vs cuBLAS + ft2_protect, and per
+    prefill (B x T = 4096 tokens) the first-token bound sweeps.  Measured on
+    `nb` distinct blocks of seeded weights in one CUDA graph (beyond L2) and
+    scaled by the model's layer count (stated)."""
+    import torch
+
+    import ft2_synth
+
+    hbm_peak = (peaks or {}).get("hbm_gbs", 6650.0)
+    stream = torch.cuda.current_stream()
+
+    def gtime(fn):
+        fn()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            fn()
+        for _ in range(3):
+            g.replay()
+        ts = []
+        for _ in range(R):
+            torch.cuda.synchronize()
+            a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            g.replay()
+            b_.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b_) * 1000.0)
+        return statistics.median(ts)
+
+    out = {"B": B, "prefill_tokens": B * T, "blocks_measured": nb,
+           "note": "per-step and per-prefill times = measured on nb blocks x (layers / nb)"}
+    for mi, (name, (arch, h, f, L, kv)) in enumerate(PAPER_MODELS.items()):
+        crit = [("v", kv, h), ("out", h, h), ("fc2", h, f)] if arch == "opt" else \
+               [("v", kv, h), ("o", h, h), ("up", f, h), ("down", h, f)]
+        layers = []
+        for bi in range(nb):
+            for li, (ln, N, K) in enumerate(crit):
+                w = ft2_synth.gen_bf16_torch((N, K), 5000 + 97 * mi + 11 * bi + li, 7,
+                                             scale_log2=ft2_synth.weight_scale_log2(K), device=dev)
+                layers.append((w, N, K))
+        xs = {K: ft2_synth.gen_bf16_torch((B, K), 5900 + K % 97, 7, device=dev) for _, _, K in layers}
+        ys = [torch.empty((B, N), dtype=torch.bfloat16, device=dev) for _, N, _ in layers]
+        bnd = torch.tensor([[-1.0, 1.0]], dtype=torch.bfloat16, device=dev).repeat(B, 1)
+        cnt = torch.zeros(B, dtype=torch.int32, device=dev)
+
+        def fused():
+            for (w, N, K), y in zip(layers, ys):
+                ft2.protect_fused_gemm(xs[K], w, y, mode=1 | 16, bounds=bnd, num_seqs=B, corrected_count=cnt)
+
+        def cublas():
+            for (w, N, K), y in zip(layers, ys):
+                torch.mm(xs[K], w.t(), out=y)
+
+        def cublas_protect():
+            for (w, N, K), y in zip(layers, ys):
+                torch.mm(xs[K], w.t(), out=y)
+                ft2.protect(y, bnd, num_seqs=B, corrected_count=cnt)
+
+        scale = L / nb
+        t_f, t_c, t_cp = gtime(fused) * scale, gtime(cublas) * scale, gtime(cublas_protect) * scale
+        wbytes = sum(N * K * 2 for _, N, K in layers) * scale
+        del layers, xs, ys
+        # prefill bound sweeps: one block's critical outputs [B*T, N], rotated over 2 copies
+        outs = [[ft2_synth.gen_bf16_torch((B * T, N), 6100 + 13 * mi + 3 * c + li, 7, device=dev)
+                 for li, (_, N, _) in enumerate(crit)] for c in range(2)]
+        so = torch.arange(0, B * T + 1, T, dtype=torch.int32, device=dev)
+        bb = torch.zeros((B, 2), dtype=torch.bfloat16, device=dev)
+        wsp = ft2.make_workspace(B, device=dev)
+
+        def sweeps():
+            for c in range(2):
+                for y in outs[c]:
+                    ft2.bounds_from_prefill(y, bb, wsp, seq_offsets=so, num_seqs=B, correct_nonfinite=True)
+
+        t_b = gtime(sweeps) / 2 * L
+        pbytes = sum(B * T * N * 2 for _, N, _ in crit) * L
+        del outs
+        torch.cuda.empty_cache()
+        out[name] = {
+            "protected_layers": len(crit) * L,
+            "decode_step_us": {"fused_check": round(t_f, 1), "cublas": round(t_c, 1),
+                               "cublas_plus_protect": round(t_cp, 1)},
+            "fused_vs_cublas_pct": round(100.0 * (t_f / t_c - 1.0), 2),
+            "fused_hbm_frac": round(wbytes / (t_f * 1e-6) / 1e9 / hbm_peak, 3),
+            "prefill_bounds_us": round(t_b, 1), "prefill_bounds_GBps": round(pbytes / (t_b * 1e-6) / 1e9, 1),
+        }
+    return out
 
 
 def c4_tp_bounds(args, dev, rank, world, B=32, T=128, blocks=40, R=20):
