@@ -292,6 +292,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             mbar_expect_tx(recv_bar, (uint32_t)((splitk - 1) * (r1 - r0) * BN * 4));
         fence_mbar_init();
         *site_n = 0;
+        if (p.w_static) {
+            // static weights: the first stages' weight tiles are requested right
+            // here, before the TMEM allocation and the CTA barrier, so the DRAM
+            // latency of the first bytes overlaps the prologue (x waits for the
+            // PDL wait below; each stage's barrier expects both boxes)
+            const int pre = nk < STAGES ? nk : STAGES;
+            for (int i = 0; i < pre; ++i) {
+                mbar_expect_tx(&full[i], C::kStageBytes);
+                tma_load_2d(SWAP ? &map_a : &map_b, &full[i], tiles + i * C::kStageBytes + (SWAP ? 0 : C::kABytes),
+                            (kb0 + i) * kBlockK, SWAP ? tileA * kBlockA : tileB * BN);
+            }
+        }
     }
     if (warp == 1) tmem_alloc(tmem_base_sh, C::kTmemCols);
     tc_fence_before();
@@ -313,12 +325,15 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             const int x_off = SWAP ? C::kABytes : 0;
             FT2_TRACE(1);
             const int pre = nk < STAGES ? nk : STAGES;
-            if (!p.w_static) griddep_wait();
-            for (int i = 0; i < pre; ++i) {
-                mbar_expect_tx(&full[i], C::kStageBytes);
-                tma_load_2d(mw, &full[i], tiles + i * C::kStageBytes + w_off, (kb0 + i) * kBlockK, w_row);
+            if (!p.w_static) {   // (static weights were requested in the prologue)
+                griddep_wait();
+                for (int i = 0; i < pre; ++i) {
+                    mbar_expect_tx(&full[i], C::kStageBytes);
+                    tma_load_2d(mw, &full[i], tiles + i * C::kStageBytes + w_off, (kb0 + i) * kBlockK, w_row);
+                }
+            } else {
+                griddep_wait();
             }
-            if (p.w_static) griddep_wait();
             FT2_TRACE(2);
             for (int i = 0; i < pre; ++i)
                 tma_load_2d(mx, &full[i], tiles + i * C::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row);
