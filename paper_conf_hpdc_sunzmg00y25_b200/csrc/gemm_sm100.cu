@@ -669,9 +669,13 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     // clusters above the portable size 8 only pay off when few (<= 16) of
     // them are needed (measured: 16 tiles x 12 beats x 8; 32 tiles x 9 loses to x 8)
     const int sk_cap = tiles <= 16 ? kMaxSplitPlanned : 8;
+    // between 33 and 64 tiles the in-situ optimum sits lower (measured at
+    // N = 6144: 240 CTAs 15.7 us, 288 CTAs 20.4 us, cuBLAS 13.7 us;
+    // profiles/r1c_splitk_mid.txt), so those shapes cap the grid at 240
+    const int cta_cap = (tiles > 32 && tiles <= 64) ? 240 : 2 * sms;
     if (g.swap) {
         for (int sk = 2; sk <= sk_cap; ++sk) {
-            if (tiles * sk > 2 * sms || g.nkb < 4 * sk) break;
+            if (tiles * sk > cta_cap || g.nkb < 4 * sk) break;
             if (max_clusters_bn(g.bn, sk) < 1) break;
             best = sk;
         }

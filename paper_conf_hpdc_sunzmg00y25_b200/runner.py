@@ -165,7 +165,7 @@ class Runner:
     """Batched greedy generation with FT2 on the critical layers."""
 
     def __init__(self, cfg: ModelConfig, batch: int, prompt_len: int, gen_len: int, seed: int = 1,
-                 device="cuda", scale: float = 2.0, coverage: str = "ft2", fuse_proj: bool = False):
+                 device="cuda", scale: float = 2.0, coverage: str = "ft2", fuse_proj: bool | None = None):
         self.cfg = cfg
         self.B = batch
         self.T = prompt_len
@@ -191,10 +191,12 @@ class Runner:
         # helps the unprotected baseline more than FT2 (measured 8.4 % FT2
         # overhead fused vs 2.8 % unfused).  Fault campaigns address sites per
         # linear layer and need fuse_proj=False.
+        import os
+        if fuse_proj is None:   # FT2_FUSE_PROJ=1 flips the default (experiments)
+            fuse_proj = os.environ.get("FT2_FUSE_PROJ", "0") == "1"
         self.fuse_proj = fuse_proj
         # critical layers whose decode check runs as cuBLAS + ft2_protect even
         # in "fused" mode (FT2_STANDALONE_LAYERS="v_proj,out_proj", experiments)
-        import os
         self.standalone_layers = set(filter(None, os.environ.get("FT2_STANDALONE_LAYERS", "").split(",")))
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
