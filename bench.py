@@ -485,8 +485,13 @@ def coverage_costs(cfg, B, T, G, dev, prompt, stream, runner_ft2, ms_off_ft2, ro
         return a, b
 
     out = {}
-    for cov in ("ft2", "maximals", "globalclipper", "all"):
-        r = runner_ft2 if cov == "ft2" else Runner(cfg, B, T, G, seed=1, device=dev, coverage=cov)
+    for cov in ("ft2", "maximals", "globalclipper", "all", "ft2+fused_qkv"):
+        if cov == "ft2":
+            r = runner_ft2
+        elif cov == "ft2+fused_qkv":   # q/k/v as one GEMM in every mode; the check on the V column slice
+            r = Runner(cfg, B, T, G, seed=1, device=dev, coverage="ft2", fuse_proj=True)
+        else:
+            r = Runner(cfg, B, T, G, seed=1, device=dev, coverage=cov)
         for m in ("fused", "off"):
             for _ in range(4):
                 r.generate(prompt, m)
@@ -498,11 +503,13 @@ def coverage_costs(cfg, B, T, G, dev, prompt, stream, runner_ft2, ms_off_ft2, ro
             for m, (a, b) in evs:
                 samples[m].append(a.elapsed_time(b))
         f, o = statistics.median(samples["fused"]), statistics.median(samples["off"])
-        out[cov] = {"protected_layers": r.n_crit, "overhead_pct": 100.0 * (1 - o / f), "ms_fused": f, "ms_off": o}
+        out[cov] = {"protected_layers": r.n_crit, "overhead_pct": 100.0 * (1 - o / f), "ms_fused": f, "ms_off": o,
+                    "tokens_per_s_fused": B * G / (f / 1e3), "tokens_per_s_off": B * G / (o / 1e3)}
         if r is not runner_ft2:
             del r
             torch.cuda.empty_cache()
-    out["note"] = "Table 1 coverages (MaxiMals: out_proj+fc2; Global Clipper: v_proj+out_proj; all linear layers)"
+    out["note"] = ("Table 1 coverages (MaxiMals: out_proj+fc2; Global Clipper: v_proj+out_proj; all linear layers); "
+                   "ft2+fused_qkv: FT2's layers with q/k/v fused into one GEMM in both modes")
     return out
 
 
