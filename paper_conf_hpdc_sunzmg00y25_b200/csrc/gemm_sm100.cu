@@ -654,6 +654,8 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     GemmPlan g;
     g.swap = M <= swap_max_m() ? 1 : 0;
     g.bn = g.swap ? (M <= 16 ? 16 : (M <= 32 ? 32 : (M <= 64 ? 64 : 128))) : 128;
+    static const int bn_env = env_int("FT2_GEMM_BN", 0);   // experiment: force the token-tile width
+    if (g.swap && (bn_env == 16 || bn_env == 32 || bn_env == 64)) g.bn = bn_env;
     const int rowsA = g.swap ? N : M, rowsB = g.swap ? M : N;
     g.tilesA = (rowsA + kBlockA - 1) / kBlockA;
     g.tilesB = (rowsB + g.bn - 1) / g.bn;
