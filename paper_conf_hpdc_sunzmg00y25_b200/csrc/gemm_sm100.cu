@@ -667,6 +667,19 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     // sweep_splitk.sh, profiles/): the best split is the largest one with
     // tiles * splitk <= 2 * SMs (two ~105 KB CTAs fit an SM), >= 4 k-blocks of
     // 64 per CTA, and a cluster of at most 8 CTAs (12 when <= 16 tiles).
+    // v/out_proj-sized decode layers (<= 16 feature tiles, K <= 2048) at
+    // 17..32 tokens: two 16-token tiles with a 4-way split give 32 clusters of
+    // 4, all resident at once, instead of 16 clusters of 8 of which only 15
+    // fit (the 16th started ~1.2 us late): in situ 12.77 -> 12.25 us per
+    // [layer_norm -> 2048x2048 linear] (profiles/r1c_bn16.txt)
+    if (g.swap && g.bn == 32 && g.tilesA <= 16 && g.nkb >= 24 && g.nkb <= 32 && bn_env == 0 &&
+        getenv("FT2_GEMM_SPLITK") == nullptr && max_clusters_bn(16, 4) >= 2 * g.tilesA) {
+        g.bn = 16;
+        g.tilesB = (rowsB + 15) / 16;
+        g.splitk = 4;
+        g.deep = 0;
+        return g;
+    }
     int best = 1;
     // clusters above the portable size 8 only pay off when few (<= 16) of
     // them are needed (measured: 16 tiles x 12 beats x 8; 32 tiles x 9 loses to x 8)

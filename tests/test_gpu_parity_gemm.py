@@ -67,7 +67,8 @@ GEMM_SHAPES = [
     (1, 768, 768),        # C1: OPT-125m-shaped out_proj, one token
     (16, 768, 768),       # C1 prefill
     (1, 2048, 2048),      # C2 v/out, B = 1
-    (32, 2048, 2048),     # C2 v/out, B = 32
+    (32, 2048, 2048),     # C2 v/out, B = 32 (two 16-token tiles, 4-way split)
+    (24, 2048, 1792),     # ragged second 16-token tile
     (32, 2048, 8192),     # C2 fc2
     (32, 4096, 4096),     # C3 v / o
     (32, 11008, 4096),    # C3 up
@@ -97,8 +98,8 @@ def test_gemm_plain_vs_cublas(ft2, M, N, K):
     assert float(d.max()) <= 1e-2 * max(1.0, float(ref.double().abs().max()))
 
 
-@pytest.mark.parametrize("M,N,K", [(1, 768, 768), (32, 2048, 2048), (32, 4096, 11008), (17, 1000, 136),
-                                   (200, 384, 512)])
+@pytest.mark.parametrize("M,N,K", [(1, 768, 768), (32, 2048, 2048), (24, 2048, 1792), (32, 4096, 11008),
+                                   (17, 1000, 136), (200, 384, 512)])
 def test_gemm_check_epilogue_bit_exact(ft2, M, N, K):
     x, w, b = _operands(M, N, K, seed=7)
     S = M if M > 1 else 1
