@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--prompt", type=int, default=128)
     ap.add_argument("--gen", type=int, default=60)
     ap.add_argument("--no-extras", action="store_true", help="skip the kernel roofline / cpu baseline legs")
-    ap.add_argument("--leg", default=None, choices=["c3", "c4", "c5", "models"],
+    ap.add_argument("--leg", default=None, choices=["c1", "c3", "c4", "c5", "models"],
                     help="run one measurement leg alone and print its JSON (c3: Llama-2-7B decode GEMMs; "
                          "c4: Llama-2-13B tensor-parallel bounds over the ranks (NCCL MAX all-reduce); "
                          "c5: SDC fault-injection campaign, trials sharded over ranks)")
@@ -279,6 +279,10 @@ def main():
         if rank == 0:
             print(json.dumps({"leg": "c3", **c3_decode_gemm(dev, ft2, load_peaks())}), flush=True)
         return 0
+    if args.leg == "c1":
+        if rank == 0:
+            print(json.dumps({"leg": "c1", **c1_leg(dev, ft2)}), flush=True)
+        return 0
     if args.leg == "models":
         if rank == 0:
             print(json.dumps({"leg": "models", **paper_models_leg(dev, ft2, load_peaks())}), flush=True)
@@ -457,6 +461,7 @@ def main():
     if not args.no_extras:
         res["coverage_overhead_pct"] = coverage_costs(cfg, B, T, G, dev, prompt, stream, runner, ms_off)
     if rank == 0 and world == 1 and not args.no_extras:
+        res["c1_single_layer"] = c1_leg(dev, ft2)
         cb = oracle_sample(args.model, B, T, G)
         res["cpu_baseline"] = {"value": cb["tokens_per_s"], "unit": "tokens/s", "cores": cb["cores"],
                                "kind": "oracle", "sample": cb["sample"]}
@@ -641,6 +646,78 @@ PAPER_MODELS = {
     "vicuna-7b": ("llama", 4096, 11008, 32, 4096), "qwen2-7b": ("llama", 3584, 18944, 28, 512),
     "qwen2-1.5b": ("llama", 1536, 8960, 28, 256),
 }
+
+
+def c1_leg(dev, ft2, R=20):
+    """configs[0]: one critical layer (OPT-125m-shaped out_proj, 768x768 +
+    bias), 16-token prefill -> first-token bounds (x2, correction), then 32
+    decode steps with one seeded 1-bit fault per step (step_policy = 1) ->
+    fused GEMM + inject + check.  GPU: the whole 33-launch request in a CUDA
+    graph (us per request and per decode step).  Beside it, the CPU oracle's
+    same pipeline (fp64 linear, R2-R7), single thread, seconds -- the
+    bench's cpu_baseline leg (parity is tests/test_gpu_c1_pipeline.py)."""
+    import torch
+
+    import ft2_synth
+
+    H, T, S = 768, 16, 32
+    w = ft2_synth.gen_bf16_torch((H, H), 1, 1, scale_log2=ft2_synth.weight_scale_log2(H), device=dev)
+    b = ft2_synth.gen_bf16_torch((H,), 3, 1, device=dev)
+    xp = ft2_synth.gen_bf16_torch((T, H), 2, 2, device=dev)
+    xs = torch.stack([ft2_synth.gen_bf16_torch((1, H), 100 + t, 2, device=dev) for t in range(1, S + 1)])
+    yp = torch.empty((T, H), dtype=torch.bfloat16, device=dev)
+    ys = torch.empty((S, 1, H), dtype=torch.bfloat16, device=dev)
+    bnd = torch.zeros((1, 2), dtype=torch.bfloat16, device=dev)
+    ws = ft2.make_workspace(1, device=dev)
+    sites = ft2.make_fault_sites(42, 0, S, 0, [H], S, T, step_policy=1, device=dev)
+    base = torch.zeros(S, dtype=torch.int32, device=dev)
+    cnt = torch.zeros(1, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def request():
+        ft2.protect_fused_gemm(xp, w, yp, bias=b, mode=0)            # prefill layer (16 tokens, swap-AB)
+        ft2.bounds_from_prefill(yp, bnd, ws, correct_nonfinite=True)  # first-token bounds
+        for t in range(1, S + 1):
+            ft2.protect_fused_gemm(xs[t - 1], w, ys[t - 1], bias=b, mode=1, bounds=bnd, num_seqs=1,
+                                   corrected_count=cnt, sites=sites, cur_layer=0, cur_step=t, base_row=base)
+
+    request()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        request()
+    for _ in range(3):
+        g.replay()
+    torch.cuda.synchronize()
+    a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for _ in range(R):
+        g.replay()
+    b_.record(stream)
+    torch.cuda.synchronize()
+    us = 1000.0 * a.elapsed_time(b_) / R
+    out = {"workload": "configs[0]: 768x768 critical layer, 16-token prefill, 32 decode steps, 1-bit fault per step",
+           "gpu_us_per_request": us, "gpu_us_per_decode_step": us / (S + 1), "launches_per_request": S + 2}
+    try:
+        import numpy as np
+
+        import oracle
+        wn, bn_ = (v.cpu().view(torch.int16).numpy().view(np.uint16) for v in (w, b))
+        xpn = xp.cpu().view(torch.int16).numpy().view(np.uint16)
+        xsn = xs.cpu().view(torch.int16).numpy().view(np.uint16)
+        sn = oracle.make_sites(42, 0, S, oracle.FAULT_1BIT, [H], n_steps=S, prompt_len=T, step_policy=1)
+        t0 = time.perf_counter()
+        _, ypn = oracle.linear_f64(xpn, wn, bn_)
+        rb, _, _ = oracle.bounds(ypn, correct_nonfinite=True)
+        for t in range(1, S + 1):
+            _, y = oracle.linear_f64(xsn[t - 1], wn, bn_)
+            oracle.inject(y, sn, 0, t, base_row=np.zeros(S, np.int32))
+            oracle.protect(y, rb)
+        out["cpu_baseline"] = {"value": time.perf_counter() - t0, "unit": "s per request", "cores": 1,
+                               "kind": "oracle", "sample": "the whole C1 request"}
+    except Exception as e:   # the oracle is test infrastructure; its absence must not break the GPU leg
+        out["cpu_baseline"] = {"unavailable": str(e)}
+    return out
 
 
 def paper_models_leg(dev, ft2, peaks, B=32, T=128, nb=4, R=5):
