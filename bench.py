@@ -268,7 +268,10 @@ def main():
     import torch.distributed as dist
 
     if world > 1:
-        dist.init_process_group("nccl")
+        # NCCL over NVLink; FT2_BENCH_BACKEND=gloo lets a multi-rank smoke run
+        # share one GPU (ranks are mapped onto the visible devices round-robin)
+        dist.init_process_group(os.environ.get("FT2_BENCH_BACKEND", "nccl"))
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
 
@@ -1010,7 +1013,7 @@ def c5_campaign(args, dev, rank, world, model="llama-2-7b", B=256, T=16, S=32):
                       "parallelism": f"trial ranges sharded over {world} rank(s)"},
            "models": {}}
     tot_ms, tot_trials = 0.0, 0
-    clk = ClockSampler(int(os.environ.get("LOCAL_RANK", "0")))
+    clk = ClockSampler(torch.cuda.current_device())
     clk.start()
     for fm, name in campaign.MODEL_NAMES.items():
         t0, t1 = campaign.trial_range(args.trials, world, rank)
