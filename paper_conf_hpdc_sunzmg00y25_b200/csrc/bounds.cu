@@ -17,6 +17,7 @@
 // its own vectors in a slow exact path.  In the common all-finite case the
 // kernel moves 2 bytes/element and does no extra work.
 #include <cuda_runtime.h>
+#include <stdlib.h>
 
 #include "ft2_device.cuh"
 #include "ft2_internal.h"
@@ -211,6 +212,8 @@ cudaError_t launch_bounds(const BoundsArgs& a, cudaStream_t st, int* n_launch) {
     const uint32_t per_iter = kThreads * (one_sweep ? 8 : 4);
     uint32_t want = (p.total_vec + per_iter - 1) / per_iter;  // one sweep per thread if possible
     uint32_t grid = want < 1 ? 1 : (want > max_grid ? max_grid : want);
+    static const uint32_t grid_env = [] { const char* e = getenv("FT2_BOUNDS_CTAS"); return e ? (uint32_t)atoi(e) : 0u; }();
+    if (grid_env > 0 && grid_env < grid) grid = grid_env;   // experiment: fewer, longer CTAs
     p.chunk = (p.total_vec + grid - 1) / grid;
     grid = (p.total_vec + p.chunk - 1) / p.chunk;
     if (grid < 1) grid = 1;
