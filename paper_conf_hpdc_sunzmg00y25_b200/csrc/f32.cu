@@ -326,16 +326,20 @@ __global__ void inject32_kernel(uint32_t* y, int64_t rows, int64_t n, int64_t ld
     y[row * ld + s.col] ^= s.xor_mask;
 }
 
-int g_grid32 = 0;
+// One full wave of resident CTAs per kernel: the two sweeps differ in register
+// count (protect32 holds 4 vectors + their addresses), so each grid is sized
+// from its own occupancy -- sizing protect32 from bounds32's 6 CTAs/SM left a
+// 20% second wave (measured 84% of HBM peak).
+int g_grid32[2] = {0, 0};
 
-int max_grid32() {
-    if (g_grid32 == 0) {
+template <typename K>
+int max_grid32(int which, K kernel) {
+    if (g_grid32[which] == 0) {
         int b = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bounds32_kernel<false>, kThreads32, 0) != cudaSuccess)
-            b = 1;
-        g_grid32 = num_sms() * (b > 0 ? b : 1);
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kThreads32, 0) != cudaSuccess) b = 1;
+        g_grid32[which] = num_sms() * (b > 0 ? b : 1);
     }
-    return g_grid32;
+    return g_grid32[which];
 }
 
 }  // namespace
@@ -358,7 +362,7 @@ cudaError_t launch_bounds32(const BoundsArgs& a, cudaStream_t st, int* n_launch)
     p.nonfinite_out = a.nonfinite_out;
     p.nv_out = a.nv_out;
     p.ws = a.ws;
-    const uint32_t per = kThreads32 * 4, mg = (uint32_t)max_grid32();
+    const uint32_t per = kThreads32 * 4, mg = (uint32_t)max_grid32(0, bounds32_kernel<false>);
     uint32_t grid = (p.total_vec + per - 1) / per;
     grid = grid < 1 ? 1 : (grid > mg ? mg : grid);
     p.chunk = (p.total_vec + grid - 1) / grid;
@@ -389,7 +393,7 @@ cudaError_t launch_protect32(const ProtectArgs& a, cudaStream_t st, int* n_launc
     p.row_mode = a.row_to_seq ? 0 : (a.S == 1 ? 2 : 1);
     p.bounds = reinterpret_cast<const uint32_t*>(a.bounds);
     p.counts = a.counts;
-    const uint32_t per = kThreads32 * 4, mg = (uint32_t)max_grid32();
+    const uint32_t per = kThreads32 * 4, mg = (uint32_t)max_grid32(1, protect32_kernel);
     uint32_t grid = (p.total_vec + per - 1) / per;
     grid = grid < 1 ? 1 : (grid > mg ? mg : grid);
     protect32_kernel<<<grid, kThreads32, 0, st>>>(p);
