@@ -113,7 +113,9 @@ def test_bounds32_patch_list_overflow(ft2):
     assert np.array_equal(gb, rb) and np.array_equal(gnf, rnf) and np.array_equal(gy, ref)
 
 
-@pytest.mark.parametrize("rows,n", [(1, 4), (3, 20), (32, 2048), (33, 11008), (512, 4100)])
+# (1500, 4100): 6.15M elements, more than two waves of the 740-CTA grid
+# (4 vectors x 4 values per thread per pass) plus a ragged tail
+@pytest.mark.parametrize("rows,n", [(1, 4), (3, 20), (32, 2048), (33, 11008), (512, 4100), (1500, 4100)])
 @pytest.mark.parametrize("mapping", ["single", "per_row", "array"])
 def test_protect32_bit_exact(ft2, rows, n, mapping):
     y = _tensor32(rows, n, seed=rows * 3 + n)

@@ -40,8 +40,10 @@ def _rand_bounds(S, seed):
 
 
 # ----------------------------------------------------------------- protect --
+# (1600, 8200): 13.1M elements, more than two full waves of the grid-stride
+# loop (148 SMs x 5 CTAs x 256 threads x 4 vectors x 8 elements) plus a ragged tail
 PROTECT_SHAPES = [(1, 8), (1, 768), (3, 24), (17, 40), (7, 1000), (32, 2048), (32, 11008), (129, 4096),
-                  (512, 4104)]
+                  (512, 4104), (1600, 8200)]
 
 
 @pytest.mark.parametrize("rows,n", PROTECT_SHAPES)
