@@ -338,6 +338,23 @@ uint64_t ft2_launch_count(void);
 /* Library version string ("ft2-b200 <semver> sm_100a"). */
 const char* ft2_version(void);
 
+/* ---- Host-model helper (NOT part of the FT2 method; PAPER.md L147-151 put
+ * the norms outside the protected linear layers).  The decoder block's norm,
+ * y[r, :] = (x[r, :] - mean) * rsqrt(var + eps) * w + b   (rms == 0, LayerNorm)
+ * y[r, :] = x[r, :] * rsqrt(mean(x^2) + eps) * w          (rms != 0, RMSNorm; b ignored)
+ * over rows x n row-major device tensors (leading dims ldx / ldy elements),
+ * dtype FT2_BF16 or FT2_FP16, fp32 statistics, round-to-nearest-even output.
+ * b may be NULL.  The kernel issues griddepcontrol.launch_dependents on
+ * entry so a following PDL launch (ft2_protect_fused_gemm) overlaps its
+ * prologue with the norm; it is not counted by ft2_launch_count.
+ * Errors: NULL x/w/y, rows < 0, n <= 0, eps < 0 or NaN -> FT2_ERR_INVALID_ARG;
+ * n % 8 != 0, n > 8192, other dtypes -> FT2_ERR_UNSUPPORTED; ld < n, ld % 8,
+ * pointers not 16-byte aligned -> FT2_ERR_MISALIGNED; launch failure ->
+ * FT2_ERR_CUDA.  rows == 0: FT2_OK, no launch (checked before the NULL
+ * checks).  Caller owns every buffer. */
+ft2_status ft2_host_norm(const void* x, int64_t ldx, const void* w, const void* b, void* y, int64_t ldy,
+                         int64_t rows, int32_t n, float eps, int rms, int dtype, void* stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -207,3 +207,12 @@ def ipc_open_handle(handle: bytes) -> int:
 
 def ipc_close(base: int):
     check("ft2_ipc_close", load().ft2_ipc_close(ctypes.c_void_p(base)))
+
+
+def host_norm(x, w, y, bias=None, eps=1e-5, rms=False, stream=None):
+    """Host-model LayerNorm / RMSNorm over the last dim of 2-D x into y
+    (include/ft2.h ft2_host_norm; not part of the FT2 method)."""
+    n = x.shape[-1]
+    check("ft2_host_norm", load().ft2_host_norm(_ptr(x), x.stride(0), _ptr(w), _ptr(bias), _ptr(y), y.stride(0),
+                                                x.shape[0], n, float(eps), int(rms), _dtype_of(x), _stream(stream)))
+    return y

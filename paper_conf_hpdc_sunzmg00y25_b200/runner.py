@@ -198,6 +198,10 @@ class Runner:
         # critical layers whose decode check runs as cuBLAS + ft2_protect even
         # in "fused" mode (FT2_STANDALONE_LAYERS="v_proj,out_proj", experiments)
         self.standalone_layers = set(filter(None, os.environ.get("FT2_STANDALONE_LAYERS", "").split(",")))
+        # decoder norms through libft2's host-model norm kernel (it triggers
+        # PDL dependents on entry, so the v_proj GEMM's prologue overlaps it);
+        # FT2_HOST_NORM=0 keeps torch's norm kernels (experiments)
+        self.host_norm = os.environ.get("FT2_HOST_NORM", "1") == "1"
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
@@ -234,6 +238,15 @@ class Runner:
 
     # ------------------------------------------------------------ helpers
     def _norm(self, x, w, b):
+        n = x.shape[-1]
+        if self.host_norm and x.is_cuda and n % 8 == 0 and n <= 8192:
+            x2 = x.reshape(-1, n)
+            if x2.stride(-1) != 1:
+                x2 = x2.contiguous()
+            y = torch.empty((x2.shape[0], n), dtype=x.dtype, device=x.device)
+            F2.host_norm(x2, w, y, bias=b if self.cfg.arch == "opt" else None,
+                         eps=1e-5 if self.cfg.arch == "opt" else 1e-6, rms=self.cfg.arch != "opt")
+            return y.view(*x.shape[:-1], n)
         if self.cfg.arch == "opt":
             return F.layer_norm(x, (x.shape[-1],), w, b, 1e-5)
         return F.rms_norm(x, (x.shape[-1],), w, 1e-6)
