@@ -345,8 +345,9 @@ const char* ft2_version(void);
  * over rows x n row-major device tensors (leading dims ldx / ldy elements),
  * dtype FT2_BF16 or FT2_FP16, fp32 statistics, round-to-nearest-even output.
  * b may be NULL.  The kernel issues griddepcontrol.launch_dependents on
- * entry so a following PDL launch (ft2_protect_fused_gemm) overlaps its
- * prologue with the norm; it is not counted by ft2_launch_count.
+ * entry when rows <= the SM count (else after each CTA's last store) so a
+ * following PDL launch (ft2_protect_fused_gemm) overlaps its prologue with
+ * the norm; it is not counted by ft2_launch_count.
  * Errors: NULL x/w/y, rows < 0, n <= 0, eps < 0 or NaN -> FT2_ERR_INVALID_ARG;
  * n % 8 != 0, n > 8192, other dtypes -> FT2_ERR_UNSUPPORTED; ld < n, ld % 8,
  * pointers not 16-byte aligned -> FT2_ERR_MISALIGNED; launch failure ->
@@ -354,6 +355,21 @@ const char* ft2_version(void);
  * checks).  Caller owns every buffer. */
 ft2_status ft2_host_norm(const void* x, int64_t ldx, const void* w, const void* b, void* y, int64_t ldy,
                          int64_t rows, int32_t n, float eps, int rms, int dtype, void* stream);
+
+/* ---- Host-model helper (NOT part of the FT2 method): the MLP activation
+ * feeding the critical fc2 / down_proj layer, elementwise over rows x n
+ * row-major device tensors (leading dims in elements):
+ *   act == 0: y = relu(a)            (NaN propagates; b ignored, may be NULL)
+ *   act == 1: y = round(round(silu(a)) * b), silu(a) = a / (1 + exp(-a)) in fp32
+ * dtype FT2_BF16 / FT2_FP16, round-to-nearest-even; y may alias a.  Issues
+ * griddepcontrol.launch_dependents as ft2_host_norm does; not counted
+ * by ft2_launch_count.  Errors: rows < 0, n <= 0, act not 0/1, NULL a / y,
+ * act == 1 with NULL b -> FT2_ERR_INVALID_ARG; other dtypes, rows * n / 8 >=
+ * 2^31 -> FT2_ERR_UNSUPPORTED; n % 8, ld < n, ld % 8, pointers not 16-byte
+ * aligned -> FT2_ERR_MISALIGNED; launch failure -> FT2_ERR_CUDA.  rows == 0:
+ * FT2_OK, no launch. */
+ft2_status ft2_host_act(const void* a, int64_t lda, const void* b, int64_t ldb, void* y, int64_t ldy, int64_t rows,
+                        int32_t n, int act, int dtype, void* stream);
 
 #ifdef __cplusplus
 }

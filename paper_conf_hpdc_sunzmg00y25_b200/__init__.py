@@ -11,8 +11,8 @@ _load()
 from . import ft2  # noqa: E402,F401
 from .ft2 import (allreduce_protect, bounds_finalize, bounds_from_prefill, gemm_workspace_bytes,  # noqa: E402,F401
                   inject_faults, launch_count, make_fault_sites, make_workspace, prefill_fused_gemm, protect,
-                  protect_fused_gemm, version, workspace_bytes, host_norm)
+                  protect_fused_gemm, version, workspace_bytes, host_norm, host_act)
 
 __all__ = ["bounds_from_prefill", "bounds_finalize", "protect", "protect_fused_gemm", "prefill_fused_gemm",
            "make_fault_sites", "inject_faults", "allreduce_protect", "make_workspace", "workspace_bytes",
-           "gemm_workspace_bytes", "launch_count", "version", "host_norm"]
+           "gemm_workspace_bytes", "launch_count", "version", "host_norm", "host_act"]

@@ -42,7 +42,7 @@ EXPORTS = [
     "ft2_workspace_bytes", "ft2_bounds_from_prefill", "ft2_bounds_finalize", "ft2_protect",
     "ft2_gemm_workspace_bytes", "ft2_protect_fused_gemm", "ft2_prefill_fused_gemm", "ft2_make_fault_sites",
     "ft2_inject_faults", "ft2_allreduce_protect", "ft2_ipc_get_handle", "ft2_ipc_open_handle", "ft2_ipc_close",
-    "ft2_status_string", "ft2_launch_count", "ft2_version", "ft2_host_norm",
+    "ft2_status_string", "ft2_launch_count", "ft2_version", "ft2_host_norm", "ft2_host_act",
 ]
 
 _lib = None
@@ -80,6 +80,7 @@ def load(path: str = LIB):
         "ft2_launch_count": (ctypes.c_uint64, []),
         "ft2_version": (ctypes.c_char_p, []),
         "ft2_host_norm": (st, [P, i64, P, P, P, i64, i64, i32, f32, ctypes.c_int, ctypes.c_int, P]),
+        "ft2_host_act": (st, [P, i64, P, i64, P, i64, i64, i32, ctypes.c_int, ctypes.c_int, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

@@ -216,3 +216,13 @@ def host_norm(x, w, y, bias=None, eps=1e-5, rms=False, stream=None):
     check("ft2_host_norm", load().ft2_host_norm(_ptr(x), x.stride(0), _ptr(w), _ptr(bias), _ptr(y), y.stride(0),
                                                 x.shape[0], n, float(eps), int(rms), _dtype_of(x), _stream(stream)))
     return y
+
+
+def host_act(a, y, b=None, act="relu", stream=None):
+    """Host-model MLP activation into y: relu(a), or silu(a) * b with
+    act="silu_mul" (include/ft2.h ft2_host_act; not part of the FT2 method)."""
+    code = {"relu": 0, "silu_mul": 1}[act]
+    check("ft2_host_act", load().ft2_host_act(_ptr(a), a.stride(0), _ptr(b), b.stride(0) if b is not None else 0,
+                                              _ptr(y), y.stride(0), a.shape[0], a.shape[-1], code, _dtype_of(a),
+                                              _stream(stream)))
+    return y

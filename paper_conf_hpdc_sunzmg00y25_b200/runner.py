@@ -198,10 +198,12 @@ class Runner:
         # critical layers whose decode check runs as cuBLAS + ft2_protect even
         # in "fused" mode (FT2_STANDALONE_LAYERS="v_proj,out_proj", experiments)
         self.standalone_layers = set(filter(None, os.environ.get("FT2_STANDALONE_LAYERS", "").split(",")))
-        # decoder norms through libft2's host-model norm kernel (it triggers
-        # PDL dependents on entry, so the v_proj GEMM's prologue overlaps it);
-        # FT2_HOST_NORM=0 keeps torch's norm kernels (experiments)
+        # decoder norms and MLP activations through libft2's host-model
+        # kernels (they trigger PDL dependents on entry, so the v_proj / fc2 /
+        # down_proj GEMM prologue overlaps them); FT2_HOST_NORM=0 keeps
+        # torch's kernels (experiments)
         self.host_norm = os.environ.get("FT2_HOST_NORM", "1") == "1"
+        self.host_act = self.host_norm and os.environ.get("FT2_HOST_ACT", "1") == "1"
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
@@ -250,6 +252,20 @@ class Runner:
         if self.cfg.arch == "opt":
             return F.layer_norm(x, (x.shape[-1],), w, b, 1e-5)
         return F.rms_norm(x, (x.shape[-1],), w, 1e-6)
+
+    def _act(self, a, b=None):
+        """relu(a) (OPT) or silu(a) * b (Llama) ahead of the critical fc2 /
+        down_proj layer; libft2's host kernel triggers PDL dependents."""
+        n = a.shape[-1]
+        # decode-sized tensors only: there the launch latency is what PDL
+        # hides; at prefill size (4096 x 8192) torch's unrolled kernel is
+        # faster than this one (measured +0.42 ms per OPT-1.3B prefill)
+        if self.host_act and a.is_cuda and n % 8 == 0 and a.dim() == 2 and a.shape[0] <= 256 and \
+                a.stride(-1) == 1 and \
+                (b is None or (b.dim() == 2 and b.stride(-1) == 1)):
+            y = torch.empty((a.shape[0], n), dtype=a.dtype, device=a.device)
+            return F2.host_act(a, y, b=b, act="relu" if b is None else "silu_mul")
+        return torch.relu(a) if b is None else F.silu(a) * b
 
     def _rope(self, x, pos_idx):
         cos = self.rope_cos[pos_idx].unsqueeze(1)
@@ -417,7 +433,7 @@ class Runner:
         x = x + self._linear(a, blk, o_name, phase, step).view(B, T, -1)
         h = self._norm(x, blk.ln2_w, blk.ln2_b).reshape(-1, cfg.hidden)
         if cfg.arch == "opt":
-            f = torch.relu(self._linear(h, blk, "fc1", phase, step))
+            f = self._act(self._linear(h, blk, "fc1", phase, step))
             y = self._linear(f, blk, "fc2", phase, step)
         else:
             if self._group_ok(blk, "gate_up"):
@@ -425,7 +441,7 @@ class Runner:
             else:
                 g = self._linear(h, blk, "gate_proj", phase, step)
                 u = self._linear(h, blk, "up_proj", phase, step)
-            y = self._linear(F.silu(g) * u, blk, "down_proj", phase, step)
+            y = self._linear(self._act(g, u), blk, "down_proj", phase, step)
         return x + y.view(B, T, -1)
 
     def _embed(self, ids, pos_idx):

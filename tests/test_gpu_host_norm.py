@@ -72,3 +72,49 @@ def test_host_norm_errors(ft2):
         ft2.host_norm(x, x[0], torch.empty_like(x), eps=-1.0)
     e = torch.empty(0, 16, device="cuda", dtype=torch.bfloat16)
     ft2.host_norm(e, x[0], torch.empty_like(e))                # rows == 0: no launch
+
+
+@pytest.mark.parametrize("rows,n", [(1, 8), (32, 8192), (33, 11008), (4096, 2048)])
+@pytest.mark.parametrize("dtype", [torch.bfloat16, torch.float16])
+def test_host_act_relu_bit_exact(ft2, rows, n, dtype):
+    g = torch.Generator(device="cuda").manual_seed(rows + n)
+    a = torch.randn(rows, n, device="cuda", generator=g).to(dtype)
+    a.view(-1)[::997] = float("nan")
+    a.view(-1)[5::1009] = float("-inf")
+    y = torch.empty_like(a)
+    ft2.host_act(a, y)
+    torch.cuda.synchronize()
+    ref = torch.relu(a)
+    assert torch.equal(torch.isnan(y), torch.isnan(ref))      # NaN propagates, as torch.relu
+    m = ~torch.isnan(ref)
+    assert torch.equal(y[m], ref[m])
+    assert not torch.any(y[m].view(torch.int16) < 0)           # no negative (or -0) outputs
+
+
+@pytest.mark.parametrize("rows,n", [(1, 8), (32, 11008), (7, 13824)])
+@pytest.mark.parametrize("dtype", [torch.bfloat16, torch.float16])
+def test_host_act_silu_mul_matches_torch(ft2, rows, n, dtype):
+    g = torch.Generator(device="cuda").manual_seed(rows * 7 + n)
+    gu = (torch.randn(rows, 2 * n, device="cuda", generator=g) * 4).to(dtype)
+    a, b = gu[:, :n], gu[:, n:]                                  # strided views, as the fused gate_up GEMM gives
+    y = torch.empty(rows, n, device="cuda", dtype=dtype)
+    ft2.host_act(a, y, b=b, act="silu_mul")
+    torch.cuda.synchronize()
+    ref = torch.nn.functional.silu(a) * b
+    ulp = 2.0 ** -7 if dtype == torch.bfloat16 else 2.0 ** -10
+    torch.testing.assert_close(y.float(), ref.float(), rtol=2 * ulp, atol=1e-3)
+    # the fp32 formula rounded twice, as torch does: almost all bit-identical
+    assert (y != ref).float().mean().item() < 1e-3
+
+
+def test_host_act_errors(ft2):
+    from paper_conf_hpdc_sunzmg00y25_b200._lib import FT2Error
+    a = torch.randn(4, 16, device="cuda").to(torch.bfloat16)
+    from paper_conf_hpdc_sunzmg00y25_b200._lib import check, load
+    with pytest.raises(FT2Error, match="INVALID_ARG"):   # silu_mul with b NULL
+        check("ft2_host_act", load().ft2_host_act(a.data_ptr(), 16, None, 0, a.data_ptr(), 16, 4, 16, 1, 0, None))
+    with pytest.raises(FT2Error, match="MISALIGNED"):
+        x = torch.randn(4, 12, device="cuda").to(torch.bfloat16)
+        ft2.host_act(x, torch.empty_like(x))
+    e = torch.empty(0, 16, device="cuda", dtype=torch.bfloat16)
+    ft2.host_act(e, torch.empty_like(e))
