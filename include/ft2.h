@@ -27,8 +27,8 @@
  *      non-finite or < 1 scale                       -> FT2_ERR_INVALID_ARG
  *      base pointer not 16-byte aligned, or ld % 8 != 0 (bf16)
  *                                                    -> FT2_ERR_MISALIGNED
- *      dtype other than FT2_BF16, shapes outside the stated limits
- *                                                    -> FT2_ERR_UNSUPPORTED
+ *      a dtype the entry point does not implement (see ft2_dtype), shapes
+ *      outside the stated limits                     -> FT2_ERR_UNSUPPORTED
  *      kernel launch failure (cudaGetLastError)      -> FT2_ERR_CUDA
  *    A zero-size tensor returns FT2_OK without launching.  Faults inside a
  *    kernel surface at the caller's next synchronisation, as with CUDA.
@@ -231,6 +231,30 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
                                   int32_t n_sites, int32_t cur_layer, int32_t cur_step,
                                   const int32_t* base_row, void* workspace, size_t ws_bytes,
                                   void* stream);
+
+/* ft2_protect_fused_gemm plus an L2 prefetch hint for the layer that runs
+ * next (e.g. the next critical layer's weights: linear layers
+ * are 94% of the compute and, at decode, a pure weight stream).  Decode shapes
+ * (M <= 128) only: once a CTA's own operands have landed in shared memory it
+ * issues cp.async.bulk.prefetch.L2 for its 1/grid share of
+ * [l2_prefetch, l2_prefetch + l2_prefetch_bytes), so HBM keeps streaming
+ * through this kernel's epilogue, the kernel boundary and the next kernel's
+ * prologue.  A hint only: results are identical with or without it, nothing
+ * is written, and the bytes are read-only for this kernel.  M > 128 ignores
+ * it.  l2_prefetch == NULL with l2_prefetch_bytes == 0 is
+ * ft2_protect_fused_gemm.
+ * Errors: l2_prefetch_bytes > 0 with a NULL pointer -> FT2_ERR_INVALID_ARG;
+ * pointer not 16-byte aligned or bytes % 16 != 0 -> FT2_ERR_MISALIGNED; else
+ * as ft2_protect_fused_gemm. */
+ft2_status ft2_protect_fused_gemm_ex(const void* x, int64_t ldx, const void* w, int64_t ldw,
+                                     const void* bias, void* y, int64_t ldy, int32_t M, int32_t N,
+                                     int32_t K, ft2_gemm_mode mode, ft2_dtype dtype, int32_t col_begin,
+                                     int32_t col_end, const int32_t* row_to_seq, const void* bounds,
+                                     int32_t num_seqs, uint32_t* corrected_count,
+                                     const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
+                                     int32_t cur_step, const int32_t* base_row, void* workspace,
+                                     size_t ws_bytes, const void* l2_prefetch, size_t l2_prefetch_bytes,
+                                     void* stream);
 
 /* The critical linear layer during first-token generation (prefill) with the
  * first-token bound derivation fused into its GEMM epilogue (SURVEY.md 8(f)

@@ -40,7 +40,7 @@ assert ctypes.sizeof(FaultSite) == 24
 
 EXPORTS = [
     "ft2_workspace_bytes", "ft2_bounds_from_prefill", "ft2_bounds_finalize", "ft2_protect",
-    "ft2_gemm_workspace_bytes", "ft2_protect_fused_gemm", "ft2_prefill_fused_gemm", "ft2_make_fault_sites",
+    "ft2_gemm_workspace_bytes", "ft2_protect_fused_gemm", "ft2_protect_fused_gemm_ex", "ft2_prefill_fused_gemm", "ft2_make_fault_sites",
     "ft2_inject_faults", "ft2_allreduce_protect", "ft2_ipc_get_handle", "ft2_ipc_open_handle", "ft2_ipc_close",
     "ft2_status_string", "ft2_launch_count", "ft2_version", "ft2_host_norm", "ft2_host_act",
 ]
@@ -66,6 +66,9 @@ def load(path: str = LIB):
         "ft2_gemm_workspace_bytes": (ctypes.c_size_t, [i32, i32, i32]),
         "ft2_protect_fused_gemm": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, ctypes.c_int, i32, i32,
                                         P, P, i32, P, P, i32, i32, i32, P, P, ctypes.c_size_t, P]),
+        "ft2_protect_fused_gemm_ex": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, ctypes.c_int, i32,
+                                           i32, P, P, i32, P, P, i32, i32, i32, P, P, ctypes.c_size_t, P,
+                                           ctypes.c_size_t, P]),
         "ft2_prefill_fused_gemm": (st, [P, i64, P, i64, P, P, i64, i32, i32, i32, ctypes.c_int, P, i32, f32, i32,
                                         P, P, P, P, i32, i32, P, P, P, ctypes.c_size_t, P]),
         "ft2_make_fault_sites": (st, [u64, u64, i32, ctypes.c_int, ctypes.c_int, ctypes.POINTER(SiteGeometry),

@@ -155,6 +155,21 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
                                   const ft2_fault_site* sites, int32_t n_sites, int32_t cur_layer,
                                   int32_t cur_step, const int32_t* base_row, void* workspace, size_t ws_bytes,
                                   void* stream) {
+    return ft2_protect_fused_gemm_ex(x, ldx, w, ldw, bias, y, ldy, M, N, K, mode, dtype, col_begin, col_end,
+                                     row_to_seq, bounds, num_seqs, corrected_count, sites, n_sites, cur_layer,
+                                     cur_step, base_row, workspace, ws_bytes, nullptr, 0, stream);
+}
+
+ft2_status ft2_protect_fused_gemm_ex(const void* x, int64_t ldx, const void* w, int64_t ldw, const void* bias,
+                                     void* y, int64_t ldy, int32_t M, int32_t N, int32_t K, ft2_gemm_mode mode,
+                                     ft2_dtype dtype, int32_t col_begin, int32_t col_end,
+                                     const int32_t* row_to_seq, const void* bounds, int32_t num_seqs,
+                                     uint32_t* corrected_count, const ft2_fault_site* sites, int32_t n_sites,
+                                     int32_t cur_layer, int32_t cur_step, const int32_t* base_row,
+                                     void* workspace, size_t ws_bytes, const void* l2_prefetch,
+                                     size_t l2_prefetch_bytes, void* stream) {
+    if (l2_prefetch_bytes > 0 && (l2_prefetch == nullptr)) return FT2_ERR_INVALID_ARG;
+    if (l2_prefetch_bytes > 0 && (!al16(l2_prefetch) || (l2_prefetch_bytes % 16))) return FT2_ERR_MISALIGNED;
     if (M < 0 || N < 0 || K < 0) return FT2_ERR_INVALID_ARG;
     if (dtype != FT2_BF16 && dtype != FT2_FP16) return FT2_ERR_UNSUPPORTED;
     if (M == 0 || N == 0) return FT2_OK;
@@ -204,6 +219,8 @@ ft2_status ft2_protect_fused_gemm(const void* x, int64_t ldx, const void* w, int
     a.ws_bytes = ws_bytes;
     a.w_static = w_static;
     a.dtype = dtype;
+    a.l2_prefetch = l2_prefetch_bytes ? l2_prefetch : nullptr;
+    a.l2_prefetch_bytes = l2_prefetch_bytes;
     int nl = 0;
     cudaError_t e = launch_gemm(a, static_cast<cudaStream_t>(stream), &nl);
     return finish(e, nl);

@@ -173,10 +173,14 @@ __device__ __forceinline__ uint32_t draw_below(uint32_t u, uint32_t n) {
 }
 
 // ------------------------------------------------------------------ loads
+// Streaming 16-byte load that does not allocate in L1.  Deliberately NOT
+// .nc: the protect kernels write back (and the bounds kernel's last CTA
+// patches) the very tensor they stream, and the non-coherent path is only
+// defined for data that is read-only for the kernel's whole lifetime.
 __device__ __forceinline__ uint4 ld_stream(const uint4* p) {
     uint4 r;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
     return r;
 }
 

@@ -71,6 +71,8 @@ struct GemmArgs {
     void* ws; size_t ws_bytes;
     int32_t w_static;
     int32_t dtype;
+    const void* l2_prefetch;     // bytes to pull into L2 once this CTA's own operands have landed
+    size_t l2_prefetch_bytes;    // (the next layer's weights; multiple of 16, 16-byte aligned)
 };
 size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch);

@@ -56,8 +56,10 @@ constexpr int kMaxSplitPlanned = 12;  // largest split the planner picks (16-CTA
 
 #ifdef FT2_GEMM_TRACE
 // Debug builds only (lib/libft2_trace.so): per-CTA timestamps.
-__device__ unsigned long long g_trace[4096 * 16];
-__device__ __forceinline__ void trace(int slot) {
+// 256 CTA rows per launch (GemmK::trace_base = 256 * (launch index mod 128))
+__device__ unsigned long long g_trace[32768 * 16];
+#define FT2_TRACE_ROWS 32768
+__device__ __forceinline__ void trace(int slot, int base) {
     unsigned long long t;
 #ifdef FT2_TRACE_CLOCK
     asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
@@ -65,9 +67,10 @@ __device__ __forceinline__ void trace(int slot) {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
 #endif
     const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-    if (cta < 4096) g_trace[cta * 16 + slot] = t;
+    if (cta < 256 && base + cta < FT2_TRACE_ROWS) g_trace[(base + cta) * 16 + slot] = t;
 }
-#define FT2_TRACE(slot) trace(slot)
+#define FT2_TRACE(slot) trace(slot, p.trace_base)
+static int g_trace_launch = 0;   // host: launches since the last ft2_debug_trace_reset
 #else
 #define FT2_TRACE(slot) ((void)0)
 #endif
@@ -90,6 +93,7 @@ struct GemmK {
     const int32_t* base_row;
     int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
     int32_t trigger;   // issue griddepcontrol.launch_dependents early (FT2_GEMM_TRIGGER, default 1)
+    int32_t w_l2;      // static weights: L2-prefetch the K slice beyond the ring before the PDL wait (FT2_GEMM_W_L2)
     // K split through global memory instead of the cluster (no cluster launch:
     // every CTA starts at once; the last split of a tile to arrive sums the
     // tile's fp32 slots in split order and finishes all 128 rows).  Opt-in
@@ -101,6 +105,10 @@ struct GemmK {
     uint32_t* gcnt;    // [tiles] arrival counters (self-cleaning)
     int32_t rows_per_slot;  // ceil(128 / splitk): rows of one split-K receive slot
     uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
+    int32_t trace_base;     // trace builds only: first g_trace row of this launch
+    const uint8_t* pf;      // L2 prefetch hint (the next layer's weights) and its size
+    uint64_t pf_bytes;
+    int32_t pf_at;          // 0: after this CTA issued its last load; 1: after its last stage landed
 };
 
 // Per-row / per-column epilogue table entry.  Feature side: bias, flags
@@ -303,6 +311,15 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 tma_load_2d(SWAP ? &map_a : &map_b, &full[i], tiles + i * C::kStageBytes + (SWAP ? 0 : C::kABytes),
                             (kb0 + i) * kBlockK, SWAP ? tileA * kBlockA : tileB * BN);
             }
+            // ... and the rest of this CTA's weight slice is pulled into L2
+            // right away (no shared memory needed), so the whole layer
+            // streams from HBM while this kernel still waits for its
+            // activations; the ring's later loads then hit L2
+            if (p.w_l2) {   // at most one more ring's worth (a whole large slice would thrash L2)
+                const int lim = nk < pre + STAGES ? nk : pre + STAGES;
+                for (int i = pre; i < lim; ++i)
+                    tma_prefetch_l2_2d(SWAP ? &map_a : &map_b, (kb0 + i) * kBlockK, SWAP ? tileA * kBlockA : tileB * BN);
+            }
         }
     }
     if (warp == 1) tmem_alloc(tmem_base_sh, C::kTmemCols);
@@ -345,6 +362,23 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 tma_load_2d(mw, &full[s], st + w_off, (kb0 + i) * kBlockK, w_row);
                 tma_load_2d(mx, &full[s], st + x_off, (kb0 + i) * kBlockK, x_row);
             }
+            if (p.pf_bytes) {
+                // L2 prefetch hint: this CTA's 1/grid share of the next
+                // layer's bytes, once its own loads are issued (pf_at 0) or
+                // have landed (pf_at 1), so the prefetch does not compete
+                // with this kernel's critical-path loads
+                if (p.pf_at && nk > 0) {
+                    const int last = nk - 1;
+                    mbar_wait(&full[last % STAGES], (uint32_t)(last / STAGES) & 1u);
+                }
+                const uint32_t ncta = gridDim.x * gridDim.y * gridDim.z;
+                const uint32_t cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+                const uint64_t chunk = ((p.pf_bytes + ncta - 1) / ncta + 255) & ~(uint64_t)255;
+                const uint64_t beg = (uint64_t)cta * chunk;
+                const uint64_t end = beg + chunk < p.pf_bytes ? beg + chunk : p.pf_bytes;
+                for (uint64_t off = beg; off < end; off += 65536)
+                    bulk_prefetch_l2(p.pf + off, (uint32_t)(end - off < 65536 ? end - off : 65536));
+            }
         }
     } else if (warp == 1) {
         if (lane == 0) {
@@ -356,6 +390,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 const int s = i % STAGES;
                 mbar_wait(&full[s], (uint32_t)(i / STAGES) & 1u);
                 if (i == 0) FT2_TRACE(3);
+                if (i == 1) FT2_TRACE(12);
+                if (i == nk - 1) FT2_TRACE(13);
                 tc_fence_after();
                 const uint32_t sa = smem_u32(tiles + s * C::kStageBytes);
                 const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + C::kABytes);
@@ -425,6 +461,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             uint32_t r[32];
             tmem_ld32(taddr, r);
             tmem_wait_ld();
+            if (a == 0) FT2_TRACE(14);
             if (nk == 0) {
 #pragma unroll
                 for (int j = 0; j < 32; ++j) r[j] = 0u;
@@ -448,6 +485,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             uint32_t r[16];
             tmem_ld16(taddr + c0, r);
             tmem_wait_ld();
+            if (a == 0 && c0 == 0) FT2_TRACE(14);
             if (nk == 0) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) r[j] = 0u;
@@ -747,6 +785,7 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
         fprintf(stderr, " occ(bn32)=%d smem=%d avail@2=%zu avail@1=%zu regs=%d static=%zu maxdyn=%d carve=%d smem/SM=%d\n",
                 occ, Cfg<32>::kBytes, avail2, avail1, fa.numRegs, fa.sharedSizeBytes, fa.maxDynamicSharedSizeBytes,
                 fa.preferredShmemCarveout, smem_sm);
+        cudaGetLastError();   // the occupancy probes above may leave an error behind
     }
     return g;
 }
@@ -835,6 +874,13 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.w_static = a.w_static;
     static const int trig = env_int("FT2_GEMM_TRIGGER", 1);
     p.trigger = trig;
+    static const int wl2 = env_int("FT2_GEMM_W_L2", 0);
+    p.w_l2 = wl2;
+    static const int pf_on = env_int("FT2_GEMM_PF", 1);      // experiments: 0 ignores the hint
+    static const int pf_at = env_int("FT2_GEMM_PF_AT", 1);
+    p.pf = pf_on ? static_cast<const uint8_t*>(a.l2_prefetch) : nullptr;
+    p.pf_bytes = p.pf ? (uint64_t)a.l2_prefetch_bytes : 0;
+    p.pf_at = pf_at;
     // K split through global memory (FT2_GEMM_GSPLIT=1; needs the workspace)
     static const int gsplit_env = env_int("FT2_GEMM_GSPLIT", 0);
     p.gsplit = 0;
@@ -848,6 +894,9 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     }
     p.rows_per_slot = (kBlockA + g.splitk - 1) / g.splitk;
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
+#ifdef FT2_GEMM_TRACE
+    p.trace_base = 256 * (g_trace_launch++ % 128);   // graph captures bake one base per captured launch
+#endif
     if (g.deep) {
         if (a.dtype == FT2_FP16) {
             switch (g.bn) {
@@ -897,6 +946,7 @@ extern "C" int ft2_debug_mark(int slot, cudaStream_t st) {
 extern "C" int ft2_debug_marks_read(void* dst) {
     return (int)cudaMemcpyFromSymbol(dst, ft2impl::g_marks, sizeof(ft2impl::g_marks));
 }
+extern "C" void ft2_debug_trace_reset(int launch) { ft2impl::g_trace_launch = launch; }
 extern "C" int ft2_debug_trace_read(void* dst, size_t bytes) {
     if (bytes > sizeof(ft2impl::g_trace)) bytes = sizeof(ft2impl::g_trace);
     return (int)cudaMemcpyFromSymbol(dst, ft2impl::g_trace, bytes);

@@ -88,8 +88,10 @@ def protect(y, bounds, row_to_seq=None, num_seqs=None, corrected_count=None, str
 
 def protect_fused_gemm(x, w, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None, row_to_seq=None, num_seqs=None,
                        corrected_count=None, col_begin=0, col_end=None, sites=None, n_sites=None,
-                       cur_layer=0, cur_step=0, base_row=None, workspace=None, stream=None):
-    """ft2_protect_fused_gemm: y = check(inject(bf16(x @ w.T + bias)))."""
+                       cur_layer=0, cur_step=0, base_row=None, workspace=None, l2_prefetch=None, stream=None):
+    """ft2_protect_fused_gemm: y = check(inject(bf16(x @ w.T + bias))).
+    l2_prefetch: optional tensor (e.g. the next layer's weights) passed to
+    ft2_protect_fused_gemm_ex as an L2 prefetch hint (its whole storage)."""
     M, K = x.shape
     N = w.shape[0]
     if col_end is None:
@@ -99,11 +101,21 @@ def protect_fused_gemm(x, w, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None, row
     if workspace is None:
         workspace = default_gemm_workspace(x.device)
     ws = workspace.numel() * workspace.element_size()
-    st = load().ft2_protect_fused_gemm(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y), y.stride(0),
-                                       M, N, K, int(mode), _dtype_of(x), col_begin, col_end, _ptr(row_to_seq), _ptr(bounds), S,
-                                       _ptr(corrected_count), _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),
-                                       _ptr(workspace), ws, _stream(stream))
-    check("ft2_protect_fused_gemm", st)
+    if l2_prefetch is None:
+        st = load().ft2_protect_fused_gemm(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y),
+                                           y.stride(0), M, N, K, int(mode), _dtype_of(x), col_begin, col_end,
+                                           _ptr(row_to_seq), _ptr(bounds), S, _ptr(corrected_count), _ptr(sites), ns,
+                                           cur_layer, cur_step, _ptr(base_row), _ptr(workspace), ws, _stream(stream))
+        check("ft2_protect_fused_gemm", st)
+        return
+    assert l2_prefetch.is_contiguous(), "l2_prefetch must be a contiguous tensor"
+    pf_bytes = (l2_prefetch.numel() * l2_prefetch.element_size()) & ~15
+    st = load().ft2_protect_fused_gemm_ex(_ptr(x), x.stride(0), _ptr(w), w.stride(0), _ptr(bias), _ptr(y),
+                                          y.stride(0), M, N, K, int(mode), _dtype_of(x), col_begin, col_end,
+                                          _ptr(row_to_seq), _ptr(bounds), S, _ptr(corrected_count), _ptr(sites), ns,
+                                          cur_layer, cur_step, _ptr(base_row), _ptr(workspace), ws,
+                                          _ptr(l2_prefetch), pf_bytes, _stream(stream))
+    check("ft2_protect_fused_gemm_ex", st)
 
 
 def prefill_fused_gemm(x, w, y, bounds_out, workspace, bias=None, seq_offsets=None, num_seqs=None, scale=2.0,

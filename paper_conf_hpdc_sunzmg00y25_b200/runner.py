@@ -204,6 +204,12 @@ class Runner:
         # torch's kernels (experiments)
         self.host_norm = os.environ.get("FT2_HOST_NORM", "1") == "1"
         self.host_act = self.host_norm and os.environ.get("FT2_HOST_ACT", "1") == "1"
+        # L2 prefetch hint of the decode GEMMs (ft2_protect_fused_gemm_ex): each
+        # fused critical-layer GEMM pulls the weights of the next one into L2
+        # once its own operands have landed.  Measured slower in situ (OPT-1.3B
+        # decode step 1.79 -> 1.82 ms; the prefetch competes with the current
+        # layer's own weight stream), so opt-in: FT2_L2_PREFETCH=1
+        self.l2_prefetch = os.environ.get("FT2_L2_PREFETCH", "0") == "1"
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
@@ -340,8 +346,32 @@ class Runner:
         mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
         F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, bounds=st.bounds[cid], num_seqs=self.B,
                               corrected_count=st.corrected[cid], sites=sites, n_sites=self.B if sites is not None else None,
-                              cur_layer=lid, cur_step=step)
+                              cur_layer=lid, cur_step=step, l2_prefetch=self._next_fused_w(blk, name))
         return y
+
+    def _fused_gemm_order(self):
+        """(block, layer-or-group name) of every decode GEMM that runs on the
+        fused tcgen05 kernel, in execution order (the critical layers, or their
+        fused q/k/v / gate/up groups)."""
+        order = []
+        for blk in self.blocks:
+            for name in self.lin_names:
+                if name not in self.crit_names:
+                    continue
+                g = next((g for g, ns in blk.groups.items() if name in ns and self._group_ok(blk, g)), None)
+                order.append((blk, g if g is not None else name))
+        return order
+
+    def _next_fused_w(self, blk, name):
+        """Weights of the fused GEMM that follows (blk, name) in a decode step
+        (the first one of the next step after the last), as an L2 prefetch hint."""
+        if not self.l2_prefetch:
+            return None
+        if getattr(self, "_next_w", None) is None:
+            order = self._fused_gemm_order()
+            w_of = lambda b_, n_: b_.wf[n_] if n_ in b_.wf else b_.w[n_]
+            self._next_w = {(b_.idx, n_): w_of(*order[(i + 1) % len(order)]) for i, (b_, n_) in enumerate(order)}
+        return self._next_w.get((blk.idx, name))
 
     def _group_ok(self, blk: Block, g: str) -> bool:
         """A fused group runs as one GEMM when fusion is on, no fault sites are
@@ -385,7 +415,8 @@ class Runner:
             y = torch.empty((M, w.shape[0]), dtype=torch.bfloat16, device=x2.device)
             mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
             F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, col_begin=offs[ci], col_end=offs[ci + 1],
-                                  bounds=st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid])
+                                  bounds=st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid],
+                                  l2_prefetch=self._next_fused_w(blk, g))
         else:
             y = F.linear(x2, w, b)
             if ci is not None and (self.mode == "standalone" or (self.mode == "fused" and M > FUSED_MAX_M)):

@@ -90,3 +90,17 @@ def test_validation_without_gpu(L):
     # fused gemm CHECK without bounds
     assert L.ft2_protect_fused_gemm(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, 4, 16, 16, 1, 0, 0, 16,
                                     None, None, 1, None, None, 0, 0, 0, None, None, 0, None) == FT2_ERR_INVALID_ARG
+
+
+def test_fused_gemm_ex_prefetch_hint_validation(L):
+    from paper_conf_hpdc_sunzmg00y25_b200._lib import FT2_ERR_INVALID_ARG, FT2_ERR_MISALIGNED, FT2_ERR_UNSUPPORTED
+    P = ctypes.c_void_p
+
+    def ex(pf, nbytes, dtype=0, M=4):
+        return L.ft2_protect_fused_gemm_ex(P(0x1000), 16, P(0x2000), 16, None, P(0x3000), 16, M, 16, 16, 0, dtype,
+                                           0, 16, None, None, 0, None, None, 0, 0, 0, None, None, 0, pf, nbytes, None)
+    assert ex(None, 16) == FT2_ERR_INVALID_ARG          # bytes without a pointer
+    assert ex(P(0x4008), 16) == FT2_ERR_MISALIGNED      # pointer not 16-byte aligned
+    assert ex(P(0x4000), 24) == FT2_ERR_MISALIGNED      # size not a multiple of 16
+    assert ex(P(0x4000), 32, dtype=2) == FT2_ERR_UNSUPPORTED   # then the ft2_protect_fused_gemm checks
+    assert ex(None, 0, dtype=2) == FT2_ERR_UNSUPPORTED

@@ -116,21 +116,60 @@ def test_gemm_check_epilogue_bit_exact(ft2, M, N, K):
     assert rc.sum() > 0   # the bounds really clip something
 
 
-def test_gemm_clip_masks_vs_oracle_non_borderline(ft2):
-    M, N, K = 32, 4096, 4096
-    x, w, b = _operands(M, N, K, seed=11)
+@pytest.mark.parametrize("M,N,K,per_seq", [(32, 4096, 4096, False),
+                                           (32, 2048, 2048, True),     # C2 v/out: 16-token tiles, 4-way split
+                                           (32, 2048, 8192, True),     # C2 fc2: 12-way split
+                                           (32, 4096, 11008, True),    # C3 down
+                                           (32, 11008, 4096, True)])   # C3 up
+def test_gemm_clip_masks_vs_oracle_non_borderline(ft2, M, N, K, per_seq):
+    """R8 mask pin: the GEMM's clip decisions equal the oracle's (fp64 linear ->
+    bf16 -> R5 with the same bounds) on every neuron not within 1e-2 relative
+    of a bound; per-sequence bounds (row r -> sequence r) at the C2/C3 decode
+    shapes, each sequence with its own (lo, hi) around the output's spread."""
+    x, w, b = _operands(M, N, K, seed=11 + N + K)
     yd, yb = oracle.linear_f64(x, w, b)
-    bnds = np.array([[oracle.f64_to_bf16(-1.0), oracle.f64_to_bf16(1.0)]], np.uint16)
+    if per_seq:
+        rng = np.random.default_rng(N + K)
+        sd = np.std(yd, axis=1)
+        S = M
+        bnds = np.array([[oracle.f64_to_bf16(-sd[r] * rng.uniform(0.8, 2.5)),
+                          oracle.f64_to_bf16(sd[r] * rng.uniform(0.8, 2.5))] for r in range(M)], np.uint16)
+        r2s = np.arange(M, dtype=np.int32)
+    else:
+        S, r2s = 1, None
+        bnds = np.array([[oracle.f64_to_bf16(-1.0), oracle.f64_to_bf16(1.0)]], np.uint16)
     ref = yb.copy()
-    oracle.protect(ref, bnds)
+    rc = oracle.protect(ref, bnds, row_to_seq=r2s)
     ref_mask = ref != yb
-    checked, cnt = _run(ft2, x, w, b, 1, bounds=bnds, S=1)
+    checked, cnt = _run(ft2, x, w, b, 1, bounds=bnds, S=S, r2s=r2s)
     plain, _ = _run(ft2, x, w, b, 0)
     gpu_mask = checked != plain
-    lo, hi = -1.0, 1.0
-    border = (np.abs(yd - lo) <= 1e-2 * abs(lo)) | (np.abs(yd - hi) <= 1e-2 * abs(hi))
+    bf = _f64(bnds)
+    lo = bf[(r2s if r2s is not None else np.zeros(M, np.int64)), 0][:, None]
+    hi = bf[(r2s if r2s is not None else np.zeros(M, np.int64)), 1][:, None]
+    border = (np.abs(yd - lo) <= 1e-2 * np.abs(lo)) | (np.abs(yd - hi) <= 1e-2 * np.abs(hi))
     assert np.array_equal(gpu_mask[~border], ref_mask[~border])
     assert ref_mask.sum() > 100
+    # counts agree up to the borderline neurons
+    nb_rows = border.sum(axis=1)
+    slack = nb_rows if S > 1 else nb_rows.sum()
+    assert np.all(np.abs(cnt[:S].astype(np.int64) - rc.astype(np.int64)) <= slack)
+
+
+@pytest.mark.parametrize("M,N,K", [(32, 2048, 2048), (32, 2048, 8192), (4, 768, 768)])
+def test_gemm_l2_prefetch_hint_changes_nothing(ft2, M, N, K):
+    """ft2_protect_fused_gemm_ex: the L2 prefetch hint is a hint only --
+    outputs and counts are bit-identical with and without it."""
+    x, w, b = _operands(M, N, K, seed=23)
+    bnds = np.array([[oracle.f64_to_bf16(-0.1), oracle.f64_to_bf16(0.1)]], np.uint16)
+    ref, rcnt = _run(ft2, x, w, b, 1, bounds=bnds, S=1)
+    nxt = torch.zeros(((3 << 20) + 16) // 2, dtype=torch.bfloat16, device="cuda")   # 3 MB + 16 B
+    y = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ft2.protect_fused_gemm(dev(x), dev(w), y, bias=dev(b), mode=1 | 16, bounds=dev(bnds), num_seqs=1,
+                           corrected_count=cnt, l2_prefetch=nxt)
+    torch.cuda.synchronize()
+    assert np.array_equal(host(y), ref) and int(cnt.item()) == int(rcnt[0])
 
 
 def test_gemm_fault_injection_in_epilogue(ft2):

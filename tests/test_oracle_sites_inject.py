@@ -145,3 +145,64 @@ def test_sites_golden_seed42():
             s = sites[m][t]
             assert (int(s["step"]), int(s["layer"]), int(s["col"])) == (int(r[1]), int(r[2]), int(r[3]))
             assert int(s["xor_mask"]) == int(r[4 + m], 16)
+
+
+# ---- neuron-uniform (size-weighted) branch of R6, reading A11's flag
+# (layer_uniform = 0): every output neuron of every linear layer is equally
+# likely ("uniformly distributed location", read over neurons).
+
+def test_neuron_uniform_equal_widths_matches_layer_uniform_layer():
+    # With equal widths w the global neuron index g = floor(u1 * L * w / 2^32)
+    # lies in layer floor(g / w) = floor(u1 * L / 2^32): exactly the layer the
+    # layer-uniform branch draws from the same u1 (floor(floor(a)/w) = floor(a/w)).
+    # An off-by-one in the layer walk or a wrong size weighting breaks this.
+    n = 20000
+    for w, L in [(768, 12), (4096, 224), (1, 7)]:
+        lu = oracle.make_sites(5, 0, n, oracle.FAULT_1BIT, [w] * L, 32, 16, layer_uniform=True)
+        nu = oracle.make_sites(5, 0, n, oracle.FAULT_1BIT, [w] * L, 32, 16, layer_uniform=False)
+        assert np.array_equal(lu["layer"], nu["layer"])
+        assert np.all(nu["col"] < w)
+        # every other field comes from the other Philox words: identical
+        for f in ("step", "token", "xor_mask", "trial", "nbits"):
+            assert np.array_equal(lu[f], nu[f])
+
+
+def _philox_u1(seed, t):
+    # word u1 of the first Philox block of trial t (R6 counter layout); the
+    # generator itself is pinned by the Random123 known answers above
+    return oracle.philox4x32_10([t & 0xFFFFFFFF, t >> 32, 0, 0x46543200], [seed & 0xFFFFFFFF, seed >> 32])[1]
+
+
+def test_neuron_uniform_hand_computed_sites_three_layers():
+    # widths 3 / 5 / 2: 10 neurons; layer boundaries at global indices 3 and 8.
+    widths = [3, 5, 2]
+    s = oracle.make_sites(11, 0, 64, oracle.FAULT_1BIT, widths, 4, 2, layer_uniform=False)
+    for t in range(64):
+        g = (_philox_u1(11, t) * 10) >> 32          # uniform global neuron index in [0, 10)
+        want = (0, g) if g < 3 else ((1, g - 3) if g < 8 else (2, g - 8))
+        assert (int(s["layer"][t]), int(s["col"][t])) == want, t
+    # a single layer: the draw is plain neuron-uniform within it
+    one = oracle.make_sites(11, 0, 64, oracle.FAULT_1BIT, [10], 4, 2, layer_uniform=False)
+    assert np.all(one["layer"] == 0)
+    assert [int(c) for c in one["col"]] == [(_philox_u1(11, t) * 10) >> 32 for t in range(64)]
+
+
+def test_neuron_uniform_chi2_size_weighted():
+    # layer frequencies proportional to width (not 1/L), neurons uniform inside
+    n = 200000
+    widths = [4096, 11008, 4096, 2048, 11008, 768]
+    s = oracle.make_sites(2024, 0, n, oracle.FAULT_1BIT, widths, 32, 16, layer_uniform=False)
+    w = np.array(widths, np.float64)
+    cnt = np.bincount(s["layer"], minlength=len(widths))
+    assert _chi2_ok(cnt, n * w / w.sum())
+    assert not _chi2_ok(cnt, np.full(len(widths), n / len(widths)))   # layer-uniform would fail
+    assert np.all(s["col"] < np.array(widths)[s["layer"]])
+    for l in (1, 5):   # columns uniform inside a layer, 16 buckets
+        c = s[s["layer"] == l]["col"] * 16 // widths[l]
+        assert _chi2_ok(np.bincount(c, minlength=16), c.size / 16)
+    # Llama-2-7B geometry (224 layers): up/gate layers get 11008/4096 the hits of q/k/v/o/down
+    t = oracle.make_sites(77, 0, n, oracle.FAULT_1BIT, LLAMA7B_WIDTHS, 32, 16, layer_uniform=False)
+    kind = np.bincount(t["layer"] % 7, minlength=7)
+    wk = np.array(LLAMA7B_WIDTHS[:7], np.float64)
+    assert _chi2_ok(kind, n * wk / wk.sum())
+    assert np.all(t["col"] < np.array(LLAMA7B_WIDTHS)[t["layer"]])

@@ -58,7 +58,7 @@ for kind in ("cublas", "ft2", "none"):
                 torch.matmul(hot_a, hot_a)
             g.replay()
         torch.cuda.synchronize()
-        buf = np.zeros(4096 * 16, np.uint64)
+        buf = np.zeros(32768 * 16, np.uint64)
         L.ft2_debug_trace_read(buf.ctypes.data, buf.nbytes)
         mk = np.zeros(64, np.uint64)
         L.ft2_debug_marks_read(mk.ctypes.data)

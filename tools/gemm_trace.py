@@ -41,7 +41,7 @@ for M, N, K in shapes:
         step()
     for _ in range(5): g.replay()
     torch.cuda.synchronize()
-    buf = np.zeros(4096 * 16, np.uint64)
+    buf = np.zeros(32768 * 16, np.uint64)
     L.ft2_debug_trace_read(buf.ctypes.data, buf.nbytes)
     t = buf.reshape(-1, 16).astype(np.int64)
     t = t[t[:, 0] > 0]
