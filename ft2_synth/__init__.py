@@ -72,10 +72,11 @@ def weight_scale_log2(K: int) -> int:
     return -int(math.ceil(math.log2(math.sqrt(K))))
 
 
-def gen_bf16(shape, tau: int, sigma: int, scale_log2: int = 0, start: int = 0) -> np.ndarray:
+def gen_bf16(shape, tau: int, sigma: int, scale_log2: int = 0, start: int = 0, outliers: bool = True) -> np.ndarray:
     """bf16 bit patterns (uint16 array of ``shape``) for tensor id ``tau``, seed ``sigma``.
 
-    Element ``i`` is the row-major flat index offset by ``start``.
+    Element ``i`` is the row-major flat index offset by ``start``.  outliers=False
+    drops the planted 2**-10 outliers (every value keeps its bulk draw).
     """
     n = int(np.prod(shape)) if len(shape) else 1
     i = np.arange(start, start + n, dtype=np.uint64)
@@ -84,11 +85,14 @@ def gen_bf16(shape, tau: int, sigma: int, scale_log2: int = 0, start: int = 0) -
     z = ((u0 >> np.uint64(16)) + (u0 & np.uint64(0xFFFF)) + (u1 >> np.uint64(16))
          + (u1 & np.uint64(0xFFFF))).astype(np.int64) - 131070
     e = np.where((u2 & np.uint64(0x3FF)) == 0, 5 + ((u2 >> np.uint64(10)) & np.uint64(3)).astype(np.int64), 0)
+    if not outliers:
+        e = np.zeros_like(e)
     v = np.ldexp(z.astype(np.float64), (e - 17 + scale_log2).astype(np.int32)).astype(np.float32)
     return _rne_f32_to_bf16_bits(v).reshape(shape)
 
 
-def gen_bf16_torch(shape, tau: int, sigma: int, scale_log2: int = 0, device="cpu", start: int = 0):
+def gen_bf16_torch(shape, tau: int, sigma: int, scale_log2: int = 0, device="cpu", start: int = 0,
+                   outliers: bool = True):
     """Same recipe as :func:`gen_bf16`, built with torch int64 ops on ``device``.
 
     Returns a ``torch.bfloat16`` tensor.  Chunked to bound temporary memory.
@@ -120,6 +124,8 @@ def gen_bf16_torch(shape, tau: int, sigma: int, scale_log2: int = 0, device="cpu
         u0, u1, u2 = c0, c1, c2
         z = (u0 >> 16) + (u0 & 0xFFFF) + (u1 >> 16) + (u1 & 0xFFFF) - 131070
         e = torch.where((u2 & 0x3FF) == 0, 5 + ((u2 >> 10) & 3), torch.zeros_like(u2))
+        if not outliers:
+            e = torch.zeros_like(u2)
         v = z.to(torch.float64) * torch.pow(2.0, (e - 17 + scale_log2).to(torch.float64))
         b = v.to(torch.float32).view(torch.int32).to(torch.int64) & M32
         lsb = (b >> 16) & 1

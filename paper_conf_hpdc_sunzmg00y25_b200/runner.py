@@ -108,21 +108,21 @@ CONFIGS = {
 }
 
 
-def _w(shape, tau, seed, device, K=None):
+def _w(shape, tau, seed, device, K=None, outliers=True):
     sl = ft2_synth.weight_scale_log2(K) if K else 0
-    return ft2_synth.gen_bf16_torch(shape, tau, seed, scale_log2=sl, device=device)
+    return ft2_synth.gen_bf16_torch(shape, tau, seed, scale_log2=sl, device=device, outliers=outliers)
 
 
 class Block:
-    def __init__(self, cfg: ModelConfig, idx: int, seed: int, device):
+    def __init__(self, cfg: ModelConfig, idx: int, seed: int, device, outliers: bool = True):
         self.cfg = cfg
         self.idx = idx
         tau0 = 1000 + 64 * idx
         self.w = {}
         self.b = {}
         for j, (name, o, i, _) in enumerate(cfg.linears()):
-            self.w[name] = _w((o, i), tau0 + 2 * j, seed, device, K=i)
-            self.b[name] = _w((o,), tau0 + 2 * j + 1, seed, device) if cfg.bias else None
+            self.w[name] = _w((o, i), tau0 + 2 * j, seed, device, K=i, outliers=outliers)
+            self.b[name] = _w((o,), tau0 + 2 * j + 1, seed, device, outliers=outliers) if cfg.bias else None
         # horizontally fused projections (same weights; the per-layer tensors
         # become views into the fused ones): qkv, and Llama's gate_up
         self.groups = {"qkv": ["q_proj", "k_proj", "v_proj"]}
@@ -165,7 +165,16 @@ class Runner:
     """Batched greedy generation with FT2 on the critical layers."""
 
     def __init__(self, cfg: ModelConfig, batch: int, prompt_len: int, gen_len: int, seed: int = 1,
-                 device="cuda", scale: float = 2.0, coverage: str = "ft2", fuse_proj: bool | None = None):
+                 device="cuda", scale: float = 2.0, coverage: str = "ft2", fuse_proj: bool | None = None,
+                 share: "Runner | None" = None, outliers: bool = True):
+        """share: another Runner of the same config, batch and lengths whose
+        weights, KV caches and static token / site buffers this one reuses
+        (no copy; see with_coverage).  Runners sharing buffers must not run
+        concurrently.  outliers=False builds the weights and embeddings without
+        the synthetic recipe's planted 2**-10 outliers: the
+        fault-injection campaign's model, whose fault-free activation range is
+        stable from the first token on (the premise of first-token bounds,
+        PAPER.md L223-L233), unlike the heavy-tailed outlier model."""
         self.cfg = cfg
         self.B = batch
         self.T = prompt_len
@@ -175,12 +184,17 @@ class Runner:
         self.device = torch.device(device)
         dv = self.device
         h = cfg.hidden
-        self.embed = _w((cfg.vocab, h), 1, seed, dv)
-        self.pos_embed = _w((cfg.max_pos + 2, h), 2, seed, dv) if cfg.arch == "opt" else None
-        self.blocks = [Block(cfg, i, seed, dv) for i in range(cfg.n_layers)]
-        self.lnf_w = torch.ones(h, dtype=torch.bfloat16, device=dv)
-        self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
-        self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h)
+        if share is not None:
+            assert (share.cfg, share.B, share.T, share.G) == (cfg, batch, prompt_len, gen_len)
+            for a in ("embed", "pos_embed", "blocks", "lnf_w", "lnf_b", "lm_head"):
+                setattr(self, a, getattr(share, a))
+        else:
+            self.embed = _w((cfg.vocab, h), 1, seed, dv, outliers=outliers)
+            self.pos_embed = _w((cfg.max_pos + 2, h), 2, seed, dv, outliers=outliers) if cfg.arch == "opt" else None
+            self.blocks = [Block(cfg, i, seed, dv, outliers=outliers) for i in range(cfg.n_layers)]
+            self.lnf_w = torch.ones(h, dtype=torch.bfloat16, device=dv)
+            self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
+            self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h, outliers=outliers)
         self.coverage = coverage
         # fuse_proj: fused q/k/v (and Llama gate/up) projections, one GEMM per
         # group; the protected layer of a group (v_proj, up_proj) is a column
@@ -215,22 +229,40 @@ class Runner:
         self.n_crit = len(self.crit_names) * cfg.n_layers
         self.state = FT2State(self.n_crit, batch, dv)
         H, D = cfg.n_heads, cfg.head_dim
-        self.k_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
-                        for _ in range(cfg.n_layers)]
-        self.v_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
-                        for _ in range(cfg.n_layers)]
-        self.seq_offsets = torch.arange(0, (batch + 1) * prompt_len, prompt_len, dtype=torch.int32, device=dv)
-        # decode-step static buffers (CUDA-graph inputs/outputs)
-        self.prompt_static = torch.zeros((batch, prompt_len), dtype=torch.int64, device=dv)
+        # buffers a with_coverage() clone shares with its parent (graphs bake in
+        # their addresses; runs are sequential on one stream)
+        shared = ("k_cache", "v_cache", "seq_offsets", "prefill_r2s", "prompt_static", "tok", "pos",
+                  "out_tokens", "sites_buf", "cur_step", "h_trace")
+        if share is not None:
+            for a in shared:
+                setattr(self, a, getattr(share, a))
+        else:
+            self.k_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
+                            for _ in range(cfg.n_layers)]
+            self.v_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
+                            for _ in range(cfg.n_layers)]
+            self.seq_offsets = torch.arange(0, (batch + 1) * prompt_len, prompt_len, dtype=torch.int32, device=dv)
+            # prefill row -> sequence (supplied-bounds check of the first token)
+            self.prefill_r2s = torch.arange(batch * prompt_len, dtype=torch.int32, device=dv) // prompt_len
+            # decode-step static buffers (CUDA-graph inputs/outputs)
+            self.prompt_static = torch.zeros((batch, prompt_len), dtype=torch.int64, device=dv)
+            self.tok = torch.zeros(batch, dtype=torch.int64, device=dv)
+            self.pos = torch.zeros(1, dtype=torch.int64, device=dv)
+            self.out_tokens = torch.zeros((batch, gen_len), dtype=torch.int64, device=dv)
+            # stable site buffer: graphs captured with faults bake in its address, so
+            # a campaign rewrites it per batch (set_sites / make_sites) and replays
+            self.sites_buf = torch.zeros(batch * F2.SITE_BYTES, dtype=torch.uint8, device=dv)
+            self.cur_step = torch.zeros(1, dtype=torch.int32, device=dv)
+            # last-position hidden state (before the final norm) of every generated
+            # token [G, B, hidden]: the campaign's deviation proxy reads it
+            self.h_trace = torch.zeros((gen_len, batch, h), dtype=torch.bfloat16, device=dv)
         self.graph_prefill = True   # first-token pass as a CUDA graph (False: eager)
-        self.tok = torch.zeros(batch, dtype=torch.int64, device=dv)
-        self.pos = torch.zeros(1, dtype=torch.int64, device=dv)
-        self.out_tokens = torch.zeros((batch, gen_len), dtype=torch.int64, device=dv)
         self.sites = None        # optional fault sites (uint8 [B*24]); site i = sequence i
-        # stable site buffer: graphs captured with faults bake in its address, so
-        # a campaign rewrites it per batch (set_sites / make_sites) and replays
-        self.sites_buf = torch.zeros(batch * F2.SITE_BYTES, dtype=torch.uint8, device=dv)
-        self.cur_step = torch.zeros(1, dtype=torch.int32, device=dv)
+        # caller-supplied ("offline") bounds [n_crit, B, 2] (set_supplied_bounds):
+        # the first-token bound sweep is skipped and the prefill outputs are
+        # checked against them like every later token
+        self.supplied_bounds = None
+        self._profile_keys = None
         self.graphs = {}
         self._pool = torch.cuda.graph_pool_handle() if self.device.type == "cuda" else None   # shared by all graphs
         self.time_phases = False
@@ -311,11 +343,21 @@ class Runner:
                 li = self._lin_id(blk.idx, name)
                 F2.bounds_from_prefill(y, None, self._nv_ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
                                        finalize=False, keys_out=self._nv_keys, nan_vulnerable_count=self._nv[li])
-            if crit and self.mode != "off":
+            if crit and self._profile_keys is not None:   # offline profiling: raw keys, all rows one range
+                cid = self._crit_id(blk.idx, name)
+                F2.bounds_from_prefill(y, None, self.state.ws, num_seqs=1, finalize=False,
+                                       keys_out=self._profile_tmp)
+                torch.maximum(self._profile_keys[cid], self._profile_tmp[0], out=self._profile_keys[cid])
+            elif crit and self.mode != "off":
                 cid = self._crit_id(blk.idx, name)
                 st = self.state
-                F2.bounds_from_prefill(y, st.bounds[cid], st.ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
-                                       scale=self.scale, correct_nonfinite=True, nonfinite_count=st.nonfinite[cid])
+                if self.supplied_bounds is not None:   # offline bounds: the first token is checked too
+                    F2.protect(y, st.bounds[cid], row_to_seq=self.prefill_r2s, num_seqs=self.B,
+                               corrected_count=st.corrected[cid])
+                else:
+                    F2.bounds_from_prefill(y, st.bounds[cid], st.ws, seq_offsets=self.seq_offsets, num_seqs=self.B,
+                                           scale=self.scale, correct_nonfinite=True,
+                                           nonfinite_count=st.nonfinite[cid])
             return y
         # decode.  The fused tcgen05 GEMM serves decode batches of up to
         # FUSED_MAX_M tokens (swap-AB, cluster split-K); larger decode batches
@@ -407,6 +449,8 @@ class Runner:
                                            nan_vulnerable_count=self._nv[self._lin_id(blk.idx, n)])
             if ci is not None and self.mode != "off":
                 cid = self._crit_id(blk.idx, names[ci])
+                if self.supplied_bounds is not None or self._profile_keys is not None:
+                    raise ValueError("supplied / profiled bounds need fuse_proj=False")
                 F2.bounds_from_prefill(y[:, offs[ci]:offs[ci + 1]], st.bounds[cid], st.ws, seq_offsets=self.seq_offsets,
                                        num_seqs=self.B, scale=self.scale, correct_nonfinite=True,
                                        nonfinite_count=st.nonfinite[cid])
@@ -493,6 +537,7 @@ class Runner:
         pidx = pos.unsqueeze(0).expand(B, T)
         for blk in self.blocks:
             x = self._block(blk, x, "prefill", pos_idx=pidx, step=0)
+        self.h_trace[0].copy_(x[:, -1])
         nxt = self._logits_next(x[:, -1])
         return nxt
 
@@ -504,11 +549,56 @@ class Runner:
         x = self._embed(self.tok.view(self.B, 1), pidx)
         for blk in self.blocks:
             x = self._block(blk, x, "decode", pos_idx=pidx, step=self._site_step)
-        nxt = self._logits_next(x[:, -1])
         gi = (self.pos - self.T + 1).clamp_(0, self.G - 1)
+        self.h_trace.index_copy_(0, gi, x[:, -1].unsqueeze(0))
+        nxt = self._logits_next(x[:, -1])
         self.out_tokens.index_copy_(1, gi, nxt.view(self.B, 1))
         self.tok.copy_(nxt)
         self.pos.add_(1)
+
+    def with_coverage(self, coverage: str) -> "Runner":
+        """A runner protecting another layer set (Table 1) over the
+        SAME weights, caches and site buffer (no copy): its own bounds,
+        counters and CUDA graphs.  Used for paired coverage comparisons."""
+        return Runner(self.cfg, self.B, self.T, self.G, device=self.device, scale=self.scale, coverage=coverage,
+                      fuse_proj=self.fuse_proj, share=self)
+
+    def set_supplied_bounds(self, bounds):
+        """Caller-supplied ("offline") bounds, bf16 [n_crit, B, 2] or [n_crit, 2]
+        (broadcast over the batch), or None to return to first-token bounds.
+        With bounds supplied the prefill skips FT2's first-token bound sweep
+        and checks the protected prefill outputs against them instead (range
+        restriction with fixed bounds, as the offline-profiled schemes
+        PAPER.md L116 / L286 compare against)."""
+        if bounds is None:
+            self.supplied_bounds = None
+            return
+        b = bounds.to(device=self.device, dtype=torch.bfloat16)
+        if b.dim() == 2:
+            b = b.unsqueeze(1).expand(self.n_crit, self.B, 2)
+        assert tuple(b.shape) == (self.n_crit, self.B, 2), b.shape
+        self.supplied_bounds = b.contiguous().clone()
+
+    def profile_offline_bounds(self, prompt_batches, scale=None):
+        """Offline bound profiling (the baseline FT2 replaces, PAPER.md L116,
+        L286): run unprotected first-token passes over `prompt_batches` (each
+        [B, T] token ids) and keep, per protected layer, the min / max over
+        every finite output of every batch, widened by `scale` (default the
+        runner's, 2).  Exact: raw order keys max-combined across batches, then
+        ft2_bounds_finalize.  Returns bf16 [n_crit, 2]."""
+        st = self.state
+        self._profile_keys = torch.full((self.n_crit, 2), -1, dtype=torch.int32, device=self.device)
+        self._profile_tmp = torch.zeros((1, 2), dtype=torch.int32, device=self.device)
+        mode, self.mode = self.mode, "off"
+        try:
+            for ids in prompt_batches:
+                self.prefill(ids.to(self.device))
+        finally:
+            self.mode = mode
+        out = torch.zeros((self.n_crit, 2), dtype=torch.bfloat16, device=self.device)
+        F2.bounds_finalize(self._profile_keys, out, scale=self.scale if scale is None else scale)
+        self._profile_keys = None
+        return out
 
     def set_sites(self, sites):
         """Fault sites for the next generate() calls (uint8 [B*24], site i =
@@ -562,7 +652,7 @@ class Runner:
         """CUDA graph of the whole first-token pass (embedding, 24 blocks with
         the FT2 bound sweeps on the critical layers, LM head, first token) on
         the static prompt buffer; one per mode."""
-        key = ("prefill", mode, self.sites is not None)
+        key = ("prefill", mode, self.sites is not None, self.supplied_bounds is not None)
         if key not in self.graphs:
             self.mode = mode
             self._site_step = None
@@ -602,6 +692,8 @@ class Runner:
         if use_graph and self.graph_prefill:
             pg = self._prefill_graph(mode)   # capture (and its warm-up) before the counters reset
         self.state.reset_counters()
+        if self.supplied_bounds is not None:
+            self.state.bounds.copy_(self.supplied_bounds)
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)] if self.time_phases else None
         if ev:
             ev[0].record()

@@ -125,3 +125,117 @@ def test_partial_batch_counts_only_its_rows(tiny):
     assert part.sdc_off <= full.sdc_off and part.detected_on <= full.detected_on
     eager = campaign.run_batch(tiny, prompts, 3, 0, 2, golden=gold, use_graph=False)
     assert eager == full
+
+
+def test_paired_coverages_on_identical_sites(tiny):
+    """NEXT(4): Table 1 coverages compared on the SAME
+    sites -- the unprotected run is shared, every coverage replays its own
+    protected generation over shared weights.  "none" (Ranger's linear-layer
+    coverage) must equal the unprotected run trial by trial; "ft2" must equal
+    the plain campaign path's FT2-on result."""
+    from paper_conf_hpdc_sunzmg00y25_b200 import campaign
+    prompts = campaign.campaign_prompts(tiny)
+    covs = {c: tiny.with_coverage(c) for c in ("ft2", "maximals", "globalclipper", "all", "none")}
+    assert covs["all"].blocks is tiny.blocks and covs["all"].sites_buf is tiny.sites_buf
+    assert [covs[c].n_crit for c in covs] == [4 * 2, 2 * 2, 2 * 2, 7 * 2, 0]   # Llama: maximals o/down, gc v/o
+    goldens = {c: campaign.golden_runs(r, prompts) for c, r in covs.items()}
+    goldens["off"] = campaign.golden_runs(tiny, prompts)
+    res = campaign.PairedResult
+    tot = {c: res() for c in list(covs) + ["off"]}
+    plain = campaign.CampaignResult()
+    for t0 in (0, 16, 32):
+        r = campaign.run_coverages(covs, tiny, prompts, 5, t0, 2, goldens)
+        for c, v in r.items():
+            tot[c].add(v)
+        plain.add(campaign.run_batch(covs["ft2"], prompts, 5, t0, 2, golden=goldens["ft2"]))
+    assert tot["none"].sdc == tot["off"].sdc and tot["none"].detected == 0
+    assert tot["ft2"].sdc == plain.sdc_on and tot["ft2"].detected == plain.detected_on
+    assert tot["ft2"].sdc_only_c == 0 and tot["ft2"].sdc_only_ref == 0
+    for c, v in tot.items():
+        assert v.trials == 48
+        # discordant pairs reconstruct the difference of the marginals
+        assert v.sdc - tot["ft2"].sdc == v.sdc_only_c - v.sdc_only_ref
+        assert v.dev_large - tot["ft2"].dev_large == v.dev_only_c - v.dev_only_ref
+    assert tot["all"].detected >= tot["ft2"].detected > 0
+
+
+def test_supplied_bounds_bypass_the_sweep_and_clip_like_the_oracle(tiny):
+    """Caller-supplied (offline) bounds: the first-token sweep is skipped (the
+    state holds exactly the supplied bounds, no prefill non-finite count),
+    every-token checks use them (R5, bit-exact on the layer's own PLAIN
+    output), and bounds wide enough to clip nothing reproduce the unprotected
+    generation exactly."""
+    import torch.nn.functional as F
+    from paper_conf_hpdc_sunzmg00y25_b200 import campaign
+    prompts = campaign.campaign_prompts(tiny)
+    ref_plain = tiny.generate(prompts, "fused_plain").clone()
+    wide = torch.tensor([-3.0e38, 3.0e38], dtype=torch.bfloat16).expand(tiny.n_crit, 2)
+    tiny.set_supplied_bounds(wide)
+    try:
+        out = tiny.generate(prompts, "fused").clone()
+        assert torch.equal(out, ref_plain)
+        assert int(tiny.state.corrected.sum()) == 0 and int(tiny.state.nonfinite.sum()) == 0
+        narrow = torch.tensor([-0.05, 0.05], dtype=torch.bfloat16).expand(tiny.n_crit, 2)
+        tiny.set_supplied_bounds(narrow)
+        tiny.generate(prompts, "fused")
+        st = tiny.state
+        assert torch.equal(st.bounds, narrow.unsqueeze(1).expand(tiny.n_crit, tiny.B, 2).to(st.bounds.device))
+        assert int(st.corrected.sum()) > 0 and int(st.nonfinite.sum()) == 0
+        # one decode layer call against the oracle: CHECK == R5(PLAIN) with the supplied bounds
+        blk = tiny.blocks[1]
+        x2 = torch.randn(tiny.B, tiny.cfg.hidden, device="cuda").to(torch.bfloat16)
+        tiny.mode = "fused_plain"
+        plain = tiny._linear(x2, blk, "v_proj", "decode").clone()
+        tiny.mode = "fused"
+        chk = tiny._linear(x2, blk, "v_proj", "decode").clone()
+        ref = plain.view(torch.int16).cpu().numpy().view(np.uint16).copy()
+        b = narrow[0].view(torch.int16).numpy().view(np.uint16).reshape(1, 2)
+        oracle.protect(ref, b)
+        assert np.array_equal(chk.view(torch.int16).cpu().numpy().view(np.uint16), ref)
+        # the prefill outputs are checked too: block 0's v_proj output lies within the bounds
+        tiny.set_supplied_bounds(narrow)
+        pos = torch.arange(tiny.T, device="cuda")
+        x = tiny._embed(prompts, pos.unsqueeze(0).expand(tiny.B, tiny.T))
+        h2 = tiny._norm(x, tiny.blocks[0].ln1_w, tiny.blocks[0].ln1_b).reshape(-1, tiny.cfg.hidden)
+        y = tiny._linear(h2, tiny.blocks[0], "v_proj", "prefill").float()
+        lo, hi = float(narrow[0, 0]), float(narrow[0, 1])
+        assert float(y.max()) <= hi and float(y.min()) >= lo
+        yr = F.linear(h2, tiny.blocks[0].w["v_proj"]).float()
+        assert float(yr.max()) > hi                # so the check really clipped
+    finally:
+        tiny.set_supplied_bounds(None)
+
+
+def test_offline_profiled_bounds_match_oracle(tiny):
+    """profile_offline_bounds: per protected layer, min / max over every output
+    of every profiling batch (x2), equal to the oracle's bounds of the
+    concatenated outputs (block 0's v_proj recomputed with the same cuBLAS call)."""
+    import torch.nn.functional as F
+    gens = [torch.Generator().manual_seed(40 + i) for i in range(2)]
+    batches = [torch.randint(0, 512, (16, 8), generator=g).cuda() for g in gens]
+    b = tiny.profile_offline_bounds(batches)
+    assert b.shape == (tiny.n_crit, 2)
+    ys = []
+    pos = torch.arange(8, device="cuda")
+    for p in batches:
+        x = tiny._embed(p, pos.unsqueeze(0).expand(16, 8))
+        h2 = tiny._norm(x, tiny.blocks[0].ln1_w, tiny.blocks[0].ln1_b).reshape(-1, tiny.cfg.hidden)
+        ys.append(F.linear(h2, tiny.blocks[0].w["v_proj"]).view(torch.int16).cpu().numpy().view(np.uint16))
+    want, _, _ = oracle.bounds(np.ascontiguousarray(np.concatenate(ys)), scale=2.0)
+    cid = tiny._crit_id(0, "v_proj")
+    assert b[cid].view(torch.int16).cpu().numpy().view(np.uint16).tolist() == want.reshape(-1).tolist()
+
+
+def test_hidden_deviation_proxy(tiny):
+    from paper_conf_hpdc_sunzmg00y25_b200 import campaign
+    prompts = campaign.campaign_prompts(tiny)
+    gold = campaign.golden_runs(tiny, prompts)
+    tot = campaign.CampaignResult()
+    for t0 in range(0, 64, 16):
+        tot.add(campaign.run_batch(tiny, prompts, 5, t0, 2, golden=gold))
+    assert 0 <= tot.dev_large_on <= tot.trials and 0 <= tot.dev_large_off <= tot.trials
+    assert tot.nonfinite_off <= tot.dev_large_off and tot.nonfinite_on <= tot.dev_large_on
+    # fault-free: zero deviation against itself
+    steps = torch.zeros(tiny.B, dtype=torch.long, device="cuda")
+    d, nf = campaign.hidden_deviation(gold.h_on, gold.h_on, steps)
+    assert float(d.max()) == 0.0 and not bool(nf.any())

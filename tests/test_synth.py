@@ -27,3 +27,22 @@ def test_distribution_shape():
     assert 1.1 < v.std().item() < 1.4 and v.abs().max().item() < 256
     assert 0.25 < v[v.abs() < 2].std().item() < 0.33
     assert np.isfinite(v.numpy()).all()
+
+
+def test_outlier_free_variant_matches_bulk_and_agrees_across_backends():
+    # outliers=False keeps every element's bulk draw and drops only the planted
+    # 2^-10 outliers; numpy and torch builds agree bit for bit
+    import torch
+    a = ft2_synth.gen_bf16((300, 700), tau=5, sigma=9)
+    b = ft2_synth.gen_bf16((300, 700), tau=5, sigma=9, outliers=False)
+    t = ft2_synth.gen_bf16_torch((300, 700), 5, 9, outliers=False).view(torch.int16).numpy().view(np.uint16)
+    assert np.array_equal(b, t)
+    va = a.astype(np.uint32) << 16
+    vb = b.astype(np.uint32) << 16
+    fa, fb = va.view(np.float32), vb.view(np.float32)
+    same = fa == fb
+    assert 0.0005 < 1 - same.mean() < 0.002          # ~2^-10 of the elements differ
+    assert np.all(np.abs(fb) < 1.0)                  # bulk: |z| * 2^-17 < 1
+    d = ~same
+    ratio = np.abs(fa[d] / fb[d])
+    assert np.all(np.isin(np.round(np.log2(ratio)).astype(int), [5, 6, 7, 8]))
