@@ -197,13 +197,28 @@ class ClockSampler:
 _ORACLE_INPUTS = {}
 
 
-def oracle_sample(model_name, B, T, G, seed=1):
+def host_cpu():
+    """nproc and the CPU model of the host the oracle runs on."""
+    import platform
+    model = platform.processor() or "?"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+def oracle_sample(model_name, B, T, G, seed=1, threads=0):
     """Time the CPU oracle on a bounded sample of the same workload: the
     critical layers (v_proj, out_proj, fc2) of ONE of the 24 blocks, for the
     prefill bounds (+correction) and ONE decode step at batch B (fp64 linear ->
     bf16 -> check-and-clip, R8 -> R5).  Extrapolated x n_layers x (G-1) decode
     steps; attention / non-critical layers are outside the oracle (and outside
-    FT2's hot path) and are not counted.  Single-threaded C."""
+    FT2's hot path) and are not counted.  Plain C; `threads` OpenMP threads
+    over independent outputs (0 = all host cores; results are identical)."""
     import numpy as np
 
     import ft2_synth
@@ -224,6 +239,7 @@ def oracle_sample(model_name, B, T, G, seed=1):
         _ORACLE_INPUTS[key] = (ws, bs, xs_dec, ys_pre)
     ws, bs, xs_dec, ys_pre = _ORACLE_INPUTS[key]
     ys_pre = [y.copy() for y in ys_pre]
+    cores = oracle.set_threads(threads)
     so = np.arange(0, (B + 1) * T, T, dtype=np.int32)
     t0 = time.perf_counter()
     bounds = []
@@ -240,7 +256,7 @@ def oracle_sample(model_name, B, T, G, seed=1):
             "sample": (f"critical layers ({', '.join(n for n, _, _ in crit)}) of 1 of {cfg.n_layers} blocks: "
                        f"prefill bounds on [{B*T}, N] + 1 decode step at B={B} (fp64 linear + check); "
                        f"extrapolated x{cfg.n_layers} blocks x{G-1} steps"),
-            "cores": 1}
+            "cores": cores}
 
 
 # ------------------------------------------------------------------ main
@@ -270,7 +286,7 @@ def main():
                 "config": {"workload": workload_name(args.model, args.batch, args.prompt, args.gen),
                            "model": args.model, "global_batch": args.batch, "seq_len": args.prompt + args.gen},
                 "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": r["cores"], "kind": "oracle",
-                                 "sample": r["sample"]},
+                                 "sample": r["sample"], **host_cpu()},
                 "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
         return 0
@@ -280,7 +296,10 @@ def main():
 
     if world > 1:
         # NCCL over NVLink; FT2_BENCH_BACKEND=gloo lets a multi-rank smoke run
-        # share one GPU (ranks are mapped onto the visible devices round-robin)
+        # share one GPU (ranks are mapped onto the visible devices round-robin).
+        # NCCL's init log stays on (communicator sizes are checkable in stderr)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group(os.environ.get("FT2_BENCH_BACKEND", "nccl"))
     local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
@@ -473,16 +492,59 @@ def main():
         rf["share_of_decode_step"] = rf["launches_per_graph"] * rf["avg_launch_us"] / dec_us
     if not args.no_extras:
         res["coverage_overhead_pct"] = coverage_costs(cfg, B, T, G, dev, prompt, stream, runner, ms_off)
+    if not args.no_extras:
+        # the paths that shard, at this run's N: configs[3]'s
+        # TP bounds + row-parallel check, configs[4]'s campaign with its trial
+        # ranges split over the ranks
+        del runner
+        torch.cuda.empty_cache()
+        res["partitioned_paths"] = partitioned_legs(args, dev, rank, world)
     if rank == 0 and world == 1 and not args.no_extras:
         res["c1_single_layer"] = c1_leg(dev, ft2)
-        cb = oracle_sample(args.model, B, T, G)
+        cb = oracle_sample(args.model, B, T, G, threads=0)
+        cb1 = oracle_sample(args.model, B, T, G, threads=1)
         res["cpu_baseline"] = {"value": cb["tokens_per_s"], "unit": "tokens/s", "cores": cb["cores"],
-                               "kind": "oracle", "sample": cb["sample"]}
+                               "kind": "oracle", "sample": cb["sample"], **host_cpu(),
+                               "single_thread": {"value": cb1["tokens_per_s"], "cores": 1},
+                               "threads_note": "OpenMP over independent outputs; bit-identical results"}
     if rank == 0:
         print(json.dumps(res), flush=True)
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def partitioned_legs(args, dev, rank, world, trials_per_rank=512):
+    """The partitioned paths of north_star at N = world ranks, in the default
+    run (so a SCALE run at 1/2/4/8 GPUs records them per N):
+    - c4: Llama-2-13B TP bounds -- per-rank column-shard sweeps, ONE NCCL MAX
+      all-reduce of int32 keys, finalize (bit-exact vs the unsharded sweep),
+      and the row-parallel decode check: NCCL all-reduce + ft2_protect vs the
+      fused one-shot ft2_allreduce_protect over peer memory (NEXT(2));
+    - c5: the fault-injection campaign with trial ranges sharded over the
+      ranks, `trials_per_rank` trials per rank and fault model (weak scaling),
+      one counter all-reduce per model."""
+    import copy
+
+    import torch
+    import torch.distributed as dist
+
+    out = {"n_ranks": world}
+    if world > 1:
+        t = torch.ones(1, device=dev)
+        dist.all_reduce(t)
+        out["comm_nranks_ok"] = int(t.item()) == world
+    out["c4_tp"] = c4_tp_bounds(args, dev, rank, world)
+    torch.cuda.empty_cache()
+    a = copy.copy(args)
+    a.trials = trials_per_rank * world
+    a.coverage_trials = 0
+    c5 = c5_campaign(a, dev, rank, world)
+    c5["scaling"] = "weak"
+    c5["trials_per_s_per_gpu"] = c5["value"] / world
+    out["c5_campaign"] = c5
+    torch.cuda.empty_cache()
+    return out
 
 
 def coverage_costs(cfg, B, T, G, dev, prompt, stream, runner_ft2, ms_off_ft2, rounds=9):
@@ -724,15 +786,21 @@ def c1_leg(dev, ft2, R=20):
         xpn = xp.cpu().view(torch.int16).numpy().view(np.uint16)
         xsn = xs.cpu().view(torch.int16).numpy().view(np.uint16)
         sn = oracle.make_sites(42, 0, S, oracle.FAULT_1BIT, [H], n_steps=S, prompt_len=T, step_policy=1)
-        t0 = time.perf_counter()
-        _, ypn = oracle.linear_f64(xpn, wn, bn_)
-        rb, _, _ = oracle.bounds(ypn, correct_nonfinite=True)
-        for t in range(1, S + 1):
-            _, y = oracle.linear_f64(xsn[t - 1], wn, bn_)
-            oracle.inject(y, sn, 0, t, base_row=np.zeros(S, np.int32))
-            oracle.protect(y, rb)
-        out["cpu_baseline"] = {"value": time.perf_counter() - t0, "unit": "s per request", "cores": 1,
-                               "kind": "oracle", "sample": "the whole C1 request"}
+
+        def request(threads):
+            cores = oracle.set_threads(threads)
+            t0 = time.perf_counter()
+            _, ypn = oracle.linear_f64(xpn, wn, bn_)
+            rb, _, _ = oracle.bounds(ypn, correct_nonfinite=True)
+            for t in range(1, S + 1):
+                _, y = oracle.linear_f64(xsn[t - 1], wn, bn_)
+                oracle.inject(y, sn, 0, t, base_row=np.zeros(S, np.int32))
+                oracle.protect(y, rb)
+            return time.perf_counter() - t0, cores
+        t1, _ = request(1)
+        tn, cores = request(0)
+        out["cpu_baseline"] = {"value": tn, "unit": "s per request", "cores": cores, "kind": "oracle",
+                               "sample": "the whole C1 request", "single_thread_s": t1, **host_cpu()}
     except Exception as e:   # the oracle is test infrastructure; its absence must not break the GPU leg
         out["cpu_baseline"] = {"unavailable": str(e)}
     return out

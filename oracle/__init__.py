@@ -38,7 +38,7 @@ DT_BF16, DT_FP16, DT_FP32 = 0, 1, 2
 def build(force: bool = False) -> str:
     """Compile the oracle with gcc (plain C, IEEE fp, no fast-math)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        cmd = ["gcc", "-O2", "-fno-fast-math", "-ffp-contract=off", "-fPIC", "-shared",
+        cmd = ["gcc", "-O2", "-fno-fast-math", "-ffp-contract=off", "-fPIC", "-shared", "-fopenmp",
                "-fvisibility=hidden", "-std=c11", "-o", _LIB, _SRC, "-lm"]
         subprocess.check_call(cmd)
     return _LIB
@@ -74,6 +74,7 @@ def lib():
             ("ft2o_protected_linear", None, [P, i64, P, i64, P, i32, i32, i32, P, i64, P, P, i32, P,
                                              P, i32, i32, i32, P]),
             ("ft2o_site_size", i32, []),
+            ("ft2o_set_threads", None, [i32]), ("ft2o_max_threads", i32, []),
             ("ft2o_nan_vulnerable_count", None, [P, i64, i64, i64, P, i32, P, ctypes.c_int]),
             ("ft2o_isnan_dt", ctypes.c_int, [u16, ctypes.c_int]), ("ft2o_isinf_dt", ctypes.c_int, [u16, ctypes.c_int]),
             ("ft2o_isfinite_dt", ctypes.c_int, [u16, ctypes.c_int]),
@@ -176,6 +177,13 @@ def bounds_from_keys(raw_keys, scale: float = 2.0, dtype=DT_BF16):
     b = np.zeros((S, 2), np.uint16)
     lib().ft2o_bounds_from_keys_dt(_p(k), S, scale, _p(b), dtype)
     return b
+
+
+def set_threads(n: int) -> int:
+    """OpenMP threads for the oracle's loops over independent outputs (results
+    are identical for any count); n < 1 = all cores.  Returns the count now in use."""
+    lib().ft2o_set_threads(int(n))
+    return int(lib().ft2o_max_threads())
 
 
 def protect(y, bounds_, row_to_seq=None, count=None, dtype=DT_BF16):

@@ -22,6 +22,9 @@
 #include <math.h>
 #include <stdint.h>
 #include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 #define EXPORT __attribute__((visibility("default")))
 
@@ -157,19 +160,45 @@ EXPORT uint16_t ft2o_clip_value(uint16_t y, uint16_t lo, uint16_t hi) { return f
 EXPORT void ft2o_protect_dt(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
                             const int32_t* row_to_seq, const uint16_t* bounds,
                             int32_t num_seqs, uint32_t* count, int dtype) {
+    /* rows are independent; a row's corrections are added to its sequence's
+     * count once (integer sum: any order gives the same count) */
+#pragma omp parallel for schedule(static)
     for (int64_t r = 0; r < rows; ++r) {
         int32_t s = row_to_seq ? row_to_seq[r] : (num_seqs == 1 ? 0 : (int32_t)r);
         if (s < 0 || s >= num_seqs) continue;
         uint16_t lo = bounds[2 * s], hi = bounds[2 * s + 1];
+        uint32_t changed = 0;
         for (int64_t j = 0; j < n; ++j) {
             uint16_t v = y[r * ld + j];
             uint16_t w = ft2o_clip_value_dt(v, lo, hi, dtype);
             if (w != v) {
                 y[r * ld + j] = w;
-                if (count) count[s] += 1;
+                changed += 1;
             }
         }
+        if (count && changed) {
+#pragma omp atomic
+            count[s] += changed;
+        }
     }
+}
+
+/* Threads the oracle's loops over independent outputs may use (OpenMP; every
+ * result is identical for any count: each output is computed by one thread
+ * in the stated order).  n < 1 restores the default. */
+EXPORT void ft2o_set_threads(int32_t n) {
+#ifdef _OPENMP
+    omp_set_num_threads(n >= 1 ? n : omp_get_num_procs());
+#else
+    (void)n;
+#endif
+}
+EXPORT int32_t ft2o_max_threads(void) {
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
 }
 EXPORT void ft2o_protect(uint16_t* y, int64_t rows, int64_t n, int64_t ld, const int32_t* row_to_seq,
                          const uint16_t* bounds, int32_t num_seqs, uint32_t* count) {
@@ -195,6 +224,8 @@ EXPORT void ft2o_bounds_dt(uint16_t* y, int64_t rows, int64_t n, int64_t ld,
                            const int32_t* seq_offsets, int32_t num_seqs, float scale,
                            int32_t correct_nonfinite, uint16_t* bounds, int32_t* raw_keys,
                            uint32_t* nonfinite, int dtype) {
+    /* sequences are independent (one thread each) */
+#pragma omp parallel for schedule(dynamic)
     for (int32_t s = 0; s < num_seqs; ++s) {
         int64_t r0 = seq_offsets ? seq_offsets[s] : 0;
         int64_t r1 = seq_offsets ? seq_offsets[s + 1] : rows;
@@ -400,6 +431,8 @@ EXPORT void ft2o_inject(uint16_t* y, int64_t rows, int64_t n, int64_t ld, const 
 EXPORT void ft2o_linear_f64_dt(const uint16_t* x, int64_t ldx, const uint16_t* w, int64_t ldw,
                                const uint16_t* bias, int32_t M, int32_t N, int32_t K,
                                double* y_f64, uint16_t* y_out, int64_t ldy, int dtype) {
+    /* every output element is one thread's sequential k = 0..K-1 sum */
+#pragma omp parallel for collapse(2) schedule(static)
     for (int32_t m = 0; m < M; ++m) {
         for (int32_t j = 0; j < N; ++j) {
             double acc = 0.0;

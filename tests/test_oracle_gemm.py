@@ -58,3 +58,27 @@ def test_protected_linear_order_inject_then_check():
     c = oracle.protect(ref, bnd, row_to_seq=np.zeros(M, np.int32))
     assert np.array_equal(y, ref) and cnt.tolist() == c.tolist()
     assert cnt[0] >= 1                           # the flipped value was out of [-2, 2] or NaN
+
+
+def test_oracle_results_do_not_depend_on_thread_count():
+    """The oracle's OpenMP loops run over independent outputs (each computed by
+    one thread in the stated order): 1 thread and all threads give identical
+    bits, counts and keys."""
+    import ft2_synth
+    x = ft2_synth.gen_bf16((7, 136), 1, 2)
+    w = ft2_synth.gen_bf16((200, 136), 2, 2, scale_log2=-4)
+    b = ft2_synth.gen_bf16((200,), 3, 2)
+    y = ft2_synth.plant_edge_values(ft2_synth.gen_bf16((64, 264), 4, 2))
+    so = np.array([0, 5, 5, 30, 64], np.int32)
+    out = []
+    for n in (1, 0):
+        oracle.set_threads(n)
+        d, lb = oracle.linear_f64(x, w, b)
+        yy = y.copy()
+        bnd, keys, nf = oracle.bounds(yy, seq_offsets=so, correct_nonfinite=True)
+        z = y.copy()
+        cnt = oracle.protect(z, bnd, row_to_seq=np.repeat(np.arange(4, dtype=np.int32), [5, 0, 25, 34]))
+        out.append((d.tobytes(), lb.tobytes(), yy.tobytes(), bnd.tobytes(), keys.tobytes(), nf.tobytes(),
+                    z.tobytes(), cnt.tobytes()))
+    oracle.set_threads(0)
+    assert out[0] == out[1]
