@@ -492,6 +492,8 @@ def main():
         rf["share_of_decode_step"] = rf["launches_per_graph"] * rf["avg_launch_us"] / dec_us
     if not args.no_extras:
         res["coverage_overhead_pct"] = coverage_costs(cfg, B, T, G, dev, prompt, stream, runner, ms_off)
+        res["c2_matrix"] = c2_matrix(dev, args)
+        res["protect_sweep"] = protect_sweep(dev, ft2, load_peaks())
     if not args.no_extras:
         # the paths that shard, at this run's N: configs[3]'s
         # TP bounds + row-parallel check, configs[4]'s campaign with its trial
@@ -1284,6 +1286,189 @@ def c3_decode_gemm(dev, ft2, peaks, M=32, copies=8, R=10, rounds=5):
                     "cublas_protect_vs_cublas_pct": 100.0 * (tot["cublas_protect"] / tot["cublas"] - 1.0),
                     "roofline": {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                                  "frac": ach / hbm_peak}}
+    out["oracle_beside"] = oracle_gemm_beside(M, 4096, 4096)
+    return out
+
+
+def oracle_gemm_beside(M, N, K):
+    """The oracle's fp64 linear + check (R8 -> R5) on one C3 shape, single
+    thread and all host cores (oracle timed beside C3)."""
+    try:
+        import ft2_synth
+        import oracle
+        x = ft2_synth.gen_bf16((M, K), 20, 1)
+        w = ft2_synth.gen_bf16((N, K), 21, 1, scale_log2=ft2_synth.weight_scale_log2(K))
+        bnd = oracle.bounds(ft2_synth.gen_bf16((16, N), 22, 1))[0]
+        out = {"shape": [M, N, K], **host_cpu()}
+        for label, th in (("single_thread", 1), ("all_cores", 0)):
+            cores = oracle.set_threads(th)
+            t0 = time.perf_counter()
+            oracle.protected_linear(x, w, None, bnd)
+            dt = time.perf_counter() - t0
+            out[label] = {"s": dt, "cores": cores, "GFLOPs": 2.0 * M * N * K / dt / 1e9}
+        return out
+    except Exception as e:   # the oracle is test infrastructure; never breaks a GPU leg
+        return {"unavailable": str(e)}
+
+
+def protect_sweep(dev, ft2, peaks, R=10):
+    """SURVEY.md 8(d) protection-kernel sweep: ft2_bounds_from_prefill and
+    ft2_protect on [rows, N] bf16 tensors of 1 MB .. 4 GB, N in {2048, 4096,
+    11008}, cold L2 (every repetition reads a different slice of a >= 1 GB
+    pool, or the 4 GB tensor itself); algorithmic bytes = 2 B read per element.
+    Plus decode-sized calls (L2-resident, us per call, back to back in a CUDA
+    graph) and the oracle's GB/s on a 64 MB tensor beside it."""
+    import torch
+
+    import ft2_synth
+
+    hbm_peak = (peaks or {}).get("hbm_gbs", 6650.0)
+    stream = torch.cuda.current_stream()
+    pool_bytes = 1 << 30
+    pool = ft2_synth.gen_bf16_torch((pool_bytes // 2,), 61, 3, device=dev)
+    ws = ft2.make_workspace(1, device=dev)
+    bnd = torch.zeros((1, 2), dtype=torch.bfloat16, device=dev)
+    wide = torch.tensor([[-3.0e38, 3.0e38]], dtype=torch.bfloat16, device=dev)
+    cnt = torch.zeros(1, dtype=torch.int32, device=dev)
+
+    def timed(fn_list, graph=True):
+        """us per call of the calls in fn_list, back to back (one CUDA graph)."""
+        for f in fn_list[:2]:
+            f()
+        torch.cuda.synchronize()
+        run = None
+        if graph:
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                for f in fn_list:
+                    f()
+            g.replay()
+            run = g.replay
+        else:
+            def run():
+                for f in fn_list:
+                    f()
+        torch.cuda.synchronize()
+        a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        run()
+        b_.record(stream)
+        torch.cuda.synchronize()
+        return 1000.0 * a.elapsed_time(b_) / len(fn_list)
+
+    rows_out = []
+    for mb in (1, 4, 16, 64, 256, 1024, 4096):
+        for n in (2048, 4096, 11008):
+            rows = max(1, (mb << 20) // (2 * n))
+            nbytes = rows * n * 2
+            if nbytes <= pool_bytes // 2:
+                nsl = pool.numel() // (rows * n)
+                views = [pool[i * rows * n:(i + 1) * rows * n].view(rows, n) for i in range(nsl)]
+                reps = [views[i % nsl] for i in range(max(R, min(4 * nsl, 200)))]
+                big = None
+            else:
+                big = ft2_synth.gen_bf16_torch((rows, n), 62, 3, device=dev)
+                reps = [big] * R
+            us_b = timed([lambda y=y: ft2.bounds_from_prefill(y, bnd, ws) for y in reps])
+            us_p = timed([lambda y=y: ft2.protect(y, wide, corrected_count=cnt) for y in reps])
+            rows_out.append({"MB": round(nbytes / 2 ** 20, 2), "shape": [rows, n],
+                             "bounds_us": round(us_b, 2), "bounds_GBps": round(nbytes / us_b / 1e3, 1),
+                             "bounds_frac": round(nbytes / us_b / 1e3 / hbm_peak, 3),
+                             "protect_us": round(us_p, 2), "protect_GBps": round(nbytes / us_p / 1e3, 1),
+                             "protect_frac": round(nbytes / us_p / 1e3 / hbm_peak, 3)})
+            del big, reps
+    torch.cuda.empty_cache()
+    # decode-sized calls: L2-resident, back to back in one graph
+    dec = {}
+    for rows, n in ((1, 2048), (32, 2048), (32, 4096), (32, 11008)):
+        ys = [ft2_synth.gen_bf16_torch((rows, n), 70 + i, 3, device=dev) for i in range(8)]
+        bb = wide.repeat(rows, 1)
+        cc = torch.zeros(rows, dtype=torch.int32, device=dev)
+
+        def body():
+            for y in ys:
+                ft2.protect(y, bb, corrected_count=cc)
+        body()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            body()
+        us = timed([g.replay] * 20, graph=False) / len(ys)
+        dec[f"{rows}x{n}"] = round(us, 3)
+    out = {"sweep": rows_out, "decode_calls_us": dec, "peak": hbm_peak, "l2": "cold (rotating slices of a 1 GB "
+           "pool, or one tensor > L2)", "algorithmic_bytes": "2 B read per element"}
+    try:
+        import numpy as np
+
+        import oracle
+        y = pool[:32 << 20].cpu().view(torch.int16).numpy().view(np.uint16).reshape(-1, 4096)
+        so = np.linspace(0, y.shape[0], 33).astype(np.int32)
+        wb = np.array([[0xFF7F, 0x7F7F]] * 32, np.uint16)   # +-max finite: nothing clips
+        r2s = np.repeat(np.arange(32, dtype=np.int32), np.diff(so))
+        ob = {**host_cpu(), "shape": list(y.shape), "sequences": 32}
+        for label, th in (("single_thread", 1), ("all_cores", 0)):
+            cores = oracle.set_threads(th)
+            yy = y.copy()
+            t0 = time.perf_counter()
+            oracle.bounds(yy, seq_offsets=so)
+            t1 = time.perf_counter()
+            oracle.protect(yy, wb, row_to_seq=r2s)
+            t2 = time.perf_counter()
+            ob[label] = {"cores": cores, "bounds_GBps": y.nbytes / (t1 - t0) / 1e9,
+                         "protect_GBps": y.nbytes / (t2 - t1) / 1e9}
+        out["oracle_beside"] = ob
+    except Exception as e:
+        out["oracle_beside"] = {"unavailable": str(e)}
+    del pool
+    torch.cuda.empty_cache()
+    return out
+
+
+def c2_matrix(dev, args, rounds=5):
+    """SURVEY.md 8(d) C2 beyond the headline: OPT-1.3B-shaped decode at B = 1
+    (the paper's one-input-per-inference setting) and
+    B = 32, 60 (QA) and 180 (math) generated tokens (L284), and the paper's
+    FP16 (L282) at the headline shape.  Per variant: protected (fused) vs
+    unprotected (off) and fused_plain tokens/s, medians of `rounds` interleaved
+    requests."""
+    import torch
+
+    from paper_conf_hpdc_sunzmg00y25_b200.runner import CONFIGS, Runner
+
+    cfg = CONFIGS[args.model]
+    stream = torch.cuda.current_stream()
+    out = {}
+    for B, G, dt in ((1, 60, torch.bfloat16), (1, 180, torch.bfloat16), (32, 180, torch.bfloat16),
+                     (32, 60, torch.float16)):
+        r = Runner(cfg, B, args.prompt, G, seed=1, device=dev, dtype=dt)
+        gen = torch.Generator().manual_seed(1234)
+        prompt = torch.randint(0, cfg.vocab, (B, args.prompt), generator=gen).to(dev)
+        modes = ("fused", "off", "fused_plain")
+        for m in modes:
+            for _ in range(3):
+                r.generate(prompt, m)
+        samples = {m: [] for m in modes}
+        for i in range(rounds):
+            r.generate(prompt, "off")
+            evs = []
+            for m in modes[i % 3:] + modes[:i % 3]:
+                a, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                r.generate(prompt, m)
+                b_.record(stream)
+                evs.append((m, a, b_))
+            torch.cuda.synchronize()
+            for m, a, b_ in evs:
+                samples[m].append(a.elapsed_time(b_))
+        med = {m: statistics.median(v) for m, v in samples.items()}
+        key = f"B{B}_gen{G}_{'fp16' if dt == torch.float16 else 'bf16'}"
+        out[key] = {"tokens_per_s": {m: B * G / (v / 1e3) for m, v in med.items()},
+                    "ms_per_request": med,
+                    "overhead_pct_vs_unprotected": 100.0 * (1 - med["off"] / med["fused"]),
+                    "epilogue_overhead_pct": 100.0 * (1 - med["fused_plain"] / med["fused"])}
+        del r
+        torch.cuda.empty_cache()
+    out["note"] = "medians of interleaved requests (mode order rotated); off = cuBLAS, fused_plain = same GEMM without the check"
     return out
 
 

@@ -223,8 +223,17 @@ def ipc_close(base: int):
 
 def host_norm(x, w, y, bias=None, eps=1e-5, rms=False, stream=None):
     """Host-model LayerNorm / RMSNorm over the last dim of 2-D x into y
-    (include/ft2.h ft2_host_norm; not part of the FT2 method)."""
+    (include/ft2.h ft2_host_norm; not part of the FT2 method).  Raises
+    ValueError when the tensors disagree (dtype, widths, rows): the C ABI only
+    sees pointers and leading dimensions."""
     n = x.shape[-1]
+    if x.dim() != 2 or y.dim() != 2 or x.stride(-1) != 1 or y.stride(-1) != 1:
+        raise ValueError("host_norm: x and y must be 2-D with unit inner stride")
+    for name, t in (("w", w), ("bias", bias), ("y", y)):
+        if t is not None and t.dtype != x.dtype:
+            raise ValueError(f"host_norm: {name} is {t.dtype}, x is {x.dtype}")
+    if w.numel() < n or (bias is not None and bias.numel() < n) or y.shape[0] < x.shape[0] or y.shape[1] < n:
+        raise ValueError("host_norm: w / bias narrower than x, or y smaller than x")
     check("ft2_host_norm", load().ft2_host_norm(_ptr(x), x.stride(0), _ptr(w), _ptr(bias), _ptr(y), y.stride(0),
                                                 x.shape[0], n, float(eps), int(rms), _dtype_of(x), _stream(stream)))
     return y
@@ -232,8 +241,16 @@ def host_norm(x, w, y, bias=None, eps=1e-5, rms=False, stream=None):
 
 def host_act(a, y, b=None, act="relu", stream=None):
     """Host-model MLP activation into y: relu(a), or silu(a) * b with
-    act="silu_mul" (include/ft2.h ft2_host_act; not part of the FT2 method)."""
+    act="silu_mul" (include/ft2.h ft2_host_act; not part of the FT2 method).
+    Raises ValueError when the tensors disagree (dtype, shape)."""
     code = {"relu": 0, "silu_mul": 1}[act]
+    if a.dim() != 2 or y.dim() != 2 or a.stride(-1) != 1 or y.stride(-1) != 1:
+        raise ValueError("host_act: a and y must be 2-D with unit inner stride")
+    if y.dtype != a.dtype or y.shape[0] < a.shape[0] or y.shape[1] < a.shape[1]:
+        raise ValueError("host_act: y must match a's dtype and cover its shape")
+    if code == 1 and (b is None or b.dim() != 2 or b.dtype != a.dtype or tuple(b.shape) != tuple(a.shape)
+                      or b.stride(-1) != 1):
+        raise ValueError("host_act: silu_mul needs b with a's dtype and shape")
     check("ft2_host_act", load().ft2_host_act(_ptr(a), a.stride(0), _ptr(b), b.stride(0) if b is not None else 0,
                                               _ptr(y), y.stride(0), a.shape[0], a.shape[-1], code, _dtype_of(a),
                                               _stream(stream)))

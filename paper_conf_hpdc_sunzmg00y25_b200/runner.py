@@ -108,21 +108,23 @@ CONFIGS = {
 }
 
 
-def _w(shape, tau, seed, device, K=None, outliers=True):
+def _w(shape, tau, seed, device, K=None, outliers=True, dtype=torch.bfloat16):
     sl = ft2_synth.weight_scale_log2(K) if K else 0
-    return ft2_synth.gen_bf16_torch(shape, tau, seed, scale_log2=sl, device=device, outliers=outliers)
+    t = ft2_synth.gen_bf16_torch(shape, tau, seed, scale_log2=sl, device=device, outliers=outliers)
+    return t if dtype == torch.bfloat16 else t.to(dtype)   # FP16 model: the same values, rounded
 
 
 class Block:
-    def __init__(self, cfg: ModelConfig, idx: int, seed: int, device, outliers: bool = True):
+    def __init__(self, cfg: ModelConfig, idx: int, seed: int, device, outliers: bool = True,
+                 dtype=torch.bfloat16):
         self.cfg = cfg
         self.idx = idx
         tau0 = 1000 + 64 * idx
         self.w = {}
         self.b = {}
         for j, (name, o, i, _) in enumerate(cfg.linears()):
-            self.w[name] = _w((o, i), tau0 + 2 * j, seed, device, K=i, outliers=outliers)
-            self.b[name] = _w((o,), tau0 + 2 * j + 1, seed, device, outliers=outliers) if cfg.bias else None
+            self.w[name] = _w((o, i), tau0 + 2 * j, seed, device, K=i, outliers=outliers, dtype=dtype)
+            self.b[name] = _w((o,), tau0 + 2 * j + 1, seed, device, outliers=outliers, dtype=dtype) if cfg.bias else None
         # horizontally fused projections (same weights; the per-layer tensors
         # become views into the fused ones): qkv, and Llama's gate_up
         self.groups = {"qkv": ["q_proj", "k_proj", "v_proj"]}
@@ -140,17 +142,17 @@ class Block:
                     self.b[n] = self.bf[g][r0:r0 + o]
                 r0 += o
         h = cfg.hidden
-        self.ln1_w = torch.ones(h, dtype=torch.bfloat16, device=device)
-        self.ln2_w = torch.ones(h, dtype=torch.bfloat16, device=device)
-        self.ln1_b = torch.zeros(h, dtype=torch.bfloat16, device=device) if cfg.arch == "opt" else None
-        self.ln2_b = torch.zeros(h, dtype=torch.bfloat16, device=device) if cfg.arch == "opt" else None
+        self.ln1_w = torch.ones(h, dtype=dtype, device=device)
+        self.ln2_w = torch.ones(h, dtype=dtype, device=device)
+        self.ln1_b = torch.zeros(h, dtype=dtype, device=device) if cfg.arch == "opt" else None
+        self.ln2_b = torch.zeros(h, dtype=dtype, device=device) if cfg.arch == "opt" else None
 
 
 class FT2State:
     """Per-request FT2 state: bounds [L_crit, B, 2], counters, workspace."""
 
-    def __init__(self, n_crit: int, B: int, device):
-        self.bounds = torch.zeros((n_crit, B, 2), dtype=torch.bfloat16, device=device)
+    def __init__(self, n_crit: int, B: int, device, dtype=torch.bfloat16):
+        self.bounds = torch.zeros((n_crit, B, 2), dtype=dtype, device=device)
         self.keys = torch.zeros((n_crit, B, 2), dtype=torch.int32, device=device)
         self.corrected = torch.zeros((n_crit, B), dtype=torch.int32, device=device)
         self.nonfinite = torch.zeros((n_crit, B), dtype=torch.int32, device=device)
@@ -166,7 +168,7 @@ class Runner:
 
     def __init__(self, cfg: ModelConfig, batch: int, prompt_len: int, gen_len: int, seed: int = 1,
                  device="cuda", scale: float = 2.0, coverage: str = "ft2", fuse_proj: bool | None = None,
-                 share: "Runner | None" = None, outliers: bool = True):
+                 share: "Runner | None" = None, outliers: bool = True, dtype=torch.bfloat16):
         """share: another Runner of the same config, batch and lengths whose
         weights, KV caches and static token / site buffers this one reuses
         (no copy; see with_coverage).  Runners sharing buffers must not run
@@ -174,7 +176,11 @@ class Runner:
         the synthetic recipe's planted 2**-10 outliers: the
         fault-injection campaign's model, whose fault-free activation range is
         stable from the first token on (the premise of first-token bounds,
-        PAPER.md L223-L233), unlike the heavy-tailed outlier model."""
+        PAPER.md L223-L233), unlike the heavy-tailed outlier model.  dtype:
+        torch.bfloat16 (BASELINE) or torch.float16 (the paper's precision,
+        PAPER.md L282) for the whole model, FT2's kernels and bounds included."""
+        assert dtype in (torch.bfloat16, torch.float16), dtype
+        self.dt = dtype
         self.cfg = cfg
         self.B = batch
         self.T = prompt_len
@@ -185,16 +191,18 @@ class Runner:
         dv = self.device
         h = cfg.hidden
         if share is not None:
-            assert (share.cfg, share.B, share.T, share.G) == (cfg, batch, prompt_len, gen_len)
+            assert (share.cfg, share.B, share.T, share.G, share.dt) == (cfg, batch, prompt_len, gen_len, dtype)
             for a in ("embed", "pos_embed", "blocks", "lnf_w", "lnf_b", "lm_head"):
                 setattr(self, a, getattr(share, a))
         else:
-            self.embed = _w((cfg.vocab, h), 1, seed, dv, outliers=outliers)
-            self.pos_embed = _w((cfg.max_pos + 2, h), 2, seed, dv, outliers=outliers) if cfg.arch == "opt" else None
-            self.blocks = [Block(cfg, i, seed, dv, outliers=outliers) for i in range(cfg.n_layers)]
-            self.lnf_w = torch.ones(h, dtype=torch.bfloat16, device=dv)
-            self.lnf_b = torch.zeros(h, dtype=torch.bfloat16, device=dv) if cfg.arch == "opt" else None
-            self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h, outliers=outliers)
+            self.embed = _w((cfg.vocab, h), 1, seed, dv, outliers=outliers, dtype=dtype)
+            self.pos_embed = _w((cfg.max_pos + 2, h), 2, seed, dv, outliers=outliers, dtype=dtype) \
+                if cfg.arch == "opt" else None
+            self.blocks = [Block(cfg, i, seed, dv, outliers=outliers, dtype=dtype) for i in range(cfg.n_layers)]
+            self.lnf_w = torch.ones(h, dtype=dtype, device=dv)
+            self.lnf_b = torch.zeros(h, dtype=dtype, device=dv) if cfg.arch == "opt" else None
+            self.lm_head = self.embed if cfg.arch == "opt" else _w((cfg.vocab, h), 3, seed, dv, K=h,
+                                                                   outliers=outliers, dtype=dtype)
         self.coverage = coverage
         # fuse_proj: fused q/k/v (and Llama gate/up) projections, one GEMM per
         # group; the protected layer of a group (v_proj, up_proj) is a column
@@ -227,7 +235,7 @@ class Runner:
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
-        self.state = FT2State(self.n_crit, batch, dv)
+        self.state = FT2State(self.n_crit, batch, dv, dtype)
         H, D = cfg.n_heads, cfg.head_dim
         # buffers a with_coverage() clone shares with its parent (graphs bake in
         # their addresses; runs are sequential on one stream)
@@ -237,9 +245,9 @@ class Runner:
             for a in shared:
                 setattr(self, a, getattr(share, a))
         else:
-            self.k_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
+            self.k_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=dtype, device=dv)
                             for _ in range(cfg.n_layers)]
-            self.v_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=torch.bfloat16, device=dv)
+            self.v_cache = [torch.zeros((batch, H, self.Tmax, D), dtype=dtype, device=dv)
                             for _ in range(cfg.n_layers)]
             self.seq_offsets = torch.arange(0, (batch + 1) * prompt_len, prompt_len, dtype=torch.int32, device=dv)
             # prefill row -> sequence (supplied-bounds check of the first token)
@@ -255,7 +263,7 @@ class Runner:
             self.cur_step = torch.zeros(1, dtype=torch.int32, device=dv)
             # last-position hidden state (before the final norm) of every generated
             # token [G, B, hidden]: the campaign's deviation proxy reads it
-            self.h_trace = torch.zeros((gen_len, batch, h), dtype=torch.bfloat16, device=dv)
+            self.h_trace = torch.zeros((gen_len, batch, h), dtype=dtype, device=dv)
         self.graph_prefill = True   # first-token pass as a CUDA graph (False: eager)
         self.sites = None        # optional fault sites (uint8 [B*24]); site i = sequence i
         # caller-supplied ("offline") bounds [n_crit, B, 2] (set_supplied_bounds):
@@ -273,8 +281,8 @@ class Runner:
             inv = 1.0 / (10000 ** (torch.arange(0, D, 2, device=dv, dtype=torch.float32) / D))
             t = torch.arange(self.Tmax, device=dv, dtype=torch.float32)
             fr = torch.outer(t, inv)
-            self.rope_cos = torch.cat([fr.cos(), fr.cos()], -1).to(torch.bfloat16)
-            self.rope_sin = torch.cat([fr.sin(), fr.sin()], -1).to(torch.bfloat16)
+            self.rope_cos = torch.cat([fr.cos(), fr.cos()], -1).to(dtype)
+            self.rope_sin = torch.cat([fr.sin(), fr.sin()], -1).to(dtype)
 
     # ------------------------------------------------------------ helpers
     def _norm(self, x, w, b):
@@ -284,9 +292,12 @@ class Runner:
             if x2.stride(-1) != 1:
                 x2 = x2.contiguous()
             y = torch.empty((x2.shape[0], n), dtype=x.dtype, device=x.device)
-            F2.host_norm(x2, w, y, bias=b if self.cfg.arch == "opt" else None,
-                         eps=1e-5 if self.cfg.arch == "opt" else 1e-6, rms=self.cfg.arch != "opt")
-            return y.view(*x.shape[:-1], n)
+            try:
+                F2.host_norm(x2, w, y, bias=b if self.cfg.arch == "opt" else None,
+                             eps=1e-5 if self.cfg.arch == "opt" else 1e-6, rms=self.cfg.arch != "opt")
+                return y.view(*x.shape[:-1], n)
+            except ValueError:   # tensors the host kernel does not take: torch's norm
+                pass
         if self.cfg.arch == "opt":
             return F.layer_norm(x, (x.shape[-1],), w, b, 1e-5)
         return F.rms_norm(x, (x.shape[-1],), w, 1e-6)
@@ -302,7 +313,10 @@ class Runner:
                 a.stride(-1) == 1 and \
                 (b is None or (b.dim() == 2 and b.stride(-1) == 1)):
             y = torch.empty((a.shape[0], n), dtype=a.dtype, device=a.device)
-            return F2.host_act(a, y, b=b, act="relu" if b is None else "silu_mul")
+            try:
+                return F2.host_act(a, y, b=b, act="relu" if b is None else "silu_mul")
+            except ValueError:   # tensors the host kernel does not take: torch's op
+                pass
         return torch.relu(a) if b is None else F.silu(a) * b
 
     def _rope(self, x, pos_idx):
@@ -384,7 +398,7 @@ class Runner:
             return y
         cid = self._crit_id(blk.idx, name)
         st = self.state
-        y = torch.empty((x2.shape[0], w.shape[0]), dtype=torch.bfloat16, device=x2.device)
+        y = torch.empty((x2.shape[0], w.shape[0]), dtype=self.dt, device=x2.device)
         mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
         F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, bounds=st.bounds[cid], num_seqs=self.B,
                               corrected_count=st.corrected[cid], sites=sites, n_sites=self.B if sites is not None else None,
@@ -456,7 +470,7 @@ class Runner:
                                        nonfinite_count=st.nonfinite[cid])
         elif ci is not None and self.mode in ("fused", "fused_plain") and M <= FUSED_MAX_M:
             cid = self._crit_id(blk.idx, names[ci])
-            y = torch.empty((M, w.shape[0]), dtype=torch.bfloat16, device=x2.device)
+            y = torch.empty((M, w.shape[0]), dtype=self.dt, device=x2.device)
             mode = (FT2_GEMM_CHECK if self.mode == "fused" else FT2_GEMM_PLAIN) | FT2_GEMM_W_STATIC
             F2.protect_fused_gemm(x2, w, y, bias=b, mode=mode, col_begin=offs[ci], col_end=offs[ci + 1],
                                   bounds=st.bounds[cid], num_seqs=self.B, corrected_count=st.corrected[cid],
@@ -545,7 +559,7 @@ class Runner:
         """One decode step on static buffers (graph-capturable)."""
         pidx = self.pos.view(1, 1).expand(self.B, 1)
         ar = torch.arange(self.Tmax, device=self.device)
-        self._mask = torch.where(ar <= self.pos, 0.0, float("-inf")).to(torch.bfloat16).view(1, 1, 1, -1)
+        self._mask = torch.where(ar <= self.pos, 0.0, float("-inf")).to(self.dt).view(1, 1, 1, -1)
         x = self._embed(self.tok.view(self.B, 1), pidx)
         for blk in self.blocks:
             x = self._block(blk, x, "decode", pos_idx=pidx, step=self._site_step)
@@ -561,7 +575,7 @@ class Runner:
         SAME weights, caches and site buffer (no copy): its own bounds,
         counters and CUDA graphs.  Used for paired coverage comparisons."""
         return Runner(self.cfg, self.B, self.T, self.G, device=self.device, scale=self.scale, coverage=coverage,
-                      fuse_proj=self.fuse_proj, share=self)
+                      fuse_proj=self.fuse_proj, share=self, dtype=self.dt)
 
     def set_supplied_bounds(self, bounds):
         """Caller-supplied ("offline") bounds, bf16 [n_crit, B, 2] or [n_crit, 2]
@@ -573,7 +587,7 @@ class Runner:
         if bounds is None:
             self.supplied_bounds = None
             return
-        b = bounds.to(device=self.device, dtype=torch.bfloat16)
+        b = bounds.to(device=self.device, dtype=self.dt)
         if b.dim() == 2:
             b = b.unsqueeze(1).expand(self.n_crit, self.B, 2)
         assert tuple(b.shape) == (self.n_crit, self.B, 2), b.shape
@@ -595,7 +609,7 @@ class Runner:
                 self.prefill(ids.to(self.device))
         finally:
             self.mode = mode
-        out = torch.zeros((self.n_crit, 2), dtype=torch.bfloat16, device=self.device)
+        out = torch.zeros((self.n_crit, 2), dtype=self.dt, device=self.device)
         F2.bounds_finalize(self._profile_keys, out, scale=self.scale if scale is None else scale)
         self._profile_keys = None
         return out

@@ -104,3 +104,22 @@ def test_fused_gemm_ex_prefetch_hint_validation(L):
     assert ex(P(0x4000), 24) == FT2_ERR_MISALIGNED      # size not a multiple of 16
     assert ex(P(0x4000), 32, dtype=2) == FT2_ERR_UNSUPPORTED   # then the ft2_protect_fused_gemm checks
     assert ex(None, 0, dtype=2) == FT2_ERR_UNSUPPORTED
+
+
+def test_host_kernel_wrappers_reject_mismatched_tensors():
+    """the host-model wrappers check what the C ABI cannot see
+    (dtypes, widths, shapes) before any launch."""
+    import torch
+    from paper_conf_hpdc_sunzmg00y25_b200 import ft2
+    x = torch.zeros((4, 16), dtype=torch.bfloat16)
+    y = torch.zeros((4, 16), dtype=torch.bfloat16)
+    with pytest.raises(ValueError):
+        ft2.host_norm(x, torch.ones(16, dtype=torch.float32), y)           # fp32 weight read as bf16
+    with pytest.raises(ValueError):
+        ft2.host_norm(x, torch.ones(8, dtype=torch.bfloat16), y)           # narrow weight
+    with pytest.raises(ValueError):
+        ft2.host_norm(x, torch.ones(16, dtype=torch.bfloat16), torch.zeros((2, 16), dtype=torch.bfloat16))
+    with pytest.raises(ValueError):
+        ft2.host_act(x, y, b=torch.zeros((4, 8), dtype=torch.bfloat16), act="silu_mul")   # narrow b
+    with pytest.raises(ValueError):
+        ft2.host_act(x, torch.zeros((4, 16), dtype=torch.float16))        # y dtype
