@@ -18,6 +18,11 @@
 //      stored to this rank's own output;
 //   4. the last CTA bumps the rank's epoch counter (device memory, so the
 //      kernel is CUDA-graph replayable).
+// P = 1 needs none of 1, 2 and 4 (stream order covers the own partial): the
+// kernel is then a plain elementwise pass.  The P partial vectors of an
+// output vector are all loaded before the fp32 sum (P NVLink round trips in
+// flight at once, not one after another), and a thread owns up to kVecs
+// output vectors.
 //
 // The partial buffers must be double-buffered by the caller (alternate per
 // call): a rank reaches call e+1's signal only after its call e finished
@@ -38,6 +43,8 @@ namespace {
 
 constexpr int kARThreads = 256;
 constexpr int kARSites = 64;
+constexpr int kARMaxP = 8;   // ranks whose partials one thread holds in registers at once
+constexpr int kVecs = 2;     // output vectors per thread per pass
 
 __device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
@@ -113,41 +120,63 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     __syncthreads();
     if (sh_ok) {
         const uint32_t nsite = min(sh_ns, (uint32_t)kARSites);
-        for (uint32_t v = v0 + tid; v < v1; v += kARThreads) {
-            const uint32_t row = fdiv(v, div_n8), c8 = v - row * n8;
-            float acc[8];
-            for (int t = 0; t < p.P; ++t)
-                add8<DT>(acc, ld_peer_v4(p.partials[t] + (int64_t)row * p.ldp + c8 * 8), t == 0);
-            if (p.bias) {
-                const uint4 b = *reinterpret_cast<const uint4*>(p.bias + c8 * 8);
-                const uint32_t bw[4] = {b.x, b.y, b.z, b.w};
+        for (uint32_t vb = v0 + tid; vb < v1; vb += kARThreads * kVecs) {
+            // issue every load of this pass first: kVecs vectors x min(P, 8) partials
+            uint4 part[kVecs][kARMaxP];
+            uint32_t vrow[kVecs], vc8[kVecs];
 #pragma unroll
-                for (int j = 0; j < 8; ++j)
-                    acc[j] = __fadd_rn(acc[j], to_f32<DT>((uint16_t)(bw[j >> 1] >> ((j & 1) * 16))));
+            for (int q = 0; q < kVecs; ++q) {
+                const uint32_t v = vb + q * kARThreads;
+                vrow[q] = fdiv(v < v1 ? v : v0, div_n8);
+                vc8[q] = (v < v1 ? v : v0) - vrow[q] * n8;
+#pragma unroll
+                for (int t = 0; t < kARMaxP; ++t)
+                    if (t < p.P && v < v1)
+                        part[q][t] = ld_peer_v4(p.partials[t] + (int64_t)vrow[q] * p.ldp + vc8[q] * 8);
             }
-            uint32_t w[4];
 #pragma unroll
-            for (int j = 0; j < 4; ++j)
-                w[j] = (uint32_t)rne16<DT>(acc[2 * j]) | ((uint32_t)rne16<DT>(acc[2 * j + 1]) << 16);
-            for (uint32_t i = 0; i < nsite; ++i) {
-                const uint32_t d = sh_site_e[i] - (v - v0) * 8u;
-                if (d < 8u) w[d >> 1] ^= (sh_site_m[i] & 0xFFFFu) << ((d & 1) * 16);
-            }
-            if (p.mode == FT2_GEMM_CHECK) {
-                const int s = row_mode == 2 ? 0 : (row_mode == 1 ? (int)row : p.row_to_seq[row]);
-                if (s >= 0 && s < p.S) {
-                    const uint32_t k = key2(*reinterpret_cast<const uint32_t*>(p.bounds + 2 * s));
-                    const uint32_t kL2 = (k & 0xFFFFu) * 0x10001u, kH2 = (k >> 16) * 0x10001u;
-                    uint32_t cnt = 0, c;
+            for (int q = 0; q < kVecs; ++q) {
+                const uint32_t v = vb + q * kARThreads;
+                if (v >= v1) break;
+                const uint32_t row = vrow[q], c8 = vc8[q];
+                float acc[8];
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) { w[j] = clip2<DT>(w[j], kL2, kH2, &c); cnt += c; }
-                    if (cnt && p.counts) atomicAdd(&p.counts[s], cnt);
+                for (int t = 0; t < kARMaxP; ++t)
+                    if (t < p.P) add8<DT>(acc, part[q][t], t == 0);
+                for (int t = kARMaxP; t < p.P; ++t)   // rank order continues beyond 8 ranks
+                    add8<DT>(acc, ld_peer_v4(p.partials[t] + (int64_t)row * p.ldp + c8 * 8), false);
+                if (p.bias) {
+                    const uint4 b = *reinterpret_cast<const uint4*>(p.bias + c8 * 8);
+                    const uint32_t bw[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        acc[j] = __fadd_rn(acc[j], to_f32<DT>((uint16_t)(bw[j >> 1] >> ((j & 1) * 16))));
                 }
+                uint32_t w[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    w[j] = (uint32_t)rne16<DT>(acc[2 * j]) | ((uint32_t)rne16<DT>(acc[2 * j + 1]) << 16);
+                for (uint32_t i = 0; i < nsite; ++i) {
+                    const uint32_t d = sh_site_e[i] - (v - v0) * 8u;
+                    if (d < 8u) w[d >> 1] ^= (sh_site_m[i] & 0xFFFFu) << ((d & 1) * 16);
+                }
+                if (p.mode == FT2_GEMM_CHECK) {
+                    const int s = row_mode == 2 ? 0 : (row_mode == 1 ? (int)row : p.row_to_seq[row]);
+                    if (s >= 0 && s < p.S) {
+                        const uint32_t k = key2(*reinterpret_cast<const uint32_t*>(p.bounds + 2 * s));
+                        const uint32_t kL2 = (k & 0xFFFFu) * 0x10001u, kH2 = (k >> 16) * 0x10001u;
+                        uint32_t cnt = 0, c;
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) { w[j] = clip2<DT>(w[j], kL2, kH2, &c); cnt += c; }
+                        if (cnt && p.counts) atomicAdd(&p.counts[s], cnt);
+                    }
+                }
+                *reinterpret_cast<uint4*>(p.y + (int64_t)row * p.ldy + c8 * 8) = make_uint4(w[0], w[1], w[2], w[3]);
             }
-            *reinterpret_cast<uint4*>(p.y + (int64_t)row * p.ldy + c8 * 8) = make_uint4(w[0], w[1], w[2], w[3]);
         }
     }
     // ---- 4. last CTA: this rank's call is complete; advance the epoch
+    if (p.P == 1) return;   // no handshake at P = 1: the epoch is never read
     __syncthreads();
     if (tid == 0) sh_last = atom_add_acq_rel_gpu(p.done, 1u) == gridDim.x - 1;
     __syncthreads();
@@ -161,8 +190,8 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
 
 cudaError_t launch_allreduce_protect(const AllreduceProtectArgs& a, cudaStream_t st, int* n_launch) {
     const uint32_t n8 = (uint32_t)(a.n / 8), total = (uint32_t)(a.rows * (a.n / 8));
-    // one vector per thread per pass; at most 2 CTAs per SM (every CTA polls)
-    uint32_t grid = (total + kARThreads - 1) / kARThreads;
+    // kVecs vectors per thread per pass; at most 2 CTAs per SM (every CTA polls)
+    uint32_t grid = (total + kARThreads * kVecs - 1) / (kARThreads * kVecs);
     const uint32_t cap = (uint32_t)(2 * num_sms());
     grid = grid < 1 ? 1 : (grid > cap ? cap : grid);
     uint32_t chunk = (total + grid - 1) / grid;
