@@ -68,10 +68,10 @@ def parse():
 
 
 def load_traffic():
-    """dram__bytes_read.sum + dram__bytes_write.sum per launch from this round's
-    committed ncu --set full capture (profiles/r1_ncu_traffic.json)."""
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch from the
+    committed ncu --set full captures (profiles/r2_ncu_traffic.json)."""
     try:
-        return json.load(open(os.path.join(ROOT, "profiles", "r1_ncu_traffic.json")))
+        return json.load(open(os.path.join(ROOT, "profiles", "r2_ncu_traffic.json")))
     except Exception:
         return {}
 
@@ -693,7 +693,8 @@ def kernel_rooflines(runner, dev, ft2):
                    "traffic": traffic.get("bounds_65536x11008", {}).get("per_launch_bytes"), "us": 1000 * ms_b,
                    "shape": [rows, n], "algorithmic_bytes": "2 B read per element"},
         "protect": {"bound": "hbm", "achieved": nb / (ms_p / 1e3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
-                    "frac": nb / (ms_p / 1e3) / 1e9 / hbm_peak, "traffic": None, "us": 1000 * ms_p,
+                    "frac": nb / (ms_p / 1e3) / 1e9 / hbm_peak,
+                    "traffic": traffic.get("protect_65536x11008", {}).get("per_launch_bytes"), "us": 1000 * ms_p,
                     "shape": [rows, n], "algorithmic_bytes": "2 B read per element (no element out of bounds)"},
         "peak_source": peak_src,
     }

@@ -208,6 +208,10 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
  * sites/n_sites/cur_layer/cur_step/base_row  optional fault injection applied
  *              to the bf16 result before the check (order: GEMM -> bias -> bf16 ->
  *              inject -> check; readings A19, A20), as in ft2_inject_faults.
+ *              Any number of sites may land in one output tile: past the
+ *              kernel's per-CTA site list (64; the M > 128 kernel: 4 per row
+ *              per 256-column tile) it rescans every site for the affected
+ *              elements, so no site is ever dropped (only slower).
  * workspace/ws_bytes  optional, 16-byte aligned, zero-filled once before first
  *              use (every call leaves its counters zero again).  Decode shapes
  *              (M <= 128) split K across a thread-block cluster and need none.
@@ -334,6 +338,8 @@ ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t 
  * y            this rank's output [rows x n] (ld), 16-bit (bf16 / fp16).
  * bias, row_to_seq, bounds, num_seqs, corrected_count, sites, n_sites,
  * cur_layer, cur_step, base_row: as in ft2_protect_fused_gemm / ft2_protect.
+ * Sites: as ft2_inject_faults, none dropped (past 64 in one CTA's chunk the
+ * kernel rescans every site).
  * Every rank must make the same sequence of calls with the same shapes.
  * Asynchronous on stream; graph-capturable (the epoch lives in device memory). */
 ft2_status ft2_allreduce_protect(const void* const* partials, int64_t ldp, int32_t P, int32_t rank,

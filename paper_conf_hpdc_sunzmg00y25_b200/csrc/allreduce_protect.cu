@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     }
     __syncthreads();
     if (sh_ok) {
-        const uint32_t nsite = min(sh_ns, (uint32_t)kARSites);
+        const uint32_t nsite = sh_ns;   // > kARSites: every site is rescanned per vector (none dropped)
         for (uint32_t vb = v0 + tid; vb < v1; vb += kARThreads * kVecs) {
             // issue every load of this pass first: kVecs vectors x min(P, 8) partials
             uint4 part[kVecs][kARMaxP];
@@ -156,9 +156,20 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
 #pragma unroll
                 for (int j = 0; j < 4; ++j)
                     w[j] = (uint32_t)rne16<DT>(acc[2 * j]) | ((uint32_t)rne16<DT>(acc[2 * j + 1]) << 16);
-                for (uint32_t i = 0; i < nsite; ++i) {
+                for (uint32_t i = 0; i < (nsite > (uint32_t)kARSites ? 0u : nsite); ++i) {
                     const uint32_t d = sh_site_e[i] - (v - v0) * 8u;
                     if (d < 8u) w[d >> 1] ^= (sh_site_m[i] & 0xFFFFu) << ((d & 1) * 16);
+                }
+                if (nsite > (uint32_t)kARSites) {   // rare overflow path: scan every site
+                    for (int i = 0; i < p.n_sites; ++i) {
+                        const ft2_fault_site st = p.sites[i];
+                        if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
+                        const int64_t r = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
+                                          (p.cur_step == 0 ? (int64_t)st.token : 0);
+                        if (r != (int64_t)row || (int64_t)st.col >= p.n) continue;
+                        const uint32_t d = (uint32_t)((int64_t)st.col - (int64_t)c8 * 8);
+                        if (d < 8u) w[d >> 1] ^= (st.xor_mask & 0xFFFFu) << ((d & 1) * 16);
+                    }
                 }
                 if (p.mode == FT2_GEMM_CHECK) {
                     const int s = row_mode == 2 ? 0 : (row_mode == 1 ? (int)row : p.row_to_seq[row]);
@@ -175,8 +186,13 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
             }
         }
     }
-    // ---- 4. last CTA: this rank's call is complete; advance the epoch
-    if (p.P == 1) return;   // no handshake at P = 1: the epoch is never read
+    // ---- 4. last CTA: this rank's call is complete; advance the epoch.
+    // P = 1: nobody reads the epoch within a call, so CTA 0 advances it
+    // without the completion counter (it stays the call counter)
+    if (p.P == 1) {
+        if (blockIdx.x == 0 && tid == 0) *reinterpret_cast<volatile uint32_t*>(p.epoch) = e;
+        return;
+    }
     __syncthreads();
     if (tid == 0) sh_last = atom_add_acq_rel_gpu(p.done, 1u) == gridDim.x - 1;
     __syncthreads();

@@ -281,6 +281,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
             // fault sites of this row inside this tile (fault-injection runs only)
             uint32_t site_c[kPMaxRowSites], site_m[kPMaxRowSites];
             int nsite = 0;
+            bool site_scan = false;   // more than kPMaxRowSites: rescan every site per chunk (never drop one)
             if (p.sites != nullptr && row_ok) {
                 for (int i = 0; i < p.n_sites; ++i) {
                     const ft2_fault_site st = p.sites[i];
@@ -288,10 +289,14 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     const int64_t r = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
                                       (p.cur_step == 0 ? (int64_t)st.token : 0);
                     const int64_t c = (int64_t)st.col - n0;
-                    if (r == m && c >= 0 && c < kPBN && (int64_t)st.col < p.N && nsite < kPMaxRowSites) {
-                        site_c[nsite] = (uint32_t)c;
-                        site_m[nsite] = st.xor_mask & 0xFFFFu;
-                        ++nsite;
+                    if (r == m && c >= 0 && c < kPBN && (int64_t)st.col < p.N) {
+                        if (nsite < kPMaxRowSites) {
+                            site_c[nsite] = (uint32_t)c;
+                            site_m[nsite] = st.xor_mask & 0xFFFFu;
+                            ++nsite;
+                        } else {
+                            site_scan = true;
+                        }
                     }
                 }
             }
@@ -425,12 +430,25 @@ __global__ void __launch_bounds__(kPThreads, 1)
 #pragma unroll
                 for (int j = 0; j < 16; ++j)
                     w[j] = pack_rne2(__uint_as_float(r[2 * j]) + bv[2 * j], __uint_as_float(r[2 * j + 1]) + bv[2 * j + 1], DT);
-                for (int i = 0; i < nsite; ++i) {
+                for (int i = 0; i < (site_scan ? 0 : nsite); ++i) {
                     const uint32_t d = site_c[i] - (uint32_t)c0;
                     if (d < 32u) {
 #pragma unroll
                         for (int j = 0; j < 16; ++j)
                             if ((d >> 1) == (uint32_t)j) w[j] ^= site_m[i] << ((d & 1u) * 16);
+                    }
+                }
+                if (site_scan) {   // rare overflow path: every site, straight from global memory
+                    for (int i = 0; i < p.n_sites; ++i) {
+                        const ft2_fault_site st = p.sites[i];
+                        if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
+                        const int64_t r = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
+                                          (p.cur_step == 0 ? (int64_t)st.token : 0);
+                        const uint32_t d = (uint32_t)((int64_t)st.col - n0 - c0);
+                        if (r != m || (int64_t)st.col >= p.N || d >= 32u) continue;
+#pragma unroll
+                        for (int j = 0; j < 16; ++j)
+                            if ((d >> 1) == (uint32_t)j) w[j] ^= (st.xor_mask & 0xFFFFu) << ((d & 1u) * 16);
                     }
                 }
                 if (p.mode == FT2_GEMM_CHECK && seq >= 0) {

@@ -187,6 +187,29 @@ __device__ __noinline__ uint2 xor_sites(uint2 w, uint32_t le0, const uint32_t* s
     return w;
 }
 
+// Overflow path (more than kMaxSitesPerCta sites landed in this CTA's slice,
+// e.g. a directed campaign): scan every site for the four elements of a quad
+// -- slow, but no site is ever dropped.  SWAP: the quad is (feature ga,
+// tokens gb0..gb0+3); otherwise (token ga, features gb0..gb0+3).
+template <bool SWAP>
+__device__ __noinline__ uint2 xor_sites_scan(uint2 w, const GemmK& p, int ga, int gb0) {
+    for (int i = 0; i < p.n_sites; ++i) {
+        const ft2_fault_site st = p.sites[i];
+        if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
+        const int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) + (p.cur_step == 0 ? (int64_t)st.token : 0);
+        const int64_t n = st.col;
+        if (m < 0 || m >= p.M || n >= p.N) continue;
+        const int64_t d = SWAP ? (n == ga ? m - gb0 : -1) : (m == ga ? n - gb0 : -1);
+        if (d < 0 || d >= 4) continue;
+        const uint32_t msk = st.xor_mask & 0xFFFFu;
+        if (d == 0) w.x ^= msk;
+        else if (d == 1) w.x ^= msk << 16;
+        else if (d == 2) w.y ^= msk;
+        else w.y ^= msk << 16;
+    }
+    return w;
+}
+
 // Check-and-clip of two packed bf16 (R5): NaN -> key(+0), clamp in key space.
 template <int DT>
 __device__ __forceinline__ uint32_t clip2_nocount(uint32_t w, uint32_t kL2, uint32_t kH2) {
@@ -201,13 +224,14 @@ template <bool SWAP, int DT>
 __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, int ga, int gb0, const TabE& re,
                                         const TabE* __restrict__ ce, uint32_t le0, float4 acc,
                                         const uint32_t* site_e, const uint32_t* site_m, uint32_t nsite,
-                                        uint32_t* row_cnt, uint32_t* col_cnt) {
+                                        uint32_t* row_cnt, uint32_t* col_cnt, const GemmK& p) {
     // feature side: SWAP ? the row : the column; token side: the other one
     const float b0 = SWAP ? re.bias : ce[0].bias, b1 = SWAP ? re.bias : ce[1].bias;
     const float b2 = SWAP ? re.bias : ce[2].bias, b3 = SWAP ? re.bias : ce[3].bias;
     uint2 w = make_uint2((uint32_t)rne16<DT>(acc.x + b0) | ((uint32_t)rne16<DT>(acc.y + b1) << 16),
                          (uint32_t)rne16<DT>(acc.z + b2) | ((uint32_t)rne16<DT>(acc.w + b3) << 16));
-    if (nsite) w = xor_sites(w, le0, site_e, site_m, nsite);
+    if (nsite > (uint32_t)kMaxSitesPerCta) w = xor_sites_scan<SWAP>(w, p, ga, gb0);
+    else if (nsite) w = xor_sites(w, le0, site_e, site_m, nsite);
     uint32_t f[4], kL01, kH01, kL23, kH23;
 #pragma unroll
     for (int j = 0; j < 4; ++j) f[j] = re.flags & ce[j].flags;  // bit0 valid, bit1 checked
@@ -451,6 +475,13 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const int nrow = r1 - r0;
         const int nvec = nrow * (BN / 4);
         const uint32_t inv = (uint32_t)((1u << 20) + nrow - 1) / (uint32_t)nrow;  // v / nrow == (v * inv) >> 20
+        // kernel parameters the finish needs, loaded while the main loop
+        // streams and kept in registers (the empty asm stops the compiler
+        // from re-reading them from the constant bank on the critical path)
+        uint16_t* y = p.y;
+        int64_t ldy = p.ldy;
+        uint32_t* counts = (p.counts != nullptr && p.mode == FT2_GEMM_CHECK) ? p.counts : nullptr;
+        asm volatile("" : "+l"(y), "+l"(ldy), "+l"(counts));
         if (cs) cluster_wait();  // every peer's receive barrier is initialised
         mbar_wait(tmem_full, 0);
         if (a == 0) FT2_TRACE(5);
@@ -521,9 +552,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             finisher = *gs_last != 0u;
         }
         if (tid == 64) FT2_TRACE(6);
-        const uint32_t nsite = min(*site_n, (uint32_t)kMaxSitesPerCta);
-        uint16_t* const y = p.y;
-        const int64_t ldy = p.ldy;
+        const uint32_t nsite = *site_n;   // > kMaxSitesPerCta: finish4 scans every site
 #pragma unroll 1
         for (int v = e; v < (finisher ? nvec : 0); v += 128) {
             // consecutive threads take consecutive rows (coalesced stores in swap-AB mode)
@@ -546,14 +575,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
             if (tid == 64) FT2_TRACE(11);
             finish4<SWAP, DT>(y, ldy, tileA * kBlockA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
-                              (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4);
+                              (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4, p);
         }
         if (tid == 64) FT2_TRACE(7);
-        if (p.counts != nullptr && p.mode == FT2_GEMM_CHECK && finisher) {
+        if (counts != nullptr && finisher) {
             named_bar(3, 128);  // every finish4 of this CTA has counted
-            if (!SWAP && row_cnt[e] != 0u) atomicAdd(&p.counts[row_tab[e].seq], row_cnt[e]);
+            if (!SWAP && row_cnt[e] != 0u) atomicAdd(&counts[row_tab[e].seq], row_cnt[e]);
             for (int c = e; SWAP && c < BN; c += 128)
-                if (col_cnt[c] != 0u) atomicAdd(&p.counts[col_tab[c].seq], col_cnt[c]);
+                if (col_cnt[c] != 0u) atomicAdd(&counts[col_tab[c].seq], col_cnt[c]);
         }
     }
     // warps 0 and 1 pair their prologue cluster arrive (no finish work for them)

@@ -170,3 +170,35 @@ def test_allreduce_protect_fp16_plain_and_row_map_p1():
         assert int(wcnt.sum()) > 0 and rpc.status() == 0
     finally:
         dist.destroy_process_group()
+
+
+def test_allreduce_protect_site_overflow_p1():
+    """more than the 64 sites a CTA's list holds, all in one CTA's
+    chunk (100 sites on row 0, base_row = 0), are all applied as the oracle's
+    R7 applies them."""
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+    port = _port()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        from gpu_util import dev, dev_i32, host, sites_to_dev
+        rpc = tp.RowParallelCheck(ROWS, N)
+        parts, bias, bounds, _ = _inputs(0, 1)
+        s = np.zeros(100, oracle.SITE_DTYPE)
+        s["step"], s["layer"], s["col"] = 1, 0, (np.arange(100) * 13) % 2048
+        s["xor_mask"] = 1 << (np.arange(100) % 16)
+        base = np.zeros(100, np.int32)
+        rpc.partial(0).copy_(dev(parts[0]))
+        y = torch.empty((ROWS, N), dtype=torch.bfloat16, device="cuda")
+        cnt = torch.zeros(ROWS, dtype=torch.int32, device="cuda")
+        rpc(0, y, bias=dev(bias), mode=1, bounds=dev(bounds), num_seqs=ROWS, corrected_count=cnt,
+            sites=sites_to_dev(s), n_sites=100, cur_layer=0, cur_step=1, base_row=dev_i32(base))
+        torch.cuda.synchronize()
+        want, wcnt = oracle.allreduce_protect(parts[:1], bias=bias, bounds_=bounds, sites=s, cur_layer=0,
+                                              cur_step=1, base_row=base)
+        plain, _ = oracle.allreduce_protect(parts[:1], bias=bias, bounds_=bounds)
+        assert int((want != plain).sum()) > 0
+        assert np.array_equal(host(y), want)
+        assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), wcnt)
+    finally:
+        dist.destroy_process_group()

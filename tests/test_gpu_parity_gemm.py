@@ -216,3 +216,36 @@ def test_gemm_shared_workspace_across_shapes(ft2):
         yr, _ = oracle.linear_f64(x, w, b)
         nbad, worst = _tol_ok(y, yr)
         assert nbad == 0, (M, N, K, nbad, worst)
+
+
+def _directed_sites(n_sites, cols, step=1, layer=0, token=0):
+    """n_sites sites, all at (step, layer), columns `cols`; with base_row = 0
+    every one lands in row 0 (+ token during the prefill): a dense, directed
+    site set that overflows any per-CTA site list."""
+    s = np.zeros(n_sites, oracle.SITE_DTYPE)
+    s["trial"] = np.arange(n_sites)
+    s["step"], s["layer"], s["token"] = step, layer, token
+    s["col"] = cols
+    s["xor_mask"] = 1 << (np.arange(n_sites) % 16)
+    s["nbits"] = 1
+    return s
+
+
+@pytest.mark.parametrize("M,N,K,step", [(32, 256, 256, 1), (8, 2048, 512, 3), (200, 512, 256, 0)])
+def test_gemm_site_overflow_is_never_dropped(ft2, M, N, K, step):
+    """more sites than the per-CTA (decode: 64) or per-row-per-tile
+    (prefill: 4) lists hold -- here 100 sites in one row and one 128/256-wide
+    tile -- must still all be applied, exactly as the oracle's R7 applies them."""
+    x, w, b = _operands(M, N, K, seed=29)
+    plain, _ = _run(ft2, x, w, b, 0)
+    sites = _directed_sites(100, (np.arange(100) * 7) % 128, step=step, token=1 if step == 0 else 0)
+    base = np.zeros(100, np.int32)
+    ref = plain.copy()
+    oracle.inject(ref, sites, 0, step, base_row=base)
+    assert int((ref != plain).sum()) >= 90      # the flips really land (a few columns repeat and cancel)
+    inj, _ = _run(ft2, x, w, b, 0, sites=sites, layer=0, step=step, base_row=base)
+    assert np.array_equal(inj, ref)
+    bnds = np.array([[oracle.f64_to_bf16(-0.5), oracle.f64_to_bf16(0.5)]], np.uint16)
+    rc = oracle.protect(ref, bnds)
+    chk, cnt = _run(ft2, x, w, b, 1, bounds=bnds, S=1, sites=sites, layer=0, step=step, base_row=base)
+    assert np.array_equal(chk, ref) and np.array_equal(cnt, rc)
