@@ -81,12 +81,14 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     __shared__ uint32_t sh_site_e[kARSites], sh_site_m[kARSites];
     const int tid = threadIdx.x;
     const uint32_t v0 = blockIdx.x * chunk, v1 = min(v0 + chunk, total_vec);
+    // P = 1 without sites: no handshake, no site list -- straight to the loads
+    const bool prologue = p.P > 1 || p.sites != nullptr;
     if (tid == 0) {
-        sh_e = *reinterpret_cast<volatile uint32_t*>(p.epoch) + 1u;
+        sh_e = p.P > 1 ? *reinterpret_cast<volatile uint32_t*>(p.epoch) + 1u : 0u;
         sh_ok = 1u;
         sh_ns = 0u;
     }
-    __syncthreads();
+    if (prologue) __syncthreads();
     const uint32_t e = sh_e;
     // ---- 1. signal: my partial (written by the preceding kernel) is ready.
     // P = 1 needs no handshake: stream order already covers my own partial.
@@ -117,9 +119,9 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
             if (k < (uint32_t)kARSites) { sh_site_e[k] = (uint32_t)(el - (uint64_t)v0 * 8u); sh_site_m[k] = s.xor_mask; }
         }
     }
-    __syncthreads();
-    if (sh_ok) {
-        const uint32_t nsite = sh_ns;   // > kARSites: every site is rescanned per vector (none dropped)
+    if (prologue) __syncthreads();
+    if (!prologue || sh_ok) {
+        const uint32_t nsite = prologue ? sh_ns : 0u;   // > kARSites: every site is rescanned per vector (none dropped)
         for (uint32_t vb = v0 + tid; vb < v1; vb += kARThreads * kVecs) {
             // issue every load of this pass first: kVecs vectors x min(P, 8) partials
             uint4 part[kVecs][kARMaxP];
@@ -190,7 +192,10 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     // P = 1: nobody reads the epoch within a call, so CTA 0 advances it
     // without the completion counter (it stays the call counter)
     if (p.P == 1) {
-        if (blockIdx.x == 0 && tid == 0) *reinterpret_cast<volatile uint32_t*>(p.epoch) = e;
+        if (blockIdx.x == 0 && tid == 0) {
+            volatile uint32_t* ep = reinterpret_cast<volatile uint32_t*>(p.epoch);
+            *ep = *ep + 1u;
+        }
         return;
     }
     __syncthreads();
@@ -206,8 +211,9 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
 
 cudaError_t launch_allreduce_protect(const AllreduceProtectArgs& a, cudaStream_t st, int* n_launch) {
     const uint32_t n8 = (uint32_t)(a.n / 8), total = (uint32_t)(a.rows * (a.n / 8));
-    // kVecs vectors per thread per pass; at most 2 CTAs per SM (every CTA polls)
-    uint32_t grid = (total + kARThreads * kVecs - 1) / (kARThreads * kVecs);
+    // one vector per thread (kVecs per pass once the grid is capped); at most
+    // 2 CTAs per SM (every CTA polls)
+    uint32_t grid = (total + kARThreads - 1) / kARThreads;
     const uint32_t cap = (uint32_t)(2 * num_sms());
     grid = grid < 1 ? 1 : (grid > cap ? cap : grid);
     uint32_t chunk = (total + grid - 1) / grid;
