@@ -197,6 +197,20 @@ class ClockSampler:
 _ORACLE_INPUTS = {}
 
 
+_T0 = time.time()
+
+
+def progress(msg):
+    """One line per bench phase on stderr (rank-tagged), so a stalled
+    multi-rank run shows where it stands."""
+    print(f"[bench r{os.environ.get('RANK', '0')} +{time.time() - _T0:7.1f}s] {msg}", file=sys.stderr, flush=True)
+
+
+def _skip(name):
+    """FT2_BENCH_SKIP=name,name...: leave out optional legs of the default run (debugging)."""
+    return name in os.environ.get("FT2_BENCH_SKIP", "").split(",")
+
+
 def host_cpu():
     """nproc and the CPU model of the host the oracle runs on."""
     import platform
@@ -383,6 +397,7 @@ def main():
         torch.cuda.nvtx.range_pop()
         return 0
 
+    progress("runner built; warming up the four modes")
     modes = ["fused", "off", "standalone", "fused_plain"]
     # warm-up: captures the prefill and decode graphs of every mode; the first
     # few replays after a capture run ~5% slow (measured), so every mode gets
@@ -398,6 +413,7 @@ def main():
     # sustained load, with or without the clock sampler), so keep serving
     # fused requests until >= FT2_BENCH_SETTLE_S seconds have passed and the
     # last three agree within 1 % (at most 3x that time).  Untimed.
+    progress("settle")
     settle = []
     t_min = float(os.environ.get("FT2_BENCH_SETTLE_S", "8"))
     t0 = time.perf_counter()
@@ -414,6 +430,7 @@ def main():
             break
     barrier()
 
+    progress("timed requests")
     clk = ClockSampler(local)
     clk.start()
     ms_fused = timed("fused", args.steps)          # the headline: K contiguous requests
@@ -485,23 +502,32 @@ def main():
     }
 
     if not args.no_extras:
+        progress("kernel rooflines")
         res.update(kernel_rooflines(runner, dev, ft2))
         rf = res["roofline"]
         dec_us = 1000.0 * phases["fused"]["decode_ms_per_step"]
         # the kernel's share of a decode step (compare with the ncu launch list in profiles/)
         rf["share_of_decode_step"] = rf["launches_per_graph"] * rf["avg_launch_us"] / dec_us
     if not args.no_extras:
-        res["coverage_overhead_pct"] = coverage_costs(cfg, B, T, G, dev, prompt, stream, runner, ms_off)
-        res["c2_matrix"] = c2_matrix(dev, args)
-        res["protect_sweep"] = protect_sweep(dev, ft2, load_peaks())
+        if not _skip("coverage"):
+            progress("coverage costs")
+            res["coverage_overhead_pct"] = coverage_costs(cfg, B, T, G, dev, prompt, stream, runner, ms_off)
+        if not _skip("c2"):
+            progress("c2 matrix")
+            res["c2_matrix"] = c2_matrix(dev, args)
+        if not _skip("sweep"):
+            progress("protection sweep")
+            res["protect_sweep"] = protect_sweep(dev, ft2, load_peaks())
     if not args.no_extras:
         # the paths that shard, at this run's N: configs[3]'s
         # TP bounds + row-parallel check, configs[4]'s campaign with its trial
         # ranges split over the ranks
         del runner
         torch.cuda.empty_cache()
+        progress("partitioned paths")
         res["partitioned_paths"] = partitioned_legs(args, dev, rank, world)
     if rank == 0 and world == 1 and not args.no_extras:
+        progress("c1 + cpu baseline")
         res["c1_single_layer"] = c1_leg(dev, ft2)
         cb = oracle_sample(args.model, B, T, G, threads=0)
         cb1 = oracle_sample(args.model, B, T, G, threads=1)
@@ -536,11 +562,13 @@ def partitioned_legs(args, dev, rank, world, trials_per_rank=512):
         t = torch.ones(1, device=dev)
         dist.all_reduce(t)
         out["comm_nranks_ok"] = int(t.item()) == world
+    progress("c4 TP bounds")
     out["c4_tp"] = c4_tp_bounds(args, dev, rank, world)
     torch.cuda.empty_cache()
     a = copy.copy(args)
     a.trials = trials_per_rank * world
     a.coverage_trials = 0
+    progress("c5 campaign")
     c5 = c5_campaign(a, dev, rank, world)
     c5["scaling"] = "weak"
     c5["trials_per_s_per_gpu"] = c5["value"] / world
@@ -991,6 +1019,7 @@ def c4_tp_bounds(args, dev, rank, world, B=32, T=128, blocks=40, R=20):
         dist.all_reduce(f, op=dist.ReduceOp.MAX)
         exact = int(f.item()) == 0
     shard_bytes = sum(rows * (e - b) * 2 for _, b, e in col_layers) + sum(y.numel() * 2 for y in row_layers)
+    progress("c4 row-parallel decode check")
     row_parallel = c4_row_parallel_decode(dev, world, B, blocks, dev_time)
     return {"leg": "c4", "metric": "TP first-token bounds phase per prefill (us, max over ranks)", "value": us_phase,
             "unit": "us", "higher_is_better": False, "n_gpus": world, "scaling": "strong",

@@ -94,16 +94,7 @@ struct GemmK {
     int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
     int32_t trigger;   // issue griddepcontrol.launch_dependents early (FT2_GEMM_TRIGGER, default 1)
     int32_t w_l2;      // static weights: L2-prefetch the K slice beyond the ring before the PDL wait (FT2_GEMM_W_L2)
-    // K split through global memory instead of the cluster (no cluster launch:
-    // every CTA starts at once; the last split of a tile to arrive sums the
-    // tile's fp32 slots in split order and finishes all 128 rows).  Opt-in
-    // experiment (FT2_GEMM_GSPLIT=1): parity-clean but measured 3-4x slower
-    // than the cluster/DSMEM split (2048x2048, M = 32: 21.3 vs 5.7 us back to
-    // back), so the late-starting 16th cluster of 8 is the cheaper evil.
-    int32_t gsplit;
-    float* gws;        // [tiles][splitk][128][BN] fp32 partial slots
-    uint32_t* gcnt;    // [tiles] arrival counters (self-cleaning)
-    int32_t rows_per_slot;  // ceil(128 / splitk): rows of one split-K receive slot
+    int32_t rows_per_slot;  // ceil(BA / splitk): rows of one split-K receive slot
     uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
     int32_t trace_base;     // trace builds only: first g_trace row of this launch
     const uint8_t* pf;      // L2 prefetch hint (the next layer's weights) and its size
@@ -151,21 +142,26 @@ __device__ __forceinline__ TabE token_entry(const GemmK& p, int m) {
 // DEEP: one CTA per SM with a ring deep enough (~180 KB) that a CTA's whole K
 // slice is in flight at once -- one DRAM round trip for few-tile decode
 // shapes.  Otherwise ~105 KB so two CTAs share an SM.
-template <int BN, bool DEEP = false>
+// BA = UMMA M (output features per tile in swap-AB): 128, or 64 for few-tile
+// decode shapes -- twice the tiles, so a split keeps a CTA's whole K slice in
+// a ring that still fits two CTAs per SM, and half the split-K bytes per CTA.
+template <int BA, int BN, bool DEEP = false>
 struct Cfg {
-    static constexpr int STAGES = DEEP ? (BN <= 16 ? 10 : (BN <= 32 ? 9 : 7))
+    static_assert(BA == 128 || (BA == 64 && BN <= 32 && !DEEP), "BA = 64 serves 16/32-token tiles");
+    static constexpr int STAGES = BA == 64 ? (BN <= 16 ? 9 : 8)
+                                : DEEP ? (BN <= 16 ? 10 : (BN <= 32 ? 9 : 7))
                                        : (BN <= 16 ? 5 : (BN <= 32 ? 4 : (BN <= 64 ? 3 : 4)));
-    static constexpr int kABytes = kBlockA * kBlockK * 2;
+    static constexpr int kABytes = BA * kBlockK * 2;
     static constexpr int kBBytes = BN * kBlockK * 2;
     static constexpr int kStageBytes = kABytes + kBBytes;
     static constexpr int kTileBytes = STAGES * kStageBytes;
-    // fp32 tile staging / split-K receive buffer: splitk slots x ceil(128/splitk)
-    // rows (<= 143 in total) x (BN + 4) fp32; the pad keeps float4 row reads
+    // fp32 tile staging / split-K receive buffer: splitk slots x ceil(BA/splitk)
+    // rows (< BA + 16 in total) x (BN + 4) fp32; the pad keeps float4 row reads
     // bank-conflict free
     static constexpr int kRecvStride = BN + 4;
-    static constexpr int kRecvBytes = 144 * kRecvStride * 4;
+    static constexpr int kRecvBytes = (BA + 16) * kRecvStride * 4;
     static constexpr int kMiscBytes = 1024;  // mbarriers, TMEM base, site list
-    static constexpr int kTabBytes = (kBlockA + BN) * (int)sizeof(TabE) + (kBlockA + BN) * 4;
+    static constexpr int kTabBytes = (BA + BN) * (int)sizeof(TabE) + (BA + BN) * 4;
     static constexpr int kBytes = 1024 /*align slack*/ + kTileBytes + kRecvBytes + kMiscBytes + kTabBytes;
     static constexpr uint32_t kTmemCols = BN < 32 ? 32 : BN;
 };
@@ -273,11 +269,11 @@ __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, i
     }
 }
 
-template <int BN, bool SWAP, int DT, bool DEEP>
+template <int BA, int BN, bool SWAP, int DT, bool DEEP>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
                 const __grid_constant__ GemmK p) {
-    using C = Cfg<BN, DEEP>;
+    using C = Cfg<BA, BN, DEEP>;
     constexpr int STAGES = C::STAGES;
     extern __shared__ uint8_t smem_raw[];
     // 1024-byte alignment (128B swizzle) by offset arithmetic on the shared
@@ -294,11 +290,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     uint32_t* site_n = tmem_base_sh + 1;
     uint32_t* site_e = site_n + 1;                // [kMaxSitesPerCta] local element a * BN + b
     uint32_t* site_m = site_e + kMaxSitesPerCta;  // [kMaxSitesPerCta] xor mask
-    uint32_t* gs_last = site_m + kMaxSitesPerCta;  // global split: this CTA finishes its tile
-    TabE* row_tab = reinterpret_cast<TabE*>(misc + C::kMiscBytes);  // [128]
-    TabE* col_tab = row_tab + kBlockA;                                // [BN]
-    uint32_t* row_cnt = reinterpret_cast<uint32_t*>(col_tab + BN);    // [128]
-    uint32_t* col_cnt = row_cnt + kBlockA;                            // [BN]
+    TabE* row_tab = reinterpret_cast<TabE*>(misc + C::kMiscBytes);  // [BA]
+    TabE* col_tab = row_tab + BA;                                     // [BN]
+    uint32_t* row_cnt = reinterpret_cast<uint32_t*>(col_tab + BN);    // [BA]
+    uint32_t* col_cnt = row_cnt + BA;                                 // [BN]
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int tileA = blockIdx.x, split = blockIdx.y, tileB = blockIdx.z;
@@ -307,11 +302,9 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     const int kb1 = (int)((int64_t)(split + 1) * p.nkb / splitk);
     const int nk = kb1 - kb0;
     // rows of the tile this CTA finishes: all of them, or its split-K slice
-    const bool gs = splitk > 1 && p.gsplit;    // split through global memory
-    const bool cs = splitk > 1 && !p.gsplit;   // split across the cluster (DSMEM)
-    const int r0 = gs ? 0 : (int)(((uint32_t)(split * kBlockA) * p.sk_magic) >> 24);
-    const int r1 = gs ? kBlockA : (int)(((uint32_t)((split + 1) * kBlockA) * p.sk_magic) >> 24);
-    const int tile_id = tileA + p.tilesA * tileB;
+    const bool cs = splitk > 1;   // split across the cluster (DSMEM)
+    const int r0 = (int)(((uint32_t)(split * BA) * p.sk_magic) >> 24);
+    const int r1 = (int)(((uint32_t)((split + 1) * BA) * p.sk_magic) >> 24);
 
     if (warp == 0 && lane == 0) {
         FT2_TRACE(0);
@@ -333,7 +326,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             for (int i = 0; i < pre; ++i) {
                 mbar_expect_tx(&full[i], C::kStageBytes);
                 tma_load_2d(SWAP ? &map_a : &map_b, &full[i], tiles + i * C::kStageBytes + (SWAP ? 0 : C::kABytes),
-                            (kb0 + i) * kBlockK, SWAP ? tileA * kBlockA : tileB * BN);
+                            (kb0 + i) * kBlockK, SWAP ? tileA * BA : tileB * BN);
             }
             // ... and the rest of this CTA's weight slice is pulled into L2
             // right away (no shared memory needed), so the whole layer
@@ -342,7 +335,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             if (p.w_l2) {   // at most one more ring's worth (a whole large slice would thrash L2)
                 const int lim = nk < pre + STAGES ? nk : pre + STAGES;
                 for (int i = pre; i < lim; ++i)
-                    tma_prefetch_l2_2d(SWAP ? &map_a : &map_b, (kb0 + i) * kBlockK, SWAP ? tileA * kBlockA : tileB * BN);
+                    tma_prefetch_l2_2d(SWAP ? &map_a : &map_b, (kb0 + i) * kBlockK, SWAP ? tileA * BA : tileB * BN);
             }
         }
     }
@@ -360,8 +353,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             // ------------------------------------------------ TMA producer
             const CUtensorMap* mw = SWAP ? &map_a : &map_b;
             const CUtensorMap* mx = SWAP ? &map_b : &map_a;
-            const int w_row = SWAP ? tileA * kBlockA : tileB * BN;
-            const int x_row = SWAP ? tileB * BN : tileA * kBlockA;
+            const int w_row = SWAP ? tileA * BA : tileB * BN;
+            const int x_row = SWAP ? tileB * BN : tileA * BA;
             const int w_off = SWAP ? 0 : C::kABytes;
             const int x_off = SWAP ? C::kABytes : 0;
             FT2_TRACE(1);
@@ -409,7 +402,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             // ------------------------------------------------ MMA issuer
             // kind::f16 operand format: 0 = F16, 1 = BF16 (bits 7-9 A, 10-12 B)
             constexpr uint32_t idesc =
-                (make_idesc(kBlockA, BN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
+                (make_idesc(BA, BN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
             for (int i = 0; i < nk; ++i) {
                 const int s = i % STAGES;
                 mbar_wait(&full[s], (uint32_t)(i / STAGES) & 1u);
@@ -431,24 +424,31 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     } else {
         // ---------------------------------------------------- epilogue warps
         const int q = warp & 3;  // TMEM lane quarter this warp may access
-        const int a = q * 32 + lane;
+        const int e = tid - 64;  // 0..127
+        // Accumulator row a of this thread.  BA = 128: TMEM lane 32q + lane
+        // holds row 32q + lane.  BA = 64 (cta_group::1, M = 64): rows 16q..16q+15
+        // sit in lanes 32q..32q+15 of the warp's quarter; lanes 16-31 hold none.
+        const int a = BA == 128 ? q * 32 + lane : q * 16 + (lane & 15);
+        const bool has_row = BA == 128 || lane < 16;
         griddep_wait();  // bias/bounds/sites/y may belong to the previous kernel
         // epilogue tables, gathered while the main loop still streams
-        row_tab[a] = SWAP ? feature_entry<DT>(p, tileA * kBlockA + a) : token_entry(p, tileA * kBlockA + a);
-        row_cnt[a] = 0u;
-        for (int c = a; c < BN; c += 128) {
+        for (int r = e; r < BA; r += 128) {
+            row_tab[r] = SWAP ? feature_entry<DT>(p, tileA * BA + r) : token_entry(p, tileA * BA + r);
+            row_cnt[r] = 0u;
+        }
+        for (int c = e; c < BN; c += 128) {
             col_tab[c] = SWAP ? token_entry(p, tileB * BN + c) : feature_entry<DT>(p, tileB * BN + c);
             col_cnt[c] = 0u;
         }
         if (p.sites != nullptr) {  // fault sites landing in my slice
-            for (int i = a; i < p.n_sites; i += 128) {
+            for (int i = e; i < p.n_sites; i += 128) {
                 const ft2_fault_site st = p.sites[i];
                 if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
                 const int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
                                   (p.cur_step == 0 ? (int64_t)st.token : 0);
                 const int64_t n = st.col;
                 if (m < 0 || m >= p.M || n >= p.N) continue;
-                const int64_t la = (SWAP ? n : m) - (int64_t)tileA * kBlockA;
+                const int64_t la = (SWAP ? n : m) - (int64_t)tileA * BA;
                 const int64_t lb = (SWAP ? m : n) - (int64_t)tileB * BN;
                 if (la < r0 || la >= r1 || lb < 0 || lb >= BN) continue;
                 const uint32_t idx = atomicAdd(site_n, 1u);
@@ -460,18 +460,17 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         }
         // Receive-slot geometry of accumulator row a (independent of the
         // accumulator, so computed while the main loop streams): its owner
-        // is the split whose row slice holds a, r0(r) = floor(128 r / splitk)
-        // evaluated as (128 r * sk_magic) >> 24 (exact for these ranges).
+        // is the split whose row slice holds a, r0(r) = floor(BA r / splitk)
+        // evaluated as (BA r * sk_magic) >> 24 (exact for these ranges).
         const int RS = p.rows_per_slot;
-        const int owner = ((a + 1) * splitk - 1) >> 7;
-        const int own_r0 = (int)(((uint32_t)(owner * kBlockA) * p.sk_magic) >> 24);
+        const int owner = ((a + 1) * splitk - 1) / BA;
+        const int own_r0 = (int)(((uint32_t)(owner * BA) * p.sk_magic) >> 24);
         const uint32_t slot_off = (uint32_t)(((split * RS + (a - own_r0)) * C::kRecvStride) * 4);
         const bool local = owner == split;
         const uint32_t dst = local ? smem_u32(recv) + slot_off : mapa(smem_u32(recv) + slot_off, (uint32_t)owner);
         const uint32_t dbar = local ? 0u : mapa(smem_u32(recv_bar), (uint32_t)owner);
         const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
         // finish-loop geometry: item v -> (row lr, column quad c4)
-        const int e = tid - 64;  // 0..127
         const int nrow = r1 - r0;
         const int nvec = nrow * (BN / 4);
         const uint32_t inv = (uint32_t)((1u << 20) + nrow - 1) / (uint32_t)nrow;  // v / nrow == (v * inv) >> 20
@@ -484,26 +483,21 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         asm volatile("" : "+l"(y), "+l"(ldy), "+l"(counts));
         if (cs) cluster_wait();  // every peer's receive barrier is initialised
         mbar_wait(tmem_full, 0);
-        if (a == 0) FT2_TRACE(5);
+        if (e == 0) FT2_TRACE(5);
         tc_fence_after();
         // Stage accumulator row a as fp32 in the receive slot of its owner
-        // (this CTA without split-K; a cluster peer with it).
+        // (this CTA without split-K; a cluster peer with it).  The TMEM loads
+        // are warp-collective: every lane issues them, rowless lanes drop the data.
         if constexpr (BN == 32) {  // one TMEM load for the whole row, then the pushes back to back
             uint32_t r[32];
             tmem_ld32(taddr, r);
             tmem_wait_ld();
-            if (a == 0) FT2_TRACE(14);
+            if (e == 0) FT2_TRACE(14);
             if (nk == 0) {
 #pragma unroll
                 for (int j = 0; j < 32; ++j) r[j] = 0u;
             }
-            if (gs) {
-                float4* g = reinterpret_cast<float4*>(p.gws + ((size_t)(tile_id * splitk + split) * kBlockA + a) * BN);
-#pragma unroll
-                for (int j = 0; j < 32; j += 4)
-                    __stcg(g + j / 4, make_float4(__uint_as_float(r[j]), __uint_as_float(r[j + 1]),
-                                                  __uint_as_float(r[j + 2]), __uint_as_float(r[j + 3])));
-            } else {
+            if (has_row) {
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) {
                     if (local) st_shared_v4(dst + (uint32_t)(j * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
@@ -516,18 +510,12 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             uint32_t r[16];
             tmem_ld16(taddr + c0, r);
             tmem_wait_ld();
-            if (a == 0 && c0 == 0) FT2_TRACE(14);
+            if (e == 0 && c0 == 0) FT2_TRACE(14);
             if (nk == 0) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) r[j] = 0u;
             }
-            if (gs) {
-                float4* g = reinterpret_cast<float4*>(p.gws + ((size_t)(tile_id * splitk + split) * kBlockA + a) * BN + c0);
-#pragma unroll
-                for (int j = 0; j < 16; j += 4)
-                    __stcg(g + j / 4, make_float4(__uint_as_float(r[j]), __uint_as_float(r[j + 1]),
-                                                  __uint_as_float(r[j + 2]), __uint_as_float(r[j + 3])));
-            } else {
+            if (has_row) {
 #pragma unroll
                 for (int j = 0; j < 16; j += 4) {
                     if (local) st_shared_v4(dst + (uint32_t)((c0 + j) * 4), r[j], r[j + 1], r[j + 2], r[j + 3]);
@@ -537,50 +525,32 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         }
         if (tid == 64) FT2_TRACE(8);
         // ------------------------------------ finish the slice (epilogue warps)
-        if (gs) __threadfence();   // my slot before my arrival
         named_bar(2, 128);  // tables, site list and my own rows are in shared memory
         if (tid == 64) FT2_TRACE(9);
         if (cs) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
-        bool finisher = true;
-        if (gs) {   // the last split of the tile to arrive finishes it
-            if (tid == 64) {
-                const bool last = atom_add_acq_rel_gpu(p.gcnt + tile_id, 1u) == (uint32_t)(splitk - 1);
-                if (last) p.gcnt[tile_id] = 0u;
-                *gs_last = last ? 1u : 0u;
-            }
-            named_bar(2, 128);
-            finisher = *gs_last != 0u;
-        }
         if (tid == 64) FT2_TRACE(6);
         const uint32_t nsite = *site_n;   // > kMaxSitesPerCta: finish4 scans every site
 #pragma unroll 1
-        for (int v = e; v < (finisher ? nvec : 0); v += 128) {
+        for (int v = e; v < nvec; v += 128) {
             // consecutive threads take consecutive rows (coalesced stores in swap-AB mode)
             const int c4 = (int)(((uint32_t)v * inv) >> 20), lr = v - c4 * nrow, la = r0 + lr;
             float4 part[kMaxSplitK];
-            if (gs) {   // the tile's slots in split order, from L2
-                const float* g = p.gws + ((size_t)tile_id * splitk * kBlockA + la) * BN + c4 * 4;
+            const float* src = recv + lr * C::kRecvStride + c4 * 4;
 #pragma unroll
-                for (int rr = 0; rr < kMaxSplitK; ++rr)
-                    if (rr < splitk) part[rr] = __ldcg(reinterpret_cast<const float4*>(g + (size_t)rr * kBlockA * BN));
-            } else {
-                const float* src = recv + lr * C::kRecvStride + c4 * 4;
-#pragma unroll
-                for (int rr = 0; rr < kMaxSplitK; ++rr)
-                    if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
-            }
+            for (int rr = 0; rr < kMaxSplitK; ++rr)
+                if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
             float4 acc = part[0];
 #pragma unroll
             for (int rr = 1; rr < kMaxSplitK; ++rr)
                 if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
             if (tid == 64) FT2_TRACE(11);
-            finish4<SWAP, DT>(y, ldy, tileA * kBlockA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
+            finish4<SWAP, DT>(y, ldy, tileA * BA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
                               (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4, p);
         }
         if (tid == 64) FT2_TRACE(7);
-        if (counts != nullptr && finisher) {
+        if (counts != nullptr) {
             named_bar(3, 128);  // every finish4 of this CTA has counted
-            if (!SWAP && row_cnt[e] != 0u) atomicAdd(&counts[row_tab[e].seq], row_cnt[e]);
+            if (!SWAP && e < BA && row_cnt[e] != 0u) atomicAdd(&counts[row_tab[e].seq], row_cnt[e]);
             for (int c = e; SWAP && c < BN; c += 128)
                 if (col_cnt[c] != 0u) atomicAdd(&counts[col_tab[c].seq], col_cnt[c]);
         }
@@ -638,16 +608,16 @@ static int spread_policy() {
     return v;
 }
 
-template <int BN, bool SWAP, int DT, bool DEEP>
+template <int BA, int BN, bool SWAP, int DT, bool DEEP>
 static cudaError_t set_attrs() {
     static cudaError_t res = [] {
-        cudaError_t e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT, DEEP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             Cfg<BN, DEEP>::kBytes + smem_pad());
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT, DEEP>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        auto* k = gemm_kernel<BA, BN, SWAP, DT, DEEP>;
+        cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg<BA, BN, DEEP>::kBytes + smem_pad());
+        if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
         // full shared-memory carveout so two ~105 KB decode CTAs share an SM
         if (e == cudaSuccess && env_int("FT2_GEMM_CARVEOUT", 1))
-            e = cudaFuncSetAttribute(gemm_kernel<BN, SWAP, DT, DEEP>, cudaFuncAttributePreferredSharedMemoryCarveout,
+            e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout,
                                      (int)cudaSharedmemCarveoutMaxShared);
         return e;
     }();
@@ -655,16 +625,16 @@ static cudaError_t set_attrs() {
 }
 
 // How many (1, sk, 1) clusters of this instantiation can be resident at once.
-template <int BN, bool SWAP, int DT = 0, bool DEEP = false>
+template <int BA, int BN, bool SWAP, int DT = 0, bool DEEP = false>
 static int max_clusters(int sk) {
     static int cache[kMaxSplitK + 1] = {0};
     if (sk < 1 || sk > kMaxSplitK) return -1;
     if (cache[sk] != 0) return cache[sk];
-    if (set_attrs<BN, SWAP, DT, DEEP>() != cudaSuccess) return cache[sk] = -1;
+    if (set_attrs<BA, BN, SWAP, DT, DEEP>() != cudaSuccess) return cache[sk] = -1;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(1, (unsigned)sk, 1);
     cfg.blockDim = dim3(kGemmThreads);
-    cfg.dynamicSmemBytes = Cfg<BN, DEEP>::kBytes + smem_pad();
+    cfg.dynamicSmemBytes = Cfg<BA, BN, DEEP>::kBytes + smem_pad();
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 1;
@@ -673,7 +643,7 @@ static int max_clusters(int sk) {
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     int n = 0;
-    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BN, SWAP, DT, DEEP>, &cfg) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveClusters(&n, gemm_kernel<BA, BN, SWAP, DT, DEEP>, &cfg) != cudaSuccess) {
         cudaGetLastError();
         n = -1;
     }
@@ -683,32 +653,44 @@ static int max_clusters(int sk) {
 static int max_clusters_bn(int bn, int sk, bool deep = false) {
     if (deep) {
         switch (bn) {
-            case 16: return max_clusters<16, true, 0, true>(sk);
-            case 32: return max_clusters<32, true, 0, true>(sk);
-            case 64: return max_clusters<64, true, 0, true>(sk);
+            case 16: return max_clusters<128, 16, true, 0, true>(sk);
+            case 32: return max_clusters<128, 32, true, 0, true>(sk);
+            case 64: return max_clusters<128, 64, true, 0, true>(sk);
             default: return -1;
         }
     }
     switch (bn) {
-        case 16: return max_clusters<16, true>(sk);
-        case 32: return max_clusters<32, true>(sk);
-        case 64: return max_clusters<64, true>(sk);
-        default: return max_clusters<128, true>(sk);
+        case 16: return max_clusters<128, 16, true>(sk);
+        case 32: return max_clusters<128, 32, true>(sk);
+        case 64: return max_clusters<128, 64, true>(sk);
+        default: return max_clusters<128, 128, true>(sk);
     }
 }
 static int deep_stages(int bn) {
     switch (bn) {
-        case 16: return Cfg<16, true>::STAGES;
-        case 32: return Cfg<32, true>::STAGES;
-        case 64: return Cfg<64, true>::STAGES;
+        case 16: return Cfg<128, 16, true>::STAGES;
+        case 32: return Cfg<128, 32, true>::STAGES;
+        case 64: return Cfg<128, 64, true>::STAGES;
         default: return 0;
     }
 }
 
-// Tiling plan: orientation, tile width, split-K factor.
+// Tiling plan: orientation, feature-tile height BA, token-tile width, split-K factor.
 struct GemmPlan {
-    int swap, bn, tilesA, tilesB, splitk, nkb, deep;
+    int swap, ba, bn, tilesA, tilesB, splitk, nkb, deep;
 };
+
+// 64-row feature tiles (UMMA M = 64) for decode batches of <= 32 tokens:
+// FT2_GEMM_BA = 64 / 128 forces the choice; 0 = the planner's rule below.
+static bool use_ba64(int32_t M, int32_t N, int32_t K) {
+    static const int ba_env = env_int("FT2_GEMM_BA", 0);
+    if (M > 32) return false;
+    if (ba_env == 64) return true;
+    if (ba_env == 128) return false;
+    (void)N;
+    (void)K;
+    return false;
+}
 
 // Largest token count that runs swap-AB on this kernel (BN = 128 token tiles
 // above 64); larger M goes to the persistent prefill kernel.
@@ -717,14 +699,35 @@ static int swap_max_m() {
     return v;
 }
 
-static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
+static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
     GemmPlan g;
     g.swap = M <= swap_max_m() ? 1 : 0;
+    g.ba = 128;
+    static const int sk_env0 = env_int("FT2_GEMM_SPLITK", 0);
+    if (g.swap && use_ba64(M, N, K)) {
+        // the smallest split whose K slice fits the ring (one DRAM round trip,
+        // weights requested before the PDL wait), at most 2 CTAs per SM and
+        // clusters of <= 8; large K keeps streaming at the largest such split
+        g.ba = 64;
+        g.bn = M <= 16 ? 16 : 32;
+        g.deep = 0;
+        g.tilesA = (N + 63) / 64;
+        g.tilesB = (M + g.bn - 1) / g.bn;
+        g.nkb = (K + kBlockK - 1) / kBlockK;
+        const int st = g.bn <= 16 ? Cfg<64, 16>::STAGES : Cfg<64, 32>::STAGES;
+        const int tiles = g.tilesA * g.tilesB;
+        int sk = 1;
+        while (sk < 8 && (g.nkb + sk - 1) / sk > st && tiles * (sk + 1) <= 2 * num_sms() && g.nkb >= 2 * (sk + 1)) ++sk;
+        if (sk_env0 > 0) sk = sk_env0 < g.nkb ? sk_env0 : g.nkb;
+        if (sk > kMaxSplitK) sk = kMaxSplitK;
+        g.splitk = sk;
+        return g;
+    }
     g.bn = g.swap ? (M <= 16 ? 16 : (M <= 32 ? 32 : (M <= 64 ? 64 : 128))) : 128;
     static const int bn_env = env_int("FT2_GEMM_BN", 0);   // experiment: force the token-tile width
     if (g.swap && (bn_env == 16 || bn_env == 32 || bn_env == 64)) g.bn = bn_env;
     const int rowsA = g.swap ? N : M, rowsB = g.swap ? M : N;
-    g.tilesA = (rowsA + kBlockA - 1) / kBlockA;
+    g.tilesA = (rowsA + kBlockA - 1) / kBlockA;   // (BA = 128 from here on)
     g.tilesB = (rowsB + g.bn - 1) / g.bn;
     g.nkb = (K + kBlockK - 1) / kBlockK;
     const int tiles = g.tilesA * g.tilesB;
@@ -793,65 +796,41 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
             }
         }
     }
-    static const bool dbg = getenv("FT2_GEMM_DEBUG") != nullptr;
-    if (dbg) {
-        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d bn=%d tiles=%dx%d nkb=%d splitk=%d deep=%d clusters(sk)=", M,
-                N, K, g.swap, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk, g.deep);
-        for (int sk = 2; sk <= 16 && g.swap; ++sk) fprintf(stderr, "%d:%d ", sk, max_clusters_bn(g.bn, sk));
-        int occ = -1;
-        if (g.bn == 32) {
-            set_attrs<32, true, 0, false>();
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gemm_kernel<32, true, 0, false>, kGemmThreads, Cfg<32>::kBytes);
-        }
-        size_t avail2 = 0, avail1 = 0;
-        cudaOccupancyAvailableDynamicSMemPerBlock(&avail2, gemm_kernel<32, true, 0, false>, 2, kGemmThreads);
-        cudaOccupancyAvailableDynamicSMemPerBlock(&avail1, gemm_kernel<32, true, 0, false>, 1, kGemmThreads);
-        cudaFuncAttributes fa;
-        cudaFuncGetAttributes(&fa, gemm_kernel<32, true, 0, false>);
-        int smem_sm = 0, dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
-        fprintf(stderr, " occ(bn32)=%d smem=%d avail@2=%zu avail@1=%zu regs=%d static=%zu maxdyn=%d carve=%d smem/SM=%d\n",
-                occ, Cfg<32>::kBytes, avail2, avail1, fa.numRegs, fa.sharedSizeBytes, fa.maxDynamicSharedSizeBytes,
-                fa.preferredShmemCarveout, smem_sm);
-        cudaGetLastError();   // the occupancy probes above may leave an error behind
-    }
     return g;
 }
 
-// Global-memory K split of the decode kernel: counters at the workspace head,
-// then [tiles][splitk][128][bn] fp32 slots.
-constexpr size_t kDecodeCounterBytes = 65536;
-static size_t decode_gsplit_bytes(const GemmPlan& g) {
-    return kDecodeCounterBytes + (size_t)g.tilesA * g.tilesB * g.splitk * kBlockA * g.bn * 4;
+static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
+    const GemmPlan g = plan_gemm_impl(M, N, K);
+    static const bool dbg = getenv("FT2_GEMM_DEBUG") != nullptr;
+    if (dbg)
+        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d ba=%d bn=%d tiles=%dx%d nkb=%d splitk=%d deep=%d\n", M, N, K,
+                g.swap, g.ba, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk, g.deep);
+    return g;
 }
 
 // The decode kernel's cluster split-K needs no global workspace; the
 // persistent kernel (M > swap_max_m()) uses one for its K splits when the
 // tiles alone cannot fill the machine (optional: less space, fewer splits).
 size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K) {
-    if (M <= swap_max_m()) {
-        if (!env_int("FT2_GEMM_GSPLIT", 0)) return 0;
-        const GemmPlan g = plan_gemm(M, N, K);
-        return g.splitk > 1 ? decode_gsplit_bytes(g) : 0;
-    }
+    if (M <= swap_max_m()) return 0;
     return plan_prefill_split(M, N, K, (size_t)-1).need_bytes;
 }
 
-template <int BN, bool SWAP, int DT, bool DEEP = false>
+template <int BA, int BN, bool SWAP, int DT, bool DEEP = false>
 static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st, int* n_launch) {
     CUtensorMap ma, mb;
     const void* pa = SWAP ? (const void*)a.w : (const void*)a.x;
     const void* pb = SWAP ? (const void*)a.x : (const void*)a.w;
     const int64_t lda = SWAP ? a.ldw : a.ldx, ldb = SWAP ? a.ldx : a.ldw;
-    if (!make_map(&ma, pa, p.rowsA, a.K, lda, kBlockA, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
+    if (!make_map(&ma, pa, p.rowsA, a.K, lda, SWAP ? BA : kBlockA, DT == 1 ? FT2_FP16 : FT2_BF16))
+        return cudaErrorInvalidValue;
     if (!make_map(&mb, pb, p.rowsB, a.K, ldb, BN, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
-    cudaError_t e = set_attrs<BN, SWAP, DT, DEEP>();
+    cudaError_t e = set_attrs<BA, BN, SWAP, DT, DEEP>();
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);
     cfg.blockDim = dim3(kGemmThreads);
-    cfg.dynamicSmemBytes = Cfg<BN, DEEP>::kBytes + smem_pad();
+    cfg.dynamicSmemBytes = Cfg<BA, BN, DEEP>::kBytes + smem_pad();
     cfg.stream = st;
     cudaLaunchAttribute attr[3];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -864,8 +843,8 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     attr[2].id = cudaLaunchAttributeClusterSchedulingPolicyPreference;
     attr[2].val.clusterSchedulingPolicyPreference = cudaClusterSchedulingPolicySpread;
     cfg.attrs = attr;
-    cfg.numAttrs = (p.splitk > 1 && !p.gsplit) ? (spread_policy() ? 3 : 2) : 1;
-    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BN, SWAP, DT, DEEP>, ma, mb, p);
+    cfg.numAttrs = p.splitk > 1 ? (spread_policy() ? 3 : 2) : 1;
+    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BA, BN, SWAP, DT, DEEP>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -910,49 +889,45 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.pf = pf_on ? static_cast<const uint8_t*>(a.l2_prefetch) : nullptr;
     p.pf_bytes = p.pf ? (uint64_t)a.l2_prefetch_bytes : 0;
     p.pf_at = pf_at;
-    // K split through global memory (FT2_GEMM_GSPLIT=1; needs the workspace)
-    static const int gsplit_env = env_int("FT2_GEMM_GSPLIT", 0);
-    p.gsplit = 0;
-    if (gsplit_env && g.splitk > 1 && !g.deep) {
-        const size_t need = decode_gsplit_bytes(g);
-        if (a.ws != nullptr && a.ws_bytes >= need) {
-            p.gsplit = 1;
-            p.gcnt = static_cast<uint32_t*>(a.ws);
-            p.gws = reinterpret_cast<float*>(static_cast<char*>(a.ws) + kDecodeCounterBytes);
-        }
-    }
-    p.rows_per_slot = (kBlockA + g.splitk - 1) / g.splitk;
+    p.rows_per_slot = (g.ba + g.splitk - 1) / g.splitk;
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
 #ifdef FT2_GEMM_TRACE
     p.trace_base = 256 * (g_trace_launch++ % 128);   // graph captures bake one base per captured launch
 #endif
+    if (g.ba == 64) {
+        if (a.dtype == FT2_FP16)
+            return g.bn == 16 ? launch_cfg<64, 16, true, 1>(a, p, st, n_launch)
+                              : launch_cfg<64, 32, true, 1>(a, p, st, n_launch);
+        return g.bn == 16 ? launch_cfg<64, 16, true, 0>(a, p, st, n_launch)
+                          : launch_cfg<64, 32, true, 0>(a, p, st, n_launch);
+    }
     if (g.deep) {
         if (a.dtype == FT2_FP16) {
             switch (g.bn) {
-                case 16: return launch_cfg<16, true, 1, true>(a, p, st, n_launch);
-                case 32: return launch_cfg<32, true, 1, true>(a, p, st, n_launch);
-                default: return launch_cfg<64, true, 1, true>(a, p, st, n_launch);
+                case 16: return launch_cfg<128, 16, true, 1, true>(a, p, st, n_launch);
+                case 32: return launch_cfg<128, 32, true, 1, true>(a, p, st, n_launch);
+                default: return launch_cfg<128, 64, true, 1, true>(a, p, st, n_launch);
             }
         }
         switch (g.bn) {
-            case 16: return launch_cfg<16, true, 0, true>(a, p, st, n_launch);
-            case 32: return launch_cfg<32, true, 0, true>(a, p, st, n_launch);
-            default: return launch_cfg<64, true, 0, true>(a, p, st, n_launch);
+            case 16: return launch_cfg<128, 16, true, 0, true>(a, p, st, n_launch);
+            case 32: return launch_cfg<128, 32, true, 0, true>(a, p, st, n_launch);
+            default: return launch_cfg<128, 64, true, 0, true>(a, p, st, n_launch);
         }
     }
     if (a.dtype == FT2_FP16) {
         switch (g.bn) {
-            case 16: return launch_cfg<16, true, 1>(a, p, st, n_launch);
-            case 32: return launch_cfg<32, true, 1>(a, p, st, n_launch);
-            case 64: return launch_cfg<64, true, 1>(a, p, st, n_launch);
-            default: return launch_cfg<128, true, 1>(a, p, st, n_launch);
+            case 16: return launch_cfg<128, 16, true, 1>(a, p, st, n_launch);
+            case 32: return launch_cfg<128, 32, true, 1>(a, p, st, n_launch);
+            case 64: return launch_cfg<128, 64, true, 1>(a, p, st, n_launch);
+            default: return launch_cfg<128, 128, true, 1>(a, p, st, n_launch);
         }
     }
     switch (g.bn) {
-        case 16: return launch_cfg<16, true, 0>(a, p, st, n_launch);
-        case 32: return launch_cfg<32, true, 0>(a, p, st, n_launch);
-        case 64: return launch_cfg<64, true, 0>(a, p, st, n_launch);
-        default: return launch_cfg<128, true, 0>(a, p, st, n_launch);
+        case 16: return launch_cfg<128, 16, true, 0>(a, p, st, n_launch);
+        case 32: return launch_cfg<128, 32, true, 0>(a, p, st, n_launch);
+        case 64: return launch_cfg<128, 64, true, 0>(a, p, st, n_launch);
+        default: return launch_cfg<128, 128, true, 0>(a, p, st, n_launch);
     }
 }
 
