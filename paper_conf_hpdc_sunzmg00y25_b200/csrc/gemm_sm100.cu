@@ -97,6 +97,9 @@ struct GemmK {
     int32_t rows_per_slot;  // ceil(BA / splitk): rows of one split-K receive slot
     uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
     int32_t trace_base;     // trace builds only: first g_trace row of this launch
+    // cA > 1: clusters (cA, splitk, 1) -- cA feature tiles of the same split
+    // share each x box through a TMA multicast (whole K slice in the ring only)
+    int32_t cA;
     const uint8_t* pf;      // L2 prefetch hint (the next layer's weights) and its size
     uint64_t pf_bytes;
     int32_t pf_at;          // 0: after this CTA issued its last load; 1: after its last stage landed
@@ -344,7 +347,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     __syncthreads();
     tc_fence_after();
     // peers may push into my receive buffer once my barrier is initialised
-    if (cs) cluster_arrive_relaxed();
+    const int cA = p.cA, rA = (int)(blockIdx.x % (unsigned)cA);
+    const bool mc = cA > 1;   // x multicast: every peer's barriers must exist before the first box
+    if (mc) {
+        cluster_arrive_relaxed();
+        cluster_wait();
+    } else if (cs) {
+        cluster_arrive_relaxed();
+    }
     const uint32_t tmem_base = *tmem_base_sh;
     if (p.trigger) griddep_launch();  // the next kernel in the stream may start its prologue (PDL)
 
@@ -369,8 +379,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 griddep_wait();
             }
             FT2_TRACE(2);
-            for (int i = 0; i < pre; ++i)
-                tma_load_2d(mx, &full[i], tiles + i * C::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row);
+            if (mc) {   // one CTA of each cA group issues a box for all of them (nk <= STAGES)
+                const uint16_t mask = (uint16_t)(((1u << cA) - 1u) << (split * cA));
+                for (int i = rA; i < pre; i += cA)
+                    tma_load_2d_mc(mx, &full[i], tiles + i * C::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row, mask);
+            } else {
+                for (int i = 0; i < pre; ++i)
+                    tma_load_2d(mx, &full[i], tiles + i * C::kStageBytes + x_off, (kb0 + i) * kBlockK, x_row);
+            }
             for (int i = STAGES; i < nk; ++i) {
                 const int s = i % STAGES;
                 mbar_wait(&empty[s], ((uint32_t)(i / STAGES) & 1u) ^ 1u);
@@ -467,8 +483,9 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const int own_r0 = (int)(((uint32_t)(owner * BA) * p.sk_magic) >> 24);
         const uint32_t slot_off = (uint32_t)(((split * RS + (a - own_r0)) * C::kRecvStride) * 4);
         const bool local = owner == split;
-        const uint32_t dst = local ? smem_u32(recv) + slot_off : mapa(smem_u32(recv) + slot_off, (uint32_t)owner);
-        const uint32_t dbar = local ? 0u : mapa(smem_u32(recv_bar), (uint32_t)owner);
+        const uint32_t owner_rank = (uint32_t)(rA + owner * cA);   // cluster rank of my row's owner
+        const uint32_t dst = local ? smem_u32(recv) + slot_off : mapa(smem_u32(recv) + slot_off, owner_rank);
+        const uint32_t dbar = local ? 0u : mapa(smem_u32(recv_bar), owner_rank);
         const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
         // finish-loop geometry: item v -> (row lr, column quad c4)
         const int nrow = r1 - r0;
@@ -481,7 +498,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         int64_t ldy = p.ldy;
         uint32_t* counts = (p.counts != nullptr && p.mode == FT2_GEMM_CHECK) ? p.counts : nullptr;
         asm volatile("" : "+l"(y), "+l"(ldy), "+l"(counts));
-        if (cs) cluster_wait();  // every peer's receive barrier is initialised
+        if (cs && !mc) cluster_wait();  // every peer's receive barrier is initialised
         mbar_wait(tmem_full, 0);
         if (e == 0) FT2_TRACE(5);
         tc_fence_after();
@@ -556,7 +573,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         }
     }
     // warps 0 and 1 pair their prologue cluster arrive (no finish work for them)
-    if (cs && warp < 2) cluster_wait();
+    if (cs && !mc && warp < 2) cluster_wait();
     tc_fence_before();
     __syncthreads();
     if (warp == 1) {
@@ -677,7 +694,7 @@ static int deep_stages(int bn) {
 
 // Tiling plan: orientation, feature-tile height BA, token-tile width, split-K factor.
 struct GemmPlan {
-    int swap, ba, bn, tilesA, tilesB, splitk, nkb, deep;
+    int swap, ba, bn, tilesA, tilesB, splitk, nkb, deep, cA;
 };
 
 // 64-row feature tiles (UMMA M = 64) for decode batches of <= 32 tokens:
@@ -687,9 +704,9 @@ static bool use_ba64(int32_t M, int32_t N, int32_t K) {
     if (M > 32) return false;
     if (ba_env == 64) return true;
     if (ba_env == 128) return false;
-    (void)N;
-    (void)K;
-    return false;
+    // measured (C3 / OPT shapes, profiles/r2_gemm_ba64.txt): better at
+    // N, K <= 4096 (Llama v/o 9.1 -> 8.9 us); worse at N = 11008 (18.2 -> 21.1)
+    return N <= 4096 && K <= 4096;
 }
 
 // Largest token count that runs swap-AB on this kernel (BN = 128 token tiles
@@ -703,6 +720,7 @@ static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
     GemmPlan g;
     g.swap = M <= swap_max_m() ? 1 : 0;
     g.ba = 128;
+    g.cA = 1;
     static const int sk_env0 = env_int("FT2_GEMM_SPLITK", 0);
     if (g.swap && use_ba64(M, N, K)) {
         // the smallest split whose K slice fits the ring (one DRAM round trip,
@@ -721,6 +739,11 @@ static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
         if (sk_env0 > 0) sk = sk_env0 < g.nkb ? sk_env0 : g.nkb;
         if (sk > kMaxSplitK) sk = kMaxSplitK;
         g.splitk = sk;
+        // x multicast across 2 feature tiles (clusters (2, splitk)) when the
+        // whole K slice sits in the ring: measured no faster (the late stages
+        // wait for weights, not x; profiles/r2_gemm_ba64.txt) -- FT2_GEMM_XMC=1
+        static const int xmc = env_int("FT2_GEMM_XMC", 0);
+        g.cA = (xmc && (g.nkb + sk - 1) / sk <= st && g.tilesA % 2 == 0 && 2 * sk <= 8) ? 2 : 1;
         return g;
     }
     g.bn = g.swap ? (M <= 16 ? 16 : (M <= 32 ? 32 : (M <= 64 ? 64 : 128))) : 128;
@@ -803,8 +826,8 @@ static GemmPlan plan_gemm(int32_t M, int32_t N, int32_t K) {
     const GemmPlan g = plan_gemm_impl(M, N, K);
     static const bool dbg = getenv("FT2_GEMM_DEBUG") != nullptr;
     if (dbg)
-        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d ba=%d bn=%d tiles=%dx%d nkb=%d splitk=%d deep=%d\n", M, N, K,
-                g.swap, g.ba, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk, g.deep);
+        fprintf(stderr, "[ft2 gemm] M=%d N=%d K=%d swap=%d ba=%d bn=%d tiles=%dx%d nkb=%d splitk=%d deep=%d cA=%d\n", M, N,
+                K, g.swap, g.ba, g.bn, g.tilesA, g.tilesB, g.nkb, g.splitk, g.deep, g.cA);
     return g;
 }
 
@@ -828,7 +851,7 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     cudaError_t e = set_attrs<BA, BN, SWAP, DT, DEEP>();
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);
+    cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);   // tilesA % cA == 0
     cfg.blockDim = dim3(kGemmThreads);
     cfg.dynamicSmemBytes = Cfg<BA, BN, DEEP>::kBytes + smem_pad();
     cfg.stream = st;
@@ -837,13 +860,13 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     static const int pdl = env_int("FT2_GEMM_PDL", 1);
     attr[0].val.programmaticStreamSerializationAllowed = pdl;
     attr[1].id = cudaLaunchAttributeClusterDimension;
-    attr[1].val.clusterDim.x = 1;
+    attr[1].val.clusterDim.x = (unsigned)p.cA;
     attr[1].val.clusterDim.y = (unsigned)p.splitk;
     attr[1].val.clusterDim.z = 1;
     attr[2].id = cudaLaunchAttributeClusterSchedulingPolicyPreference;
     attr[2].val.clusterSchedulingPolicyPreference = cudaClusterSchedulingPolicySpread;
     cfg.attrs = attr;
-    cfg.numAttrs = p.splitk > 1 ? (spread_policy() ? 3 : 2) : 1;
+    cfg.numAttrs = (p.splitk > 1 || p.cA > 1) ? (spread_policy() ? 3 : 2) : 1;
     e = cudaLaunchKernelEx(&cfg, gemm_kernel<BA, BN, SWAP, DT, DEEP>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
@@ -890,6 +913,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.pf_bytes = p.pf ? (uint64_t)a.l2_prefetch_bytes : 0;
     p.pf_at = pf_at;
     p.rows_per_slot = (g.ba + g.splitk - 1) / g.splitk;
+    p.cA = g.cA;
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
 #ifdef FT2_GEMM_TRACE
     p.trace_base = 256 * (g_trace_launch++ % 128);   // graph captures bake one base per captured launch

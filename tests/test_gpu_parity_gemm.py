@@ -249,3 +249,42 @@ def test_gemm_site_overflow_is_never_dropped(ft2, M, N, K, step):
     rc = oracle.protect(ref, bnds)
     chk, cnt = _run(ft2, x, w, b, 1, bounds=bnds, S=1, sites=sites, layer=0, step=step, base_row=base)
     assert np.array_equal(chk, ref) and np.array_equal(cnt, rc)
+
+
+@pytest.mark.parametrize("env", [{"FT2_GEMM_BA": "64"}, {"FT2_GEMM_BA": "128"},
+                                 {"FT2_GEMM_BA": "64", "FT2_GEMM_XMC": "1"}])
+def test_gemm_tile_variants_in_subprocess(env):
+    """The 64- and 128-row feature tiles and the opt-in x multicast (planner
+    knobs read once per process) give results within R8's tolerance and
+    epilogues bit-exact with the oracle applied to their own PLAIN output."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import numpy as np, torch, sys
+sys.path[:0] = [ROOT, ROOT + "/tests"]
+import oracle, ft2_synth
+import paper_conf_hpdc_sunzmg00y25_b200 as ft2
+from gpu_util import dev, host
+for M, N, K in ((32, 2048, 2048), (16, 1024, 512), (32, 4096, 4096), (8, 640, 2304)):
+    x = ft2_synth.gen_bf16((M, K), 20, 5); w = ft2_synth.gen_bf16((N, K), 21, 5, scale_log2=ft2_synth.weight_scale_log2(K))
+    b = ft2_synth.gen_bf16((N,), 22, 5)
+    y = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+    ft2.protect_fused_gemm(dev(x), dev(w), y, bias=dev(b), mode=0)
+    torch.cuda.synchronize(); plain = host(y)
+    yd, _ = oracle.linear_f64(x, w, b)
+    g = plain.astype(np.uint32) << 16
+    gv = g.view(np.float32).astype(np.float64)
+    rms = np.sqrt(np.mean(yd ** 2, axis=1, keepdims=True))
+    assert np.all(np.abs(gv - yd) <= 1e-2 * np.maximum(np.abs(yd), 1e-2 * rms)), (M, N, K)
+    bnd = np.array([[oracle.f64_to_bf16(-0.05), oracle.f64_to_bf16(0.05)]], np.uint16)
+    cnt = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ft2.protect_fused_gemm(dev(x), dev(w), y, bias=dev(b), mode=1, bounds=dev(bnd), num_seqs=1, corrected_count=cnt)
+    torch.cuda.synchronize()
+    ref = plain.copy(); rc = oracle.protect(ref, bnd)
+    assert np.array_equal(host(y), ref) and int(cnt.item()) == int(rc[0]), (M, N, K)
+print("ok")
+'''.replace("ROOT", repr(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
+    r = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env}, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-3000:]
