@@ -1080,7 +1080,10 @@ def c4_row_parallel_decode(dev, world, B, blocks, dev_time, n=5120, R=20):
         for i in range(L):
             rpc(i, ys[i], bias=bias, mode=1, bounds=bnd, num_seqs=B, corrected_count=cnt)
 
-    out = {"layers": L, "shape": [B, n], "tp": world}
+    # one CUDA graph per variant; a gloo group (the one-GPU multi-rank smoke
+    # run) cannot be captured, so there the NCCL-path variant runs eagerly
+    capture = world == 1 or dist.get_backend() == "nccl"
+    out = {"layers": L, "shape": [B, n], "tp": world, "graphs": capture}
     for name, fn in (("nccl_allreduce_plus_protect", nccl_protect), ("fused_allreduce_protect", fused)):
         s_ = torch.cuda.Stream()
         s_.wait_stream(torch.cuda.current_stream())
@@ -1088,10 +1091,13 @@ def c4_row_parallel_decode(dev, world, B, blocks, dev_time, n=5120, R=20):
             fn()
         torch.cuda.current_stream().wait_stream(s_)
         torch.cuda.synchronize()
-        g = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(g):
-            fn()
-        out[name + "_us_per_step"] = dev_time(g.replay, R)
+        if capture:
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                fn()
+            out[name + "_us_per_step"] = dev_time(g.replay, R)
+        else:
+            out[name + "_us_per_step"] = dev_time(fn, 3)
     out["status"] = rpc.status()
     return out
 

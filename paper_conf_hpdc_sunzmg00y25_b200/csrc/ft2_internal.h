@@ -7,6 +7,21 @@
 
 namespace ft2impl {
 
+// Programmatic dependent launch (PDL) contract of this library.  Kernels
+// launched with programmaticStreamSerializationAllowed (the decode and prefill
+// GEMMs) may start while the previous kernel in the stream still runs: before
+// their griddepcontrol.wait they may only touch data no earlier kernel writes
+// (their own shared memory and TMEM, tensor-map prefetches, and -- with
+// FT2_GEMM_W_STATIC -- the static weight tiles).  Every global read of an
+// upstream output (x, bias, bounds, sites, row maps) and EVERY global write
+// (y, counters, workspaces) comes after the wait.  Kernels that trigger their
+// dependents early (griddepcontrol.launch_dependents: the GEMMs after their
+// prologue, ft2_host_norm / ft2_host_act on entry) rely on that rule: a new
+// PDL-launched kernel that wrote before its wait would race with them.
+// tests/test_gpu_host_norm.py::test_pdl_chain_graph_replay checks the chain
+// (norm -> act -> fused GEMM, replayed with changing inputs) bit for bit
+// against stream-ordered launches.
+
 // Workspace of the bounds reduction (u32 words unless noted):
 //   [4s+0] lo slot  = 0x10000 - min key  (0 = no finite value yet)
 //   [4s+1] hi slot  = max key + 1        (0 = none)
