@@ -692,6 +692,36 @@ def kernel_rooflines(runner, dev, ft2):
             "l2_prefetch_hint": bool(runner.l2_prefetch),
             "bytes_per_launch_avg": nbytes / len(launches), "peak_source": peak_src,
             "algorithmic_bytes": "N*K*2 (W) + M*K*2 (x) + M*N*2 (y) + N*2 (bias) per launch"}
+    # ---- the same kernel streaming (large K, not launch-latency bound): M = 32,
+    # 2048 x 65536 (268 MB of weights per launch), two weight copies alternated
+    wbig = [ft2_synth.gen_bf16_torch((2048, 65536), 80 + i, 1, scale_log2=-8, device=dev) for i in range(2)]
+    xbig = ft2_synth.gen_bf16_torch((B, 65536), 82, 1, device=dev)
+    ybig = torch.empty((B, 2048), dtype=torch.bfloat16, device=dev)
+    bwide = torch.tensor([[-3.0e38, 3.0e38]], dtype=torch.bfloat16, device=dev)
+    cnt1 = torch.zeros(1, dtype=torch.int32, device=dev)
+    it = [0]
+
+    def stream_one():
+        it[0] += 1
+        ft2.protect_fused_gemm(xbig, wbig[it[0] % 2], ybig, mode=1 | 16, bounds=bwide, num_seqs=1,
+                               corrected_count=cnt1)
+    for _ in range(3):
+        stream_one()
+    torch.cuda.synchronize()
+    a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a_.record(stream)
+    for _ in range(10):
+        stream_one()
+    b_.record(stream)
+    torch.cuda.synchronize()
+    us_s = 1000.0 * a_.elapsed_time(b_) / 10
+    nb_s = 2048 * 65536 * 2 + B * 65536 * 2 + B * 2048 * 2
+    gemm["streaming"] = {"shape": [B, 2048, 65536], "us": us_s, "achieved": nb_s / us_s / 1e3,
+                         "frac": nb_s / us_s / 1e3 / hbm_peak,
+                         "note": "same kernel with a 268 MB weight stream per launch: the bandwidth it reaches "
+                                 "when not bound by the per-launch dependency chain"}
+    del wbig, xbig
+    torch.cuda.empty_cache()
     # ---- protection kernels at the 1.44 GB size
     rows, n = 65536, 11008
     y = ft2_synth.gen_bf16_torch((rows, n), 11, 5, device=dev)
