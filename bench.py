@@ -101,6 +101,7 @@ class ClockSampler:
         self.nvml = None
         self.lines = []
         self.samples = []     # (sm_mhz, max_mhz, reasons bitmask)
+        self.extra = []       # (mem_mhz, power_w)
 
     def _nvml_handle(self):
         import pynvml as N
@@ -148,6 +149,8 @@ class ClockSampler:
         while not self.stop_ev.is_set():
             try:
                 self.samples.append((N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM), mx, int(get_reasons(h))))
+                # memory clock and board power beside (the bimodal request time)
+                self.extra.append((N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_MEM), N.nvmlDeviceGetPowerUsage(h) / 1e3))
             except Exception:
                 pass
             self.stop_ev.wait(self.period)
@@ -165,9 +168,14 @@ class ClockSampler:
                     "sw_power_cap": 0x4}
             reasons = sorted({n for _, _, r in self.samples for n, b in bits.items() if r & b})
             sm = [c for c, _, _ in self.samples]
+            mem = [m for m, _ in self.extra]
+            pw = [w for _, w in self.extra]
             return {"sm_mhz": statistics.median(sm) if sm else None,
                     "sm_max_mhz": max(m for _, m, _ in self.samples) if self.samples else None,
-                    "reasons": reasons, "samples": len(sm), "source": "nvml"}
+                    "reasons": reasons, "samples": len(sm), "source": "nvml",
+                    "mem_mhz": statistics.median(mem) if mem else None,
+                    "mem_mhz_min": min(mem) if mem else None,
+                    "power_w_median": statistics.median(pw) if pw else None}
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         self.proc.terminate()
@@ -365,6 +373,7 @@ def main():
 
     def timed(mode, K, e2e=False):
         out_host = torch.empty((B, G), dtype=torch.int64).pin_memory()
+        runner.time_phases = not e2e   # per-request prefill / decode split (3 events inside generate)
         barrier()
         torch.cuda.synchronize()
         evs = [torch.cuda.Event(enable_timing=True) for _ in range(K + 1)]
@@ -381,6 +390,11 @@ def main():
         barrier()
         ms = evs[0].elapsed_time(evs[K]) / K
         per_request[(mode, e2e)] = [round(evs[i].elapsed_time(evs[i + 1]), 3) for i in range(K)]
+        if runner.time_phases:
+            per_request[(mode, "phases")] = [(round(e[0].elapsed_time(e[1]), 3), round(e[1].elapsed_time(e[2]), 3))
+                                             for e in runner._phase_events]
+            runner._phase_events = []
+            runner.time_phases = False
         if world > 1:
             t = torch.tensor([ms], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -494,6 +508,7 @@ def main():
                 "d2h_bytes_per_step": B * G * 8},
         "gpu_launches": launches,
         "ms_per_request_timed": per_request.get(("fused", False)),
+        "ms_prefill_decode_per_request_timed": per_request.get(("fused", "phases")),
         "settle_ms_per_request": settle,
         "phases": phases,
         "ft2_activity_per_request": {"corrected_neurons": corrected, "prefill_nonfinite": nonfinite,
