@@ -426,13 +426,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 if (i == 1) FT2_TRACE(12);
                 if (i == nk - 1) FT2_TRACE(13);
                 tc_fence_after();
+                if (i == 2) FT2_TRACE(10);
                 const uint32_t sa = smem_u32(tiles + s * C::kStageBytes);
                 const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + C::kABytes);
 #pragma unroll
                 for (int k = 0; k < kBlockK / kUmmaK; ++k)  // 16 elements = 32 B along K per MMA
                     tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc,
                            (i > 0 || k > 0) ? 1u : 0u);
-                tc_commit(&empty[s]);
+                if (i == 2) FT2_TRACE(15);
+                // release the stage only if the producer will refill it: a
+                // commit costs the issuing thread ~300 cycles (measured), and
+                // with the whole K slice in the ring none is ever refilled
+                if (i + STAGES < nk) tc_commit(&empty[s]);
             }
             tc_commit(tmem_full);
             FT2_TRACE(4);
@@ -447,6 +452,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const int a = BA == 128 ? q * 32 + lane : q * 16 + (lane & 15);
         const bool has_row = BA == 128 || lane < 16;
         griddep_wait();  // bias/bounds/sites/y may belong to the previous kernel
+
         // epilogue tables, gathered while the main loop still streams
         for (int r = e; r < BA; r += 128) {
             row_tab[r] = SWAP ? feature_entry<DT>(p, tileA * BA + r) : token_entry(p, tileA * BA + r);
@@ -914,6 +920,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.pf_at = pf_at;
     p.rows_per_slot = (g.ba + g.splitk - 1) / g.splitk;
     p.cA = g.cA;
+
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
 #ifdef FT2_GEMM_TRACE
     p.trace_base = 256 * (g_trace_launch++ % 128);   // graph captures bake one base per captured launch

@@ -252,7 +252,8 @@ def test_gemm_site_overflow_is_never_dropped(ft2, M, N, K, step):
 
 
 @pytest.mark.parametrize("env", [{"FT2_GEMM_BA": "64"}, {"FT2_GEMM_BA": "128"},
-                                 {"FT2_GEMM_BA": "64", "FT2_GEMM_XMC": "1"}])
+                                 {"FT2_GEMM_BA": "64", "FT2_GEMM_XMC": "1"},
+                                 {"FT2_GEMM_BA": "128", "FT2_GEMM_BN": "16"}])
 def test_gemm_tile_variants_in_subprocess(env):
     """The 64- and 128-row feature tiles and the opt-in x multicast (planner
     knobs read once per process) give results within R8's tolerance and
@@ -266,7 +267,7 @@ sys.path[:0] = [ROOT, ROOT + "/tests"]
 import oracle, ft2_synth
 import paper_conf_hpdc_sunzmg00y25_b200 as ft2
 from gpu_util import dev, host
-for M, N, K in ((32, 2048, 2048), (16, 1024, 512), (32, 4096, 4096), (8, 640, 2304)):
+for M, N, K in ((32, 2048, 2048), (16, 1024, 512), (32, 4096, 4096), (8, 640, 2304), (27, 2048, 1000), (3, 512, 72)):
     x = ft2_synth.gen_bf16((M, K), 20, 5); w = ft2_synth.gen_bf16((N, K), 21, 5, scale_log2=ft2_synth.weight_scale_log2(K))
     b = ft2_synth.gen_bf16((N,), 22, 5)
     y = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
