@@ -35,6 +35,21 @@ for (M, N, K) in [(8, 384, 512), (32, 256, 128), (1, 200, 72), (160, 256, 192)]:
     ft2.protect_fused_gemm(x, w, out, bias=bias, mode=1, bounds=bb, num_seqs=1, corrected_count=c, sites=sites,
                            cur_layer=0, cur_step=1)
     ft2.protect_fused_gemm(x, w, out, bias=bias, mode=0)
+# round 2: 128-row tiles (BA=64 is the default for these shapes), and site
+# lists that overflow (100 directed sites in one row / tile -> the rescan path)
+import numpy as _np
+for (M, N, K) in [(32, 512, 512), (200, 512, 256)]:
+    x = ft2_synth.gen_bf16_torch((M, K), 12, 1, device=dev)
+    w = ft2_synth.gen_bf16_torch((N, K), 13, 1, scale_log2=-4, device=dev)
+    out = torch.empty((M, N), dtype=torch.bfloat16, device=dev)
+    raw = _np.zeros(100, [("trial", "<u4"), ("step", "<u2"), ("layer", "<u2"), ("token", "<u4"), ("col", "<u4"),
+                          ("xor_mask", "<u4"), ("model", "u1"), ("nbits", "u1"), ("pad", "u1", (2,))])
+    raw["step"], raw["col"], raw["xor_mask"] = (1 if M <= 128 else 0), (_np.arange(100) * 7) % 128, 1
+    dsites = torch.from_numpy(raw.view(_np.uint8).copy()).to(dev)
+    base = torch.zeros(100, dtype=torch.int32, device=dev)
+    ft2.protect_fused_gemm(x, w, out, mode=1, bounds=torch.tensor([[-0.3, 0.3]], dtype=torch.bfloat16, device=dev),
+                           num_seqs=1, sites=dsites, n_sites=100, cur_layer=0, cur_step=(1 if M <= 128 else 0),
+                           base_row=base)
 # FP32 variants (bounds with correction, protect, inject)
 y32 = torch.randn((48, 260), device=dev)
 y32.view(-1)[::37] = float("nan")
