@@ -39,6 +39,16 @@ sys.path.insert(0, ROOT)
 METRIC = "protected generated tokens/s (FT2 on critical layers; overhead vs unprotected)"
 
 
+def settle_switched(settle, drop=0.97):
+    """True once the settle requests show the one-time switch to the fast
+    state (a drop of >= 3 % that stayed for the last three requests)."""
+    if len(settle) < 6:
+        return False
+    first = statistics.median(settle[:3])
+    last = settle[-3:]
+    return max(last) <= drop * first and max(last) <= 1.01 * min(last)
+
+
 def workload_name(model, B, T, G):
     return f"{model}-shaped full decode with FT2 (configs[1]), B={B}/GPU, prompt {T}, gen {G}"
 
@@ -422,25 +432,41 @@ def main():
     for _ in range(max(3, args.warmup)):
         runner.generate(prompt, "fused")
     torch.cuda.synchronize()
-    # Settle: per-request times are bimodal right after start-up (measured
-    # 125.7 vs 135.2 ms for the same request, switching a few seconds into
-    # sustained load, with or without the clock sampler), so keep serving
-    # fused requests until >= FT2_BENCH_SETTLE_S seconds have passed and the
-    # last three agree within 1 % (at most 3x that time).  Untimed.
+    # Settle.  A fresh process serves its first requests in a slow state:
+    # the same CUDA-graph replays take ~8 % longer (OPT-1.3B: 122.6 vs 113.6 ms
+    # per request, decode 1.90 vs 1.75 ms per step) at unchanged SM / memory
+    # clocks, with lower board power, then switch once, within one request,
+    # to the fast state and stay there -- measured after 6 s and after 37 s of
+    # sustained load in two runs (tools/bimodal_probe.py,
+    # profiles/r2_bimodal_probe.json).  So: serve fused requests (untimed)
+    # until >= FT2_BENCH_SETTLE_S seconds have passed and the last three agree
+    # within 1 %, then keep serving up to FT2_BENCH_SETTLE_MAX_S seconds in
+    # total in case the switch is still to come (a request 3 % below the
+    # settled level restarts the stability check).  Every request is reported.
     progress("settle")
     settle = []
     t_min = float(os.environ.get("FT2_BENCH_SETTLE_S", "8"))
+    t_max = float(os.environ.get("FT2_BENCH_SETTLE_MAX_S", "60"))
     t0 = time.perf_counter()
+    level = None
     while True:
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         runner.generate(prompt, "fused")
         b.record(stream)
         b.synchronize()
-        settle.append(round(a.elapsed_time(b), 2))
+        ms_req = a.elapsed_time(b)
+        settle.append(round(ms_req, 2))
         el = time.perf_counter() - t0
         last = settle[-3:]
-        if (el >= t_min and len(last) == 3 and max(last) <= 1.01 * min(last)) or el >= 3 * t_min:
+        stable = len(last) == 3 and max(last) <= 1.01 * min(last)
+        if level is not None and ms_req < 0.97 * level:
+            level = None              # the switch: settle again at the new level
+        if level is None and el >= t_min and stable:
+            level = statistics.median(last)
+        if level is not None and (el >= t_max or settle_switched(settle)):
+            break
+        if el >= 1.5 * t_max:
             break
     barrier()
 

@@ -82,14 +82,18 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     const int tid = threadIdx.x;
     const uint32_t v0 = blockIdx.x * chunk, v1 = min(v0 + chunk, total_vec);
     // P = 1 without sites: no handshake, no site list -- straight to the loads
+    // (the shared words are only touched on the prologue path)
     const bool prologue = p.P > 1 || p.sites != nullptr;
-    if (tid == 0) {
-        sh_e = p.P > 1 ? *reinterpret_cast<volatile uint32_t*>(p.epoch) + 1u : 0u;
-        sh_ok = 1u;
-        sh_ns = 0u;
+    uint32_t e = 0u;
+    if (prologue) {
+        if (tid == 0) {
+            sh_e = p.P > 1 ? *reinterpret_cast<volatile uint32_t*>(p.epoch) + 1u : 0u;
+            sh_ok = 1u;
+            sh_ns = 0u;
+        }
+        __syncthreads();
+        e = sh_e;
     }
-    if (prologue) __syncthreads();
-    const uint32_t e = sh_e;
     // ---- 1. signal: my partial (written by the preceding kernel) is ready.
     // P = 1 needs no handshake: stream order already covers my own partial.
     if (p.P > 1 && blockIdx.x == 0 && tid < p.P) {
@@ -119,9 +123,14 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
             if (k < (uint32_t)kARSites) { sh_site_e[k] = (uint32_t)(el - (uint64_t)v0 * 8u); sh_site_m[k] = s.xor_mask; }
         }
     }
-    if (prologue) __syncthreads();
-    if (!prologue || sh_ok) {
-        const uint32_t nsite = prologue ? sh_ns : 0u;   // > kARSites: every site is rescanned per vector (none dropped)
+    bool ok = true;
+    uint32_t nsite = 0u;   // > kARSites: every site is rescanned per vector (none dropped)
+    if (prologue) {
+        __syncthreads();
+        ok = sh_ok != 0u;
+        nsite = sh_ns;
+    }
+    if (ok) {
         for (uint32_t vb = v0 + tid; vb < v1; vb += kARThreads * kVecs) {
             // issue every load of this pass first: kVecs vectors x min(P, 8) partials
             uint4 part[kVecs][kARMaxP];

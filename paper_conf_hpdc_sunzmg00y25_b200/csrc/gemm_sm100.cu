@@ -712,6 +712,8 @@ static bool use_ba64(int32_t M, int32_t N, int32_t K) {
     if (ba_env == 128) return false;
     // measured (C3 / OPT shapes, profiles/r2_gemm_ba64.txt): better at
     // N, K <= 4096 (Llama v/o 9.1 -> 8.9 us); worse at N = 11008 (18.2 -> 21.1)
+    // (also N <= 2048 at any K, i.e. OPT fc2: back to back 7.06 vs 6.90 us per
+    // launch, in situ within noise -- not taken)
     return N <= 4096 && K <= 4096;
 }
 
