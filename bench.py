@@ -1531,25 +1531,20 @@ def protect_sweep(dev, ft2, peaks, R=10):
     return out
 
 
-def c2_matrix(dev, args, rounds=5):
-    """SURVEY.md 8(d) C2 beyond the headline: OPT-1.3B-shaped decode at B = 1
-    (the paper's one-input-per-inference setting, PAPER.md L282, L330) and
-    B = 32, 60 (QA) and 180 (math) generated tokens (L284), and the paper's
-    FP16 (L282) at the headline shape.  Per variant: protected (fused) vs
-    unprotected (off) and fused_plain tokens/s, medians of `rounds` interleaved
-    requests."""
+def decode_variants(dev, variants, prompt_len, rounds=5):
+    """Protected (fused) vs unprotected (off) vs fused_plain generation for
+    (model, B, G, dtype) variants: medians of `rounds` interleaved requests."""
     import torch
 
     from paper_conf_hpdc_sunzmg00y25_b200.runner import CONFIGS, Runner
 
-    cfg = CONFIGS[args.model]
     stream = torch.cuda.current_stream()
     out = {}
-    for B, G, dt in ((1, 60, torch.bfloat16), (1, 180, torch.bfloat16), (32, 180, torch.bfloat16),
-                     (32, 60, torch.float16)):
-        r = Runner(cfg, B, args.prompt, G, seed=1, device=dev, dtype=dt)
+    for model, B, G, dt in variants:
+        cfg = CONFIGS[model]
+        r = Runner(cfg, B, prompt_len, G, seed=1, device=dev, dtype=dt)
         gen = torch.Generator().manual_seed(1234)
-        prompt = torch.randint(0, cfg.vocab, (B, args.prompt), generator=gen).to(dev)
+        prompt = torch.randint(0, cfg.vocab, (B, prompt_len), generator=gen).to(dev)
         modes = ("fused", "off", "fused_plain")
         for m in modes:
             for _ in range(3):
@@ -1568,15 +1563,28 @@ def c2_matrix(dev, args, rounds=5):
             for m, a, b_ in evs:
                 samples[m].append(a.elapsed_time(b_))
         med = {m: statistics.median(v) for m, v in samples.items()}
-        key = f"B{B}_gen{G}_{'fp16' if dt == torch.float16 else 'bf16'}"
+        key = f"{model}_B{B}_gen{G}_{'fp16' if dt == torch.float16 else 'bf16'}"
         out[key] = {"tokens_per_s": {m: B * G / (v / 1e3) for m, v in med.items()},
-                    "ms_per_request": med,
+                    "ms_per_request": med, "protected_layers": r.n_crit,
                     "overhead_pct_vs_unprotected": 100.0 * (1 - med["off"] / med["fused"]),
                     "epilogue_overhead_pct": 100.0 * (1 - med["fused_plain"] / med["fused"])}
         del r
         torch.cuda.empty_cache()
     out["note"] = "medians of interleaved requests (mode order rotated); off = cuBLAS, fused_plain = same GEMM without the check"
     return out
+
+
+def c2_matrix(dev, args, rounds=5):
+    """SURVEY.md 8(d) C2 beyond the headline: OPT-1.3B-shaped decode at B = 1
+    (the paper's one-input-per-inference setting, PAPER.md L282, L330) and
+    B = 32, 60 (QA) and 180 (math) generated tokens (L284), and the paper's
+    FP16 (L282) at the headline shape; plus configs[3]'s Llama-2-13B-shaped
+    model decoded whole on one GPU (P = 1: FT2 on / off tok/s; the
+    tensor-parallel split itself is the c4 leg's bounds exchange)."""
+    import torch
+    return decode_variants(dev, [(args.model, 1, 60, torch.bfloat16), (args.model, 1, 180, torch.bfloat16),
+                                 (args.model, 32, 180, torch.bfloat16), (args.model, 32, 60, torch.float16),
+                                 ("llama-2-13b", 32, 60, torch.bfloat16)], args.prompt, rounds)
 
 
 def prefill_derive_roofline(dev, ft2, peaks, time_it):

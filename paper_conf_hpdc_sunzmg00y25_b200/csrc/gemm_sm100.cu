@@ -356,7 +356,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         cluster_arrive_relaxed();
     }
     const uint32_t tmem_base = *tmem_base_sh;
-    if (p.trigger) griddep_launch();  // the next kernel in the stream may start its prologue (PDL)
+    // the next kernel in the stream may start its prologue (PDL): right here
+    // (trigger 1), or once this CTA's operands are all consumed (trigger 2, by
+    // the MMA thread below) so its early weight requests do not share the
+    // L2 -> SM path with this CTA's own operand stream
+    if (p.trigger == 1) griddep_launch();
 
     if (warp == 0) {
         if (lane == 0) {
@@ -440,6 +444,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 if (i + STAGES < nk) tc_commit(&empty[s]);
             }
             tc_commit(tmem_full);
+            if (p.trigger == 2) griddep_launch();
             FT2_TRACE(4);
         }
     } else {
