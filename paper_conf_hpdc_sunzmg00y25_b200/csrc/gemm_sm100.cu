@@ -346,6 +346,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
+    // the next kernel in the stream may start its prologue (PDL): right here
+    // (trigger 1), or once this CTA's operands are all consumed (trigger 2, by
+    // the MMA thread below) so its early weight requests do not share the
+    // L2 -> SM path with this CTA's own operand stream
+    if (p.trigger == 1) griddep_launch();
     // peers may push into my receive buffer once my barrier is initialised
     const int cA = p.cA, rA = (int)(blockIdx.x % (unsigned)cA);
     const bool mc = cA > 1;   // x multicast: every peer's barriers must exist before the first box
@@ -356,11 +361,6 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         cluster_arrive_relaxed();
     }
     const uint32_t tmem_base = *tmem_base_sh;
-    // the next kernel in the stream may start its prologue (PDL): right here
-    // (trigger 1), or once this CTA's operands are all consumed (trigger 2, by
-    // the MMA thread below) so its early weight requests do not share the
-    // L2 -> SM path with this CTA's own operand stream
-    if (p.trigger == 1) griddep_launch();
 
     if (warp == 0) {
         if (lane == 0) {
