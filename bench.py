@@ -332,7 +332,13 @@ def main():
         # NCCL's init log stays on (communicator sizes are checkable in stderr)
         os.environ.setdefault("NCCL_DEBUG", "INFO")
         os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
-        dist.init_process_group(os.environ.get("FT2_BENCH_BACKEND", "nccl"))
+        # a failing optional leg must not take the headline line down with it:
+        # a stuck collective times out (5 min) and raises instead of killing
+        # the process (CleanUpOnly), and the legs below catch it
+        os.environ.setdefault("TORCH_NCCL_ASYNC_ERROR_HANDLING", "2")
+        import datetime
+        dist.init_process_group(os.environ.get("FT2_BENCH_BACKEND", "nccl"),
+                                timeout=datetime.timedelta(seconds=300))
     local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -566,7 +572,11 @@ def main():
         del runner
         torch.cuda.empty_cache()
         progress("partitioned paths")
-        res["partitioned_paths"] = partitioned_legs(args, dev, rank, world)
+        try:
+            res["partitioned_paths"] = partitioned_legs(args, dev, rank, world)
+        except Exception as e:   # optional leg: record, keep the headline
+            res["partitioned_paths"] = {"error": f"{type(e).__name__}: {e}"[:500]}
+            progress(f"partitioned paths failed: {e}")
     if rank == 0 and world == 1 and not args.no_extras:
         progress("c1 + cpu baseline")
         res["c1_single_layer"] = c1_leg(dev, ft2)
@@ -579,7 +589,10 @@ def main():
     if rank == 0:
         print(json.dumps(res), flush=True)
     if world > 1:
-        dist.destroy_process_group()
+        try:
+            dist.destroy_process_group()
+        except Exception:
+            pass
     return 0
 
 
