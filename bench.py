@@ -617,16 +617,22 @@ def partitioned_legs(args, dev, rank, world, trials_per_rank=512):
         dist.all_reduce(t)
         out["comm_nranks_ok"] = int(t.item()) == world
     progress("c4 TP bounds")
-    out["c4_tp"] = c4_tp_bounds(args, dev, rank, world)
+    try:
+        out["c4_tp"] = c4_tp_bounds(args, dev, rank, world)
+    except Exception as e:
+        out["c4_tp"] = {"error": f"{type(e).__name__}: {e}"[:500]}
     torch.cuda.empty_cache()
     a = copy.copy(args)
     a.trials = trials_per_rank * world
     a.coverage_trials = 0
     progress("c5 campaign")
-    c5 = c5_campaign(a, dev, rank, world)
-    c5["scaling"] = "weak"
-    c5["trials_per_s_per_gpu"] = c5["value"] / world
-    out["c5_campaign"] = c5
+    try:
+        c5 = c5_campaign(a, dev, rank, world)
+        c5["scaling"] = "weak"
+        c5["trials_per_s_per_gpu"] = c5["value"] / world
+        out["c5_campaign"] = c5
+    except Exception as e:
+        out["c5_campaign"] = {"error": f"{type(e).__name__}: {e}"[:500]}
     torch.cuda.empty_cache()
     return out
 
