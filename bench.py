@@ -1169,15 +1169,32 @@ def c4_row_parallel_decode(dev, world, B, blocks, dev_time, n=5120, R=20):
                 dist.all_reduce(bufs[i])
             ft2.protect(bufs[i], bnd, num_seqs=B, corrected_count=cnt)
 
+    def nccl_bias_protect():   # the row-parallel bias is added after the sum (Megatron order)
+        for i in range(L):
+            if world > 1:
+                dist.all_reduce(bufs[i])
+            bufs[i].add_(bias)
+            ft2.protect(bufs[i], bnd, num_seqs=B, corrected_count=cnt)
+
     def fused():
         for i in range(L):
             rpc(i, ys[i], bias=bias, mode=1, bounds=bnd, num_seqs=B, corrected_count=cnt)
+
+    def fused_nobias():   # like-for-like with nccl_allreduce_plus_protect; P = 1 runs in place
+        for i in range(L):
+            rpc(i, rpc.partial(i) if world == 1 else ys[i], mode=1, bounds=bnd, num_seqs=B, corrected_count=cnt)
 
     # one CUDA graph per variant; a gloo group (the one-GPU multi-rank smoke
     # run) cannot be captured, so there the NCCL-path variant runs eagerly
     capture = world == 1 or dist.get_backend() == "nccl"
     out = {"layers": L, "shape": [B, n], "tp": world, "graphs": capture}
-    for name, fn in (("nccl_allreduce_plus_protect", nccl_protect), ("fused_allreduce_protect", fused)):
+    out["variants"] = {"nccl_allreduce_plus_protect": "NCCL sum all-reduce (none at P = 1) + ft2_protect, no bias",
+                       "nccl_allreduce_bias_protect": "NCCL sum all-reduce + bias add (torch) + ft2_protect",
+                       "fused_allreduce_protect": "ft2_allreduce_protect with bias into a separate output",
+                       "fused_allreduce_protect_nobias": "ft2_allreduce_protect without bias (P = 1: in place, "
+                                                         "only changed vectors written)"}
+    for name, fn in (("nccl_allreduce_plus_protect", nccl_protect), ("nccl_allreduce_bias_protect", nccl_bias_protect),
+                     ("fused_allreduce_protect", fused), ("fused_allreduce_protect_nobias", fused_nobias)):
         s_ = torch.cuda.Stream()
         s_.wait_stream(torch.cuda.current_stream())
         with torch.cuda.stream(s_):

@@ -325,23 +325,30 @@ ft2_status ft2_inject_faults(ft2_tensor y, const ft2_fault_site* sites, int32_t 
  * summed in fp32 in rank order 0..P-1 (reading A22), so every rank computes
  * the same bits; the check is ft2_protect's (FT2_GEMM_CHECK) or none
  * (FT2_GEMM_PLAIN: a plain one-shot all-reduce).
- * partials     device array [P] of device pointers: rank t's partial output
- *              [rows x n] (16-bit, row stride ldp) as mapped in THIS process
- *              (this rank's own buffer at index rank).  Double-buffer them:
- *              alternate two buffers per call.
- * flags        device array [P] of device pointers: rank t's flag array of P
+ * partials     HOST array [P] (P <= 64) of device pointers, 16-byte aligned:
+ *              rank t's partial output [rows x n] (16-bit, row stride ldp) as
+ *              mapped in THIS process (this rank's own buffer at index rank).
+ *              Passed by value to the kernel (a captured graph keeps them).
+ *              Double-buffer them: alternate two buffers per call.
+ * flags        HOST array [P] of device pointers: rank t's flag array of P
  *              uint32 (zero-filled once, before the first call of any rank).
  * epoch, done, status  this rank's device uint32 words (zero-filled once):
  *              the call counter, a self-cleaning CTA counter, and an error
  *              word set to 1 if a peer did not arrive within 2^24 polls
  *              (the kernel then returns without writing y).
  * y            this rank's output [rows x n] (ld), 16-bit (bf16 / fp16).
+ *              It may alias partials[rank] only when P == 1 (peers read the
+ *              partials during the call); then, as in ft2_protect, only the
+ *              16-byte vectors whose bits change are written back.
  * bias, row_to_seq, bounds, num_seqs, corrected_count, sites, n_sites,
  * cur_layer, cur_step, base_row: as in ft2_protect_fused_gemm / ft2_protect.
  * Sites: as ft2_inject_faults, none dropped (past 64 in one CTA's chunk the
  * kernel rescans every site).
  * Every rank must make the same sequence of calls with the same shapes.
- * Asynchronous on stream; graph-capturable (the epoch lives in device memory). */
+ * Asynchronous on stream; graph-capturable (the epoch lives in device memory).
+ * Launched with programmatic dependent launch: the kernel runs
+ * griddepcontrol.wait before touching any global memory and releases its own
+ * dependents right after it (FT2_AR_PDL=0 launches it plainly). */
 ft2_status ft2_allreduce_protect(const void* const* partials, int64_t ldp, int32_t P, int32_t rank,
                                  uint32_t* const* flags, uint32_t* epoch, uint32_t* done, uint32_t* status,
                                  ft2_tensor y, const void* bias, ft2_gemm_mode mode,

@@ -331,7 +331,7 @@ ft2_status ft2_allreduce_protect(const void* const* partials, int64_t ldp, int32
     ft2_status s = check_tensor(y);
     if (s != FT2_OK) return s;
     if (y.dtype == FT2_FP32) return FT2_ERR_UNSUPPORTED;
-    if (P < 1 || P > 64 || rank < 0 || rank >= P) return FT2_ERR_INVALID_ARG;
+    if (P < 1 || P > kARMaxRanks || rank < 0 || rank >= P) return FT2_ERR_INVALID_ARG;
     if (partials == nullptr || flags == nullptr || epoch == nullptr || done == nullptr || status == nullptr)
         return FT2_ERR_INVALID_ARG;
     const int32_t m = (int32_t)mode & ~FT2_GEMM_W_STATIC;
@@ -344,12 +344,16 @@ ft2_status ft2_allreduce_protect(const void* const* partials, int64_t ldp, int32
     if (n_sites < 0 || (n_sites > 0 && sites == nullptr)) return FT2_ERR_INVALID_ARG;
     if ((y.rows * (y.n / 8)) >= (int64_t(1) << 31)) return FT2_ERR_UNSUPPORTED;
     if (y.rows == 0 || y.n == 0) return FT2_OK;   // identical on every rank: nobody waits
-    AllreduceProtectArgs a;
-    a.partials = reinterpret_cast<const uint16_t* const*>(partials);
+    AllreduceProtectArgs a = {};
+    for (int t = 0; t < P; ++t) {   // host arrays: every pointer must be set
+        if (partials[t] == nullptr || flags[t] == nullptr) return FT2_ERR_INVALID_ARG;
+        if (!al16(partials[t])) return FT2_ERR_MISALIGNED;
+        a.partials[t] = static_cast<const uint16_t*>(partials[t]);
+        a.flags[t] = flags[t];
+    }
     a.ldp = ldp;
     a.P = P;
     a.rank = rank;
-    a.flags = flags;
     a.epoch = epoch;
     a.done = done;
     a.status = status;

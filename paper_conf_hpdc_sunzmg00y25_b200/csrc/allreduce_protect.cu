@@ -31,6 +31,7 @@
 // `status` and returns (a dead peer cannot hang the GPU).
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "ft2_device.cuh"
 #include "ft2_internal.h"
@@ -63,6 +64,16 @@ __device__ __forceinline__ uint4 ld_peer_v4(const void* p) {
     return r;
 }
 
+// w[d / 2] ^= the 16-bit mask in half d % 2 -- by static indices, so w stays
+// in registers (a dynamic w[d >> 1] would move it to local memory)
+__device__ __forceinline__ void xor_word(uint32_t (&w)[4], uint32_t d, uint32_t mask) {
+    const uint32_t m = (mask & 0xFFFFu) << ((d & 1u) * 16), q = d >> 1;
+    w[0] ^= q == 0u ? m : 0u;   // branch-free selects (an if would be folded back into w[q])
+    w[1] ^= q == 1u ? m : 0u;
+    w[2] ^= q == 2u ? m : 0u;
+    w[3] ^= q == 3u ? m : 0u;
+}
+
 template <int DT>
 __device__ __forceinline__ void add8(float (&acc)[8], uint4 v, bool first) {
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
@@ -73,7 +84,9 @@ __device__ __forceinline__ void add8(float (&acc)[8], uint4 v, bool first) {
     }
 }
 
-template <int DT>
+// PB: partials held in registers per output vector (P <= PB, or PB = 8 and the
+// ranks beyond 8 are streamed) -- a compile-time bound keeps small P lean
+template <int DT, int PB>
 __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const AllreduceProtectArgs p, uint32_t chunk,
                                                                        uint32_t n8, uint32_t total_vec, FastDiv div_n8,
                                                                        int row_mode) {
@@ -84,6 +97,12 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     // P = 1 without sites: no handshake, no site list -- straight to the loads
     // (the shared words are only touched on the prologue path)
     const bool prologue = p.P > 1 || p.sites != nullptr;
+    // programmatic dependent launch: the grid launches while the producer of
+    // the partials (or the previous layer) drains; everything below -- the
+    // epoch, the partials, bias, bounds, sites -- may belong to it.  The next
+    // kernel may start its own prologue right away (it waits likewise).
+    griddep_wait();
+    griddep_launch();
     uint32_t e = 0u;
     if (prologue) {
         if (tid == 0) {
@@ -131,18 +150,38 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
         nsite = sh_ns;
     }
     if (ok) {
+        const int32_t P = p.P;
         for (uint32_t vb = v0 + tid; vb < v1; vb += kARThreads * kVecs) {
-            // issue every load of this pass first: kVecs vectors x min(P, 8) partials
-            uint4 part[kVecs][kARMaxP];
-            uint32_t vrow[kVecs], vc8[kVecs];
+            // every load of this pass is issued before any arithmetic: the
+            // read-only operands (bias, the row's bounds word) first, then
+            // kVecs vectors x min(P, 8) partials (the peer loads carry a memory
+            // clobber, so plain loads placed before them stay before them)
+            uint4 part[kVecs][PB], bv[kVecs];
+            uint32_t vrow[kVecs], vc8[kVecs], bw[kVecs];
+            int vs[kVecs];
 #pragma unroll
             for (int q = 0; q < kVecs; ++q) {
                 const uint32_t v = vb + q * kARThreads;
-                vrow[q] = fdiv(v < v1 ? v : v0, div_n8);
-                vc8[q] = (v < v1 ? v : v0) - vrow[q] * n8;
+                const uint32_t vv = v < v1 ? v : v0;
+                vrow[q] = fdiv(vv, div_n8);
+                vc8[q] = vv - vrow[q] * n8;
+                bv[q] = p.bias ? __ldg(reinterpret_cast<const uint4*>(p.bias + vc8[q] * 8)) : make_uint4(0, 0, 0, 0);
+                vs[q] = -1;
+                bw[q] = 0u;
+                if (p.mode == FT2_GEMM_CHECK) {
+                    const int s = row_mode == 2 ? 0 : (row_mode == 1 ? (int)vrow[q] : __ldg(p.row_to_seq + vrow[q]));
+                    if (s >= 0 && s < p.S) {
+                        vs[q] = s;
+                        bw[q] = __ldg(reinterpret_cast<const uint32_t*>(p.bounds + 2 * s));
+                    }
+                }
+            }
 #pragma unroll
-                for (int t = 0; t < kARMaxP; ++t)
-                    if (t < p.P && v < v1)
+            for (int q = 0; q < kVecs; ++q) {
+                const uint32_t v = vb + q * kARThreads;
+#pragma unroll
+                for (int t = 0; t < PB; ++t)
+                    if (t < P && v < v1)
                         part[q][t] = ld_peer_v4(p.partials[t] + (int64_t)vrow[q] * p.ldp + vc8[q] * 8);
             }
 #pragma unroll
@@ -152,16 +191,15 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
                 const uint32_t row = vrow[q], c8 = vc8[q];
                 float acc[8];
 #pragma unroll
-                for (int t = 0; t < kARMaxP; ++t)
-                    if (t < p.P) add8<DT>(acc, part[q][t], t == 0);
-                for (int t = kARMaxP; t < p.P; ++t)   // rank order continues beyond 8 ranks
+                for (int t = 0; t < PB; ++t)
+                    if (t < P) add8<DT>(acc, part[q][t], t == 0);
+                for (int t = PB; t < P; ++t)   // rank order continues beyond PB ranks
                     add8<DT>(acc, ld_peer_v4(p.partials[t] + (int64_t)row * p.ldp + c8 * 8), false);
                 if (p.bias) {
-                    const uint4 b = *reinterpret_cast<const uint4*>(p.bias + c8 * 8);
-                    const uint32_t bw[4] = {b.x, b.y, b.z, b.w};
+                    const uint32_t bb[4] = {bv[q].x, bv[q].y, bv[q].z, bv[q].w};
 #pragma unroll
                     for (int j = 0; j < 8; ++j)
-                        acc[j] = __fadd_rn(acc[j], to_f32<DT>((uint16_t)(bw[j >> 1] >> ((j & 1) * 16))));
+                        acc[j] = __fadd_rn(acc[j], to_f32<DT>((uint16_t)(bb[j >> 1] >> ((j & 1) * 16))));
                 }
                 uint32_t w[4];
 #pragma unroll
@@ -169,7 +207,7 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
                     w[j] = (uint32_t)rne16<DT>(acc[2 * j]) | ((uint32_t)rne16<DT>(acc[2 * j + 1]) << 16);
                 for (uint32_t i = 0; i < (nsite > (uint32_t)kARSites ? 0u : nsite); ++i) {
                     const uint32_t d = sh_site_e[i] - (v - v0) * 8u;
-                    if (d < 8u) w[d >> 1] ^= (sh_site_m[i] & 0xFFFFu) << ((d & 1) * 16);
+                    if (d < 8u) xor_word(w, d, sh_site_m[i]);
                 }
                 if (nsite > (uint32_t)kARSites) {   // rare overflow path: scan every site
                     for (int i = 0; i < p.n_sites; ++i) {
@@ -179,21 +217,24 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
                                           (p.cur_step == 0 ? (int64_t)st.token : 0);
                         if (r != (int64_t)row || (int64_t)st.col >= p.n) continue;
                         const uint32_t d = (uint32_t)((int64_t)st.col - (int64_t)c8 * 8);
-                        if (d < 8u) w[d >> 1] ^= (st.xor_mask & 0xFFFFu) << ((d & 1) * 16);
+                        if (d < 8u) xor_word(w, d, st.xor_mask);
                     }
                 }
-                if (p.mode == FT2_GEMM_CHECK) {
-                    const int s = row_mode == 2 ? 0 : (row_mode == 1 ? (int)row : p.row_to_seq[row]);
-                    if (s >= 0 && s < p.S) {
-                        const uint32_t k = key2(*reinterpret_cast<const uint32_t*>(p.bounds + 2 * s));
-                        const uint32_t kL2 = (k & 0xFFFFu) * 0x10001u, kH2 = (k >> 16) * 0x10001u;
-                        uint32_t cnt = 0, c;
+                if (vs[q] >= 0) {
+                    const uint32_t k = key2(bw[q]);
+                    const uint32_t kL2 = (k & 0xFFFFu) * 0x10001u, kH2 = (k >> 16) * 0x10001u;
+                    uint32_t cnt = 0, c;
 #pragma unroll
-                        for (int j = 0; j < 4; ++j) { w[j] = clip2<DT>(w[j], kL2, kH2, &c); cnt += c; }
-                        if (cnt && p.counts) atomicAdd(&p.counts[s], cnt);
-                    }
+                    for (int j = 0; j < 4; ++j) { w[j] = clip2<DT>(w[j], kL2, kH2, &c); cnt += c; }
+                    if (cnt && p.counts) atomicAdd(&p.counts[vs[q]], cnt);
                 }
-                *reinterpret_cast<uint4*>(p.y + (int64_t)row * p.ldy + c8 * 8) = make_uint4(w[0], w[1], w[2], w[3]);
+                uint16_t* const dst = p.y + (int64_t)row * p.ldy + c8 * 8;
+                // P = 1 in place (y aliases the partial): like ft2_protect, a
+                // vector is written back only when the check changed it
+                if (P == 1 && dst == p.partials[0] + (int64_t)row * p.ldp + c8 * 8 && w[0] == part[q][0].x &&
+                    w[1] == part[q][0].y && w[2] == part[q][0].z && w[3] == part[q][0].w)
+                    continue;
+                *reinterpret_cast<uint4*>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
             }
         }
     }
@@ -201,10 +242,7 @@ __global__ void __launch_bounds__(kARThreads) allreduce_protect_kernel(const All
     // P = 1: nobody reads the epoch within a call, so CTA 0 advances it
     // without the completion counter (it stays the call counter)
     if (p.P == 1) {
-        if (blockIdx.x == 0 && tid == 0) {
-            volatile uint32_t* ep = reinterpret_cast<volatile uint32_t*>(p.epoch);
-            *ep = *ep + 1u;
-        }
+        if (blockIdx.x == 0 && tid == 0) atomicAdd(p.epoch, 1u);   // fire-and-forget (RED), no round trip
         return;
     }
     __syncthreads();
@@ -228,10 +266,25 @@ cudaError_t launch_allreduce_protect(const AllreduceProtectArgs& a, cudaStream_t
     uint32_t chunk = (total + grid - 1) / grid;
     grid = (total + chunk - 1) / chunk;
     const int row_mode = a.row_to_seq ? 0 : (a.S == 1 ? 2 : 1);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kARThreads);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    static const int pdl = [] { const char* v = getenv("FT2_AR_PDL"); return v ? atoi(v) : 1; }();
+    attr[0].val.programmaticStreamSerializationAllowed = pdl;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    const FastDiv dv = make_fastdiv(n8);
+    cudaError_t e;
+#define FT2_AR_LAUNCH(DT_, PB_) cudaLaunchKernelEx(&cfg, allreduce_protect_kernel<DT_, PB_>, a, chunk, n8, total, dv, row_mode)
     if (a.dtype == FT2_FP16)
-        allreduce_protect_kernel<1><<<grid, kARThreads, 0, st>>>(a, chunk, n8, total, make_fastdiv(n8), row_mode);
+        e = a.P == 1 ? FT2_AR_LAUNCH(1, 1) : a.P == 2 ? FT2_AR_LAUNCH(1, 2) : a.P <= 4 ? FT2_AR_LAUNCH(1, 4) : FT2_AR_LAUNCH(1, kARMaxP);
     else
-        allreduce_protect_kernel<0><<<grid, kARThreads, 0, st>>>(a, chunk, n8, total, make_fastdiv(n8), row_mode);
+        e = a.P == 1 ? FT2_AR_LAUNCH(0, 1) : a.P == 2 ? FT2_AR_LAUNCH(0, 2) : a.P <= 4 ? FT2_AR_LAUNCH(0, 4) : FT2_AR_LAUNCH(0, kARMaxP);
+#undef FT2_AR_LAUNCH
+    if (e != cudaSuccess) return e;
     ++*n_launch;
     return cudaGetLastError();
 }

@@ -125,11 +125,14 @@ cudaError_t launch_inject32(void* y, int64_t rows, int64_t n, int64_t ld, const 
                             cudaStream_t st, int* n_launch);
 
 // Row-parallel sum all-reduce fused with the check (allreduce_protect.cu).
+constexpr int kARMaxRanks = 64;
 struct AllreduceProtectArgs {
-    const uint16_t* const* partials;  // device array [P] of (peer-mapped) partial outputs
+    // the P (peer-mapped) partial outputs and flag arrays, by value in the
+    // kernel parameters: no dependent pointer load before the data loads
+    const uint16_t* partials[kARMaxRanks];
     int64_t ldp;
     int32_t P, rank;
-    uint32_t* const* flags;           // device array [P]: rank t's flag array [P]
+    uint32_t* flags[kARMaxRanks];     // rank t's flag array [P]
     uint32_t* epoch;                  // this rank's call counter (device)
     uint32_t* done;                   // this rank's CTA completion counter (device, self-cleaning)
     uint32_t* status;                 // this rank's error word (1 = peer timeout)

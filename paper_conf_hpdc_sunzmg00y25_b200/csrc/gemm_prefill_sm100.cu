@@ -435,7 +435,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     if (d < 32u) {
 #pragma unroll
                         for (int j = 0; j < 16; ++j)
-                            if ((d >> 1) == (uint32_t)j) w[j] ^= site_m[i] << ((d & 1u) * 16);
+                            w[j] ^= (d >> 1) == (uint32_t)j ? site_m[i] << ((d & 1u) * 16) : 0u;   // branch-free: w stays in registers
                     }
                 }
                 if (site_scan) {   // rare overflow path: every site, straight from global memory
@@ -448,7 +448,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
                         if (r != m || (int64_t)st.col >= p.N || d >= 32u) continue;
 #pragma unroll
                         for (int j = 0; j < 16; ++j)
-                            if ((d >> 1) == (uint32_t)j) w[j] ^= (st.xor_mask & 0xFFFFu) << ((d & 1u) * 16);
+                            w[j] ^= (d >> 1) == (uint32_t)j ? (st.xor_mask & 0xFFFFu) << ((d & 1u) * 16) : 0u;
                     }
                 }
                 if (p.mode == FT2_GEMM_CHECK && seq >= 0) {
@@ -480,7 +480,9 @@ __global__ void __launch_bounds__(kPThreads, 1)
 #pragma unroll
                     for (int j = 0; j < 4; ++j) dst[j] = make_uint4(w[4 * j], w[4 * j + 1], w[4 * j + 2], w[4 * j + 3]);
                 } else {
-                    for (int j = 0; j < nvalid; ++j) yrow[nb + j] = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
+#pragma unroll
+                    for (int j = 0; j < 32; ++j)   // static indices into w (a runtime bound would spill w to local memory)
+                        if (j < nvalid) yrow[nb + j] = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
                 }
             }
             // accumulator buffer drained: hand it back to the MMA warp (the leader's)

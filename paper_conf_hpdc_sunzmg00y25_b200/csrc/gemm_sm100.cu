@@ -70,9 +70,18 @@ __device__ __forceinline__ void trace(int slot, int base) {
     if (cta < 256 && base + cta < FT2_TRACE_ROWS) g_trace[(base + cta) * 16 + slot] = t;
 }
 #define FT2_TRACE(slot) trace(slot, p.trace_base)
+// slot 10 holds the SM id + 1 of the CTA (CTAs of one launch sharing an SM share its tensor pipe)
+__device__ __forceinline__ void trace_smid(int base) {
+    uint32_t sm;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    const int cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+    if (cta < 256 && base + cta < FT2_TRACE_ROWS) g_trace[(base + cta) * 16 + 10] = sm + 1u;
+}
+#define FT2_TRACE_SMID() trace_smid(p.trace_base)
 static int g_trace_launch = 0;   // host: launches since the last ft2_debug_trace_reset
 #else
 #define FT2_TRACE(slot) ((void)0)
+#define FT2_TRACE_SMID() ((void)0)
 #endif
 
 struct GemmK {
@@ -103,6 +112,14 @@ struct GemmK {
     const uint8_t* pf;      // L2 prefetch hint (the next layer's weights) and its size
     uint64_t pf_bytes;
     int32_t pf_at;          // 0: after this CTA issued its last load; 1: after its last stage landed
+    // (host-side selector of the MMA2 instantiation; the kernel uses the template flag)
+    // 1: two MMA issuers -- warp 1 and, once it has issued every load (whole K
+    // slice in the ring), warp 0's producer thread -- each issuing half of
+    // every stage's MMAs into its own accumulator (TMEM columns [0, BN) and
+    // [cols, cols + BN)), summed in that order by the epilogue.  Measured: one
+    // thread issues an M = 64 kind::f16 MMA every ~53 cycles, two warps
+    // together one every ~35 (profiles/r2_mma_probe.txt)
+    int32_t mma2;
 };
 
 // Per-row / per-column epilogue table entry.  Feature side: bias, flags
@@ -272,7 +289,7 @@ __device__ __forceinline__ void finish4(uint16_t* __restrict__ y, int64_t ldy, i
     }
 }
 
-template <int BA, int BN, bool SWAP, int DT, bool DEEP>
+template <int BA, int BN, bool SWAP, int DT, bool DEEP, bool MMA2 = false>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
                 const __grid_constant__ GemmK p) {
@@ -311,10 +328,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 
     if (warp == 0 && lane == 0) {
         FT2_TRACE(0);
+        FT2_TRACE_SMID();
         prefetch_tmap(&map_a);
         prefetch_tmap(&map_b);
         for (int s = 0; s < STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-        mbar_init(tmem_full, 1);
+        mbar_init(tmem_full, MMA2 ? 2u : 1u);
         mbar_init(recv_bar, 1);
         if (cs)  // bytes the other splits will push into my slice
             mbar_expect_tx(recv_bar, (uint32_t)((splitk - 1) * (r1 - r0) * BN * 4));
@@ -335,14 +353,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             // right away (no shared memory needed), so the whole layer
             // streams from HBM while this kernel still waits for its
             // activations; the ring's later loads then hit L2
-            if (p.w_l2) {   // at most one more ring's worth (a whole large slice would thrash L2)
-                const int lim = nk < pre + STAGES ? nk : pre + STAGES;
+            if (p.w_l2) {   // one more ring's worth (w_l2 1), or the whole slice (w_l2 2: layers that fit L2 easily)
+                const int lim = (p.w_l2 >= 2 || nk < pre + STAGES) ? nk : pre + STAGES;
                 for (int i = pre; i < lim; ++i)
                     tma_prefetch_l2_2d(SWAP ? &map_a : &map_b, (kb0 + i) * kBlockK, SWAP ? tileA * BA : tileB * BN);
             }
         }
     }
-    if (warp == 1) tmem_alloc(tmem_base_sh, C::kTmemCols);
+    if (warp == 1) tmem_alloc(tmem_base_sh, (MMA2 ? 2u : 1u) * C::kTmemCols);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
@@ -399,6 +417,25 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 tma_load_2d(mw, &full[s], st + w_off, (kb0 + i) * kBlockK, w_row);
                 tma_load_2d(mx, &full[s], st + x_off, (kb0 + i) * kBlockK, x_row);
             }
+            if constexpr (MMA2) {
+                // second MMA issuer (the host sets mma2 only when nk <= STAGES:
+                // no stage is ever refilled, so no stage release is needed):
+                // the upper half of every stage's K16 steps into accumulator 1
+                constexpr uint32_t idesc2 =
+                    (make_idesc(BA, BN) & ~((7u << 7) | (7u << 10))) | ((DT == 1 ? 0u : 1u) * ((1u << 7) | (1u << 10)));
+                for (int i = 0; i < nk; ++i) {
+                    const int s = i % STAGES;
+                    mbar_wait(&full[s], (uint32_t)(i / STAGES) & 1u);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(tiles + s * C::kStageBytes);
+                    const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + C::kABytes);
+#pragma unroll
+                    for (int k = kBlockK / kUmmaK / 2; k < kBlockK / kUmmaK; ++k)
+                        tc_mma(tmem_base + C::kTmemCols, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc2,
+                               (i > 0 || k > kBlockK / kUmmaK / 2) ? 1u : 0u);
+                }
+                tc_commit(tmem_full);
+            }
             if (p.pf_bytes) {
                 // L2 prefetch hint: this CTA's 1/grid share of the next
                 // layer's bytes, once its own loads are issued (pf_at 0) or
@@ -430,13 +467,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 if (i == 1) FT2_TRACE(12);
                 if (i == nk - 1) FT2_TRACE(13);
                 tc_fence_after();
-                if (i == 2) FT2_TRACE(10);
                 const uint32_t sa = smem_u32(tiles + s * C::kStageBytes);
                 const uint64_t da = make_sdesc(sa), db = make_sdesc(sa + C::kABytes);
+                if constexpr (MMA2) {   // the lower half of the stage's K16 steps (the producer issues the rest)
 #pragma unroll
-                for (int k = 0; k < kBlockK / kUmmaK; ++k)  // 16 elements = 32 B along K per MMA
-                    tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc,
-                           (i > 0 || k > 0) ? 1u : 0u);
+                    for (int k = 0; k < kBlockK / kUmmaK / 2; ++k)
+                        tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc, (i > 0 || k > 0) ? 1u : 0u);
+                } else {
+#pragma unroll
+                    for (int k = 0; k < kBlockK / kUmmaK; ++k)  // 16 elements = 32 B along K per MMA
+                        tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc,
+                               (i > 0 || k > 0) ? 1u : 0u);
+                }
                 if (i == 2) FT2_TRACE(15);
                 // release the stage only if the producer will refill it: a
                 // commit costs the issuing thread ~300 cycles (measured), and
@@ -519,6 +561,13 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         if constexpr (BN == 32) {  // one TMEM load for the whole row, then the pushes back to back
             uint32_t r[32];
             tmem_ld32(taddr, r);
+            if constexpr (MMA2) {   // + the second issuer's accumulator (fixed order: deterministic)
+                uint32_t r2[32];
+                tmem_ld32(taddr + C::kTmemCols, r2);
+                tmem_wait_ld();
+#pragma unroll
+                for (int j = 0; j < 32; ++j) r[j] = __float_as_uint(__uint_as_float(r[j]) + __uint_as_float(r2[j]));
+            }
             tmem_wait_ld();
             if (e == 0) FT2_TRACE(14);
             if (nk == 0) {
@@ -537,6 +586,13 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         for (int c0 = 0; c0 < BN; c0 += 16) {
             uint32_t r[16];
             tmem_ld16(taddr + c0, r);
+            if constexpr (MMA2) {
+                uint32_t r2[16];
+                tmem_ld16(taddr + C::kTmemCols + c0, r2);
+                tmem_wait_ld();
+#pragma unroll
+                for (int j = 0; j < 16; ++j) r[j] = __float_as_uint(__uint_as_float(r[j]) + __uint_as_float(r2[j]));
+            }
             tmem_wait_ld();
             if (e == 0 && c0 == 0) FT2_TRACE(14);
             if (nk == 0) {
@@ -589,7 +645,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     __syncthreads();
     if (warp == 1) {
         tc_fence_after();
-        tmem_dealloc(tmem_base, C::kTmemCols);
+        tmem_dealloc(tmem_base, (MMA2 ? 2u : 1u) * C::kTmemCols);
     }
 }
 
@@ -636,10 +692,10 @@ static int spread_policy() {
     return v;
 }
 
-template <int BA, int BN, bool SWAP, int DT, bool DEEP>
+template <int BA, int BN, bool SWAP, int DT, bool DEEP, bool MMA2 = false>
 static cudaError_t set_attrs() {
     static cudaError_t res = [] {
-        auto* k = gemm_kernel<BA, BN, SWAP, DT, DEEP>;
+        auto* k = gemm_kernel<BA, BN, SWAP, DT, DEEP, MMA2>;
         cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              Cfg<BA, BN, DEEP>::kBytes + smem_pad());
         if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
@@ -748,7 +804,8 @@ static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
         const int st = g.bn <= 16 ? Cfg<64, 16>::STAGES : Cfg<64, 32>::STAGES;
         const int tiles = g.tilesA * g.tilesB;
         int sk = 1;
-        while (sk < 8 && (g.nkb + sk - 1) / sk > st && tiles * (sk + 1) <= 2 * num_sms() && g.nkb >= 2 * (sk + 1)) ++sk;
+        static const int cap64 = env_int("FT2_GEMM_CTA_CAP", 2 * num_sms());   // experiment: CTAs per launch
+        while (sk < 8 && (g.nkb + sk - 1) / sk > st && tiles * (sk + 1) <= cap64 && g.nkb >= 2 * (sk + 1)) ++sk;
         if (sk_env0 > 0) sk = sk_env0 < g.nkb ? sk_env0 : g.nkb;
         if (sk > kMaxSplitK) sk = kMaxSplitK;
         g.splitk = sk;
@@ -793,7 +850,8 @@ static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
     // between 33 and 64 tiles the in-situ optimum sits lower (measured at
     // N = 6144: 240 CTAs 15.7 us, 288 CTAs 20.4 us, cuBLAS 13.7 us;
     // profiles/r1c_splitk_mid.txt), so those shapes cap the grid at 240
-    const int cta_cap = (tiles > 32 && tiles <= 64) ? 240 : 2 * sms;
+    static const int cap_env = env_int("FT2_GEMM_CTA_CAP", 0);   // experiment: CTAs per launch
+    const int cta_cap = cap_env > 0 ? cap_env : ((tiles > 32 && tiles <= 64) ? 240 : 2 * sms);
     if (g.swap) {
         for (int sk = 2; sk <= sk_cap; ++sk) {
             if (tiles * sk > cta_cap || g.nkb < 4 * sk) break;
@@ -852,7 +910,7 @@ size_t gemm_ws_bytes(int32_t M, int32_t N, int32_t K) {
     return plan_prefill_split(M, N, K, (size_t)-1).need_bytes;
 }
 
-template <int BA, int BN, bool SWAP, int DT, bool DEEP = false>
+template <int BA, int BN, bool SWAP, int DT, bool DEEP = false, bool MMA2 = false>
 static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st, int* n_launch) {
     CUtensorMap ma, mb;
     const void* pa = SWAP ? (const void*)a.w : (const void*)a.x;
@@ -861,7 +919,7 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     if (!make_map(&ma, pa, p.rowsA, a.K, lda, SWAP ? BA : kBlockA, DT == 1 ? FT2_FP16 : FT2_BF16))
         return cudaErrorInvalidValue;
     if (!make_map(&mb, pb, p.rowsB, a.K, ldb, BN, DT == 1 ? FT2_FP16 : FT2_BF16)) return cudaErrorInvalidValue;
-    cudaError_t e = set_attrs<BA, BN, SWAP, DT, DEEP>();
+    cudaError_t e = set_attrs<BA, BN, SWAP, DT, DEEP, MMA2>();
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)p.tilesA, (unsigned)p.splitk, (unsigned)p.tilesB);   // tilesA % cA == 0
@@ -880,7 +938,7 @@ static cudaError_t launch_cfg(const GemmArgs& a, const GemmK& p, cudaStream_t st
     attr[2].val.clusterSchedulingPolicyPreference = cudaClusterSchedulingPolicySpread;
     cfg.attrs = attr;
     cfg.numAttrs = (p.splitk > 1 || p.cA > 1) ? (spread_policy() ? 3 : 2) : 1;
-    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BA, BN, SWAP, DT, DEEP>, ma, mb, p);
+    e = cudaLaunchKernelEx(&cfg, gemm_kernel<BA, BN, SWAP, DT, DEEP, MMA2>, ma, mb, p);
     ++*n_launch;
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -919,7 +977,8 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     static const int trig = env_int("FT2_GEMM_TRIGGER", 1);
     p.trigger = trig;
     static const int wl2 = env_int("FT2_GEMM_W_L2", 0);
-    p.w_l2 = wl2;
+    static const int64_t wl2_max = (int64_t)env_int("FT2_GEMM_W_L2_MAX_MB", 48) << 20;
+    p.w_l2 = (wl2 >= 2 && (int64_t)a.N * a.K * 2 > wl2_max) ? 1 : wl2;
     static const int pf_on = env_int("FT2_GEMM_PF", 1);      // experiments: 0 ignores the hint
     static const int pf_at = env_int("FT2_GEMM_PF_AT", 1);
     p.pf = pf_on ? static_cast<const uint8_t*>(a.l2_prefetch) : nullptr;
@@ -927,6 +986,11 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.pf_at = pf_at;
     p.rows_per_slot = (g.ba + g.splitk - 1) / g.splitk;
     p.cA = g.cA;
+    {   // two MMA issuers: 64-row tiles whose whole K slice sits in the ring (FT2_GEMM_MMA2=0 turns it off)
+        static const int mma2_env = env_int("FT2_GEMM_MMA2", 1);
+        const int st = g.bn <= 16 ? Cfg<64, 16>::STAGES : Cfg<64, 32>::STAGES;
+        p.mma2 = (mma2_env && g.ba == 64 && g.cA == 1 && (g.nkb + g.splitk - 1) / g.splitk <= st) ? 1 : 0;
+    }
 
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
 #ifdef FT2_GEMM_TRACE
@@ -934,10 +998,14 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
 #endif
     if (g.ba == 64) {
         if (a.dtype == FT2_FP16)
-            return g.bn == 16 ? launch_cfg<64, 16, true, 1>(a, p, st, n_launch)
-                              : launch_cfg<64, 32, true, 1>(a, p, st, n_launch);
-        return g.bn == 16 ? launch_cfg<64, 16, true, 0>(a, p, st, n_launch)
-                          : launch_cfg<64, 32, true, 0>(a, p, st, n_launch);
+            return p.mma2 ? (g.bn == 16 ? launch_cfg<64, 16, true, 1, false, true>(a, p, st, n_launch)
+                                        : launch_cfg<64, 32, true, 1, false, true>(a, p, st, n_launch))
+                          : (g.bn == 16 ? launch_cfg<64, 16, true, 1>(a, p, st, n_launch)
+                                        : launch_cfg<64, 32, true, 1>(a, p, st, n_launch));
+        return p.mma2 ? (g.bn == 16 ? launch_cfg<64, 16, true, 0, false, true>(a, p, st, n_launch)
+                                    : launch_cfg<64, 32, true, 0, false, true>(a, p, st, n_launch))
+                      : (g.bn == 16 ? launch_cfg<64, 16, true, 0>(a, p, st, n_launch)
+                                    : launch_cfg<64, 32, true, 0>(a, p, st, n_launch));
     }
     if (g.deep) {
         if (a.dtype == FT2_FP16) {

@@ -187,14 +187,18 @@ def version() -> str:
 def allreduce_protect(partial_ptrs, ldp, P, rank, flag_ptrs, words, y, bias=None, mode=FT2_GEMM_CHECK, bounds=None,
                       row_to_seq=None, num_seqs=None, corrected_count=None, sites=None, n_sites=None, cur_layer=0,
                       cur_step=0, base_row=None, stream=None):
-    """ft2_allreduce_protect.  partial_ptrs / flag_ptrs: device int64 [P]
-    tensors of (peer-mapped) pointers; words: device int32 [3] (epoch, done,
-    status) of this rank; y: this rank's output."""
+    """ft2_allreduce_protect.  partial_ptrs / flag_ptrs: sequences of P
+    (peer-mapped) device addresses (host ints); words: device int32 [3]
+    (epoch, done, status) of this rank; y: this rank's output."""
     t = _as_ft2_tensor(y)
     S = num_seqs if num_seqs is not None else (bounds.numel() // 2 if bounds is not None else 0)
     ns = 0 if sites is None else (n_sites if n_sites is not None else sites.numel() // SITE_BYTES)
     wp = words.data_ptr()
-    st = load().ft2_allreduce_protect(_ptr(partial_ptrs), int(ldp), int(P), int(rank), _ptr(flag_ptrs),
+    if len(partial_ptrs) != P or len(flag_ptrs) != P:
+        raise ValueError("allreduce_protect: one partial and one flag pointer per rank")
+    pp = (ctypes.c_void_p * P)(*[int(v) for v in partial_ptrs])
+    fp = (ctypes.c_void_p * P)(*[int(v) for v in flag_ptrs])
+    st = load().ft2_allreduce_protect(pp, int(ldp), int(P), int(rank), fp,
                                       ctypes.c_void_p(wp), ctypes.c_void_p(wp + 4), ctypes.c_void_p(wp + 8), t,
                                       _ptr(bias), int(mode), _ptr(row_to_seq), _ptr(bounds), S,
                                       _ptr(corrected_count), _ptr(sites), ns, cur_layer, cur_step, _ptr(base_row),

@@ -103,8 +103,8 @@ class RowParallelCheck:
                 bp, bf = basep + op, basef + of
             pptr.append((bp, bp + rows * n * elt))
             fptr.append(bf)
-        self.partial_ptrs = [torch.tensor([p[b] for p in pptr], dtype=torch.int64, device=dev) for b in (0, 1)]
-        self.flag_ptrs = torch.tensor(fptr, dtype=torch.int64, device=dev)
+        self.partial_ptrs = [[p[b] for p in pptr] for b in (0, 1)]   # host ints, passed by value
+        self.flag_ptrs = list(fptr)
         dist.barrier(group=group)   # every rank mapped everything before any call
 
     def partial(self, i: int) -> torch.Tensor:

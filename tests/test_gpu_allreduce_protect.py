@@ -202,3 +202,34 @@ def test_allreduce_protect_site_overflow_p1():
         assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), wcnt)
     finally:
         dist.destroy_process_group()
+
+
+def test_allreduce_protect_p1_in_place():
+    """P = 1 with y aliasing this rank's partial and no bias: the kernel writes
+    back only the vectors the check (or a fault site) changed, like
+    ft2_protect -- the result must still equal the oracle bit for bit, both
+    where vectors were rewritten (clipped, faulted) and where they were not."""
+    from paper_conf_hpdc_sunzmg00y25_b200 import tp
+    port = _port()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        from gpu_util import dev, host, sites_to_dev
+        rpc = tp.RowParallelCheck(ROWS, N)
+        for i in range(CALLS):
+            parts, _, bounds, sites = _inputs(i, 1)
+            y = rpc.partial(i)
+            y.copy_(dev(parts[0]))
+            cnt = torch.zeros(ROWS, dtype=torch.int32, device="cuda")
+            rpc(i, y, mode=1, bounds=dev(bounds), num_seqs=ROWS, corrected_count=cnt,
+                sites=sites_to_dev(sites), n_sites=ROWS, cur_layer=0, cur_step=1)
+            torch.cuda.synchronize()
+            want, wcnt = oracle.allreduce_protect(parts[:1], bounds_=bounds, sites=sites, cur_layer=0, cur_step=1)
+            got = host(y)
+            assert np.array_equal(got, want), i
+            assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), wcnt), i
+            changed = (want != parts[0]).reshape(ROWS, N // 8, 8).any(axis=2)
+            assert changed.any() and not changed.all()   # both paths ran
+        assert rpc.status() == 0
+    finally:
+        dist.destroy_process_group()

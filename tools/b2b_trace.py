@@ -8,8 +8,9 @@ the gap between consecutive launches' last end."""
 import ctypes, os, sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 CLK = bool(os.environ.get("CLOCK"))   # libft2_trace_clk.so: slots hold %clock64 (SM cycles)
+NOTRACE = os.environ.get("NOTRACE") == "1"   # the product library: timing line only
 os.environ["FT2_LIB"] = os.path.join(ROOT, "paper_conf_hpdc_sunzmg00y25_b200", "lib",
-                                     "libft2_trace_clk.so" if CLK else "libft2_trace.so")
+                                     os.environ.get("LIBNAME", "libft2.so") if NOTRACE else ("libft2_trace_clk.so" if CLK else "libft2_trace.so"))
 sys.path.insert(0, ROOT)
 import numpy as np
 import torch
@@ -18,8 +19,9 @@ from paper_conf_hpdc_sunzmg00y25_b200 import _lib
 import ft2_synth
 
 L = _lib.load()
-L.ft2_debug_trace_read.argtypes = [ctypes.c_void_p, ctypes.c_size_t]
-L.ft2_debug_trace_reset.argtypes = [ctypes.c_int]
+if not NOTRACE:
+  L.ft2_debug_trace_read.argtypes = [ctypes.c_void_p, ctypes.c_size_t]
+  L.ft2_debug_trace_reset.argtypes = [ctypes.c_int]
 M = int(os.environ.get("M", "32"))
 NBLK = int(os.environ.get("NBLK", "8"))
 shapes = [tuple(map(int, s.split("x"))) for s in os.environ.get("SHAPES", "2048x2048,2048x2048,2048x8192").split(",")]
@@ -56,7 +58,8 @@ def run_all():
 
 run_all()
 torch.cuda.synchronize()
-L.ft2_debug_trace_reset(0)
+if not NOTRACE:
+    L.ft2_debug_trace_reset(0)
 g = torch.cuda.CUDAGraph()
 with torch.cuda.graph(g):
     run_all()
@@ -73,15 +76,31 @@ ms = e0.elapsed_time(e1) / 10
 nbytes = sum(w.numel() * 2 + x.numel() * 2 + y.numel() * 2 + b.numel() * 2 for x, w, b, y in launches)
 print(f"graph of {len(launches)} launches: {1000 * ms / len(launches):.2f} us/launch, "
       f"{nbytes / (ms / 1e3) / 1e9:.0f} GB/s algorithmic", flush=True)
+if NOTRACE:
+    sys.exit(0)
 g.replay()
 torch.cuda.synchronize()
 buf = np.zeros(32768 * 16, np.uint64)
 L.ft2_debug_trace_read(buf.ctypes.data, buf.nbytes)
 t = buf.reshape(128, 256, 16).astype(np.int64)
+# slot 10 = SM id + 1: how many CTAs of one launch share an SM (and its tensor pipe)
+occ = {}
+for i in range(len(launches)):
+    sm = t[i % 128][:, 10]
+    sm = sm[sm > 0] - 1
+    if sm.size == 0:
+        continue
+    per_sm = np.bincount(sm, minlength=148)
+    h = np.bincount(per_sm, minlength=4)[:4]
+    occ.setdefault(tuple(launches[i][1].shape), []).append((sm.size, int((per_sm > 0).sum()), int(h[2] + h[3:].sum())))
+for k, v in occ.items():
+    a = np.array(v)
+    print(f"SM sharing {k[0]}x{k[1]}: CTAs {int(np.median(a[:, 0]))}, SMs used {np.median(a[:, 1]):.0f}, "
+          f"SMs with >= 2 CTAs of the launch {np.median(a[:, 2]):.0f} (median over launches)")
 if CLK:
     # per-CTA SM-cycle deltas from the moment its producer's PDL wait returned
     # (slot 2), medians over the CTAs of every launch of a shape
-    sl = [0, 1, 2, 3, 12, 10, 15, 13, 4, 5, 14, 8, 9, 6, 11, 7]
+    sl = [0, 1, 2, 3, 12, 15, 13, 4, 5, 14, 8, 9, 6, 11, 7]
     per = {}
     for i in range(len(launches)):
         r = t[i % 128]
