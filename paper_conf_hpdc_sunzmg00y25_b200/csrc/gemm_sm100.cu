@@ -480,6 +480,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                                (i > 0 || k > 0) ? 1u : 0u);
                 }
                 if (i == 2) FT2_TRACE(15);
+                if (p.trigger == 3 && i == (nk - 1) / 2) griddep_launch();   // experiment: mid-stream trigger
                 // release the stage only if the producer will refill it: a
                 // commit costs the issuing thread ~300 cycles (measured), and
                 // with the whole K slice in the ring none is ever refilled
@@ -988,8 +989,12 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cA = g.cA;
     {   // two MMA issuers: 64-row tiles whose whole K slice sits in the ring (FT2_GEMM_MMA2=0 turns it off)
         static const int mma2_env = env_int("FT2_GEMM_MMA2", 1);
-        const int st = g.bn <= 16 ? Cfg<64, 16>::STAGES : Cfg<64, 32>::STAGES;
-        p.mma2 = (mma2_env && g.ba == 64 && g.cA == 1 && (g.nkb + g.splitk - 1) / g.splitk <= st) ? 1 : 0;
+        // (128-row tiles: opt-in, FT2_GEMM_MMA2=2 -- two warps issue an M = 128 MMA every ~47
+        // cycles against ~53 for one, profiles/r2_mma_probe.txt)
+        const int st = g.ba == 64 ? (g.bn <= 16 ? Cfg<64, 16>::STAGES : Cfg<64, 32>::STAGES)
+                                  : (g.bn <= 16 ? Cfg<128, 16>::STAGES : Cfg<128, 32>::STAGES);
+        const bool shape_ok = g.ba == 64 || (mma2_env == 2 && !g.deep && g.bn <= 32);
+        p.mma2 = (mma2_env && shape_ok && g.cA == 1 && (g.nkb + g.splitk - 1) / g.splitk <= st) ? 1 : 0;
     }
 
     p.sk_magic = (uint32_t)(((1u << 24) + g.splitk - 1) / g.splitk);
@@ -1020,6 +1025,13 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
             case 32: return launch_cfg<128, 32, true, 0, true>(a, p, st, n_launch);
             default: return launch_cfg<128, 64, true, 0, true>(a, p, st, n_launch);
         }
+    }
+    if (p.mma2) {   // 128-row tiles with the whole K slice in the ring (opt-in)
+        if (a.dtype == FT2_FP16)
+            return g.bn == 16 ? launch_cfg<128, 16, true, 1, false, true>(a, p, st, n_launch)
+                              : launch_cfg<128, 32, true, 1, false, true>(a, p, st, n_launch);
+        return g.bn == 16 ? launch_cfg<128, 16, true, 0, false, true>(a, p, st, n_launch)
+                          : launch_cfg<128, 32, true, 0, false, true>(a, p, st, n_launch);
     }
     if (a.dtype == FT2_FP16) {
         switch (g.bn) {
