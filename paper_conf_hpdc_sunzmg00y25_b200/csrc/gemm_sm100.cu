@@ -101,7 +101,7 @@ struct GemmK {
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
     int32_t w_static;  // weights not written by the preceding kernel: prefetch before the PDL wait
-    int32_t trigger;   // issue griddepcontrol.launch_dependents early (FT2_GEMM_TRIGGER, default 1)
+    int32_t trigger;   // where griddepcontrol.launch_dependents is issued (FT2_GEMM_TRIGGER, default 3; see below)
     int32_t w_l2;      // static weights: L2-prefetch the K slice beyond the ring before the PDL wait (FT2_GEMM_W_L2)
     int32_t rows_per_slot;  // ceil(BA / splitk): rows of one split-K receive slot
     uint32_t sk_magic;      // ceil(2^24 / splitk): floor(n / splitk) == (n * sk_magic) >> 24 for n < 2^20
@@ -365,9 +365,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     __syncthreads();
     tc_fence_after();
     // the next kernel in the stream may start its prologue (PDL): right here
-    // (trigger 1), or once this CTA's operands are all consumed (trigger 2, by
-    // the MMA thread below) so its early weight requests do not share the
-    // L2 -> SM path with this CTA's own operand stream
+    // (trigger 1), once this CTA's operands are all consumed (trigger 2, by
+    // the MMA thread below), or -- the default -- once the MMA thread has
+    // issued half of the CTA's k-blocks (trigger 3).  A later trigger keeps the
+    // next launch's early weight requests off the L2 -> SM path while this
+    // launch's x boxes (its critical path after the wait) stream in; measured
+    // back to back (profiles/r2_trigger_ab.txt): OPT graph 6.17 / 6.03 / 5.94 us
+    // per launch for 1 / 2 / 3, 2048x2048 4.59 / 4.43 / 4.20; in situ (a host
+    // kernel before every critical GEMM) all three equal
     if (p.trigger == 1) griddep_launch();
     // peers may push into my receive buffer once my barrier is initialised
     const int cA = p.cA, rA = (int)(blockIdx.x % (unsigned)cA);
@@ -480,7 +485,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                                (i > 0 || k > 0) ? 1u : 0u);
                 }
                 if (i == 2) FT2_TRACE(15);
-                if (p.trigger == 3 && i == (nk - 1) / 2) griddep_launch();   // experiment: mid-stream trigger
+                if (p.trigger == 3 && i == (nk - 1) / 2) griddep_launch();   // mid-stream trigger (default)
                 // release the stage only if the producer will refill it: a
                 // commit costs the issuing thread ~300 cycles (measured), and
                 // with the whole K slice in the ring none is ever refilled
@@ -975,7 +980,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st, int* n_launch) {
     p.cur_step = a.cur_step;
     p.base_row = a.base_row;
     p.w_static = a.w_static;
-    static const int trig = env_int("FT2_GEMM_TRIGGER", 1);
+    static const int trig = env_int("FT2_GEMM_TRIGGER", 3);
     p.trigger = trig;
     static const int wl2 = env_int("FT2_GEMM_W_L2", 0);
     static const int64_t wl2_max = (int64_t)env_int("FT2_GEMM_W_L2_MAX_MB", 48) << 20;
