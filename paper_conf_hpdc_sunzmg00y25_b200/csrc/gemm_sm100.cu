@@ -486,6 +486,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 }
                 if (i == 2) FT2_TRACE(15);
                 if (p.trigger == 3 && i == (nk - 1) / 2) griddep_launch();   // mid-stream trigger (default)
+                if (p.trigger >= 10 && i == (nk - 1) * (p.trigger - 10) / 8) griddep_launch();   // experiment: eighths
                 // release the stage only if the producer will refill it: a
                 // commit costs the issuing thread ~300 cycles (measured), and
                 // with the whole K slice in the ring none is ever refilled
