@@ -74,8 +74,10 @@ constexpr int kSplitCounters = 16384;   // split-K arrival counters at the head 
 struct PrefK {
     int32_t M, N, K, tilesM, ntiles, nkb;
     // split-K for grids the tiles alone cannot fill (small M): `splits` units
-    // per tile, fp32 partial slots [half-tile][split][128][256] in skws, one
-    // arrival counter per 128 x 256 half-tile in skcnt (self-cleaning)
+    // per tile, all in one wave, fp32 partial slots [half-tile][split][128][256]
+    // in skws, two counters per 128 x 256 half-tile in skcnt (partials
+    // written / partials read; self-cleaning).  Every split finishes 1/splits
+    // of its half-tile's 32-column groups from all the partials.
     int32_t splits;
     float* skws;
     uint32_t* skcnt;
@@ -95,6 +97,13 @@ struct PrefK {
     int32_t n_sites, cur_layer, cur_step;
     const int32_t* base_row;
 };
+
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+constexpr int kMaxSplits = 4;   // K splits the planner picks (partials of all splits held in registers)
 
 __device__ __forceinline__ uint32_t pack_rne2(float a, float b, int dt) {
     return dt == 1 ? ((uint32_t)rne16<1>(a) | ((uint32_t)rne16<1>(b) << 16))
@@ -146,7 +155,6 @@ __global__ void __launch_bounds__(kPThreads, 1)
     uint64_t* tmem_empty = tmem_full + 2;    // [2]
     uint32_t* tmem_base_sh = reinterpret_cast<uint32_t*>(tmem_empty + 2);
     uint32_t* last_sh = tmem_base_sh + 1;
-    uint32_t* skl_sh = tmem_base_sh + 2;  // "this unit finishes its half-tile" (split-K)
     uint32_t* tab_lo = reinterpret_cast<uint32_t*>(misc + kPMiscBytes);  // 0x10000 - min key (0: none)
     uint32_t* tab_hi = tab_lo + kPSeqTab;                                 // max key + 1 (0: none)
     uint32_t* tab_nf = tab_hi + kPSeqTab;                                 // non-finite count
@@ -351,15 +359,17 @@ __global__ void __launch_bounds__(kPThreads, 1)
                 __threadfence();
                 named_bar(1, 32 * kPEpiWarps);
                 if (tid == 64) {
-                    const bool last = atom_add_acq_rel_gpu(p.skcnt + half, 1u) == (uint32_t)(p.splits - 1);
-                    if (last) p.skcnt[half] = 0u;   // every split arrived: reset for the next launch
-                    *skl_sh = last ? 1u : 0u;
+                    // my partial is written; wait for every split's (they all run in
+                    // this one wave -- the host splits only when units * splits <= slots)
+                    atom_add_acq_rel_gpu(p.skcnt + 2 * half, 1u);
+                    while (ld_acquire_gpu(p.skcnt + 2 * half) < (uint32_t)p.splits) {
+                    }
                 }
                 named_bar(1, 32 * kPEpiWarps);
-                if (*skl_sh == 0u) continue;   // another split finishes this half-tile
             }
 #pragma unroll 1
             for (int c0 = h0; c0 < h0 + kPBN / 2; c0 += 32) {
+                if (split && (c0 >> 5) % p.splits != ks) continue;   // another split finishes these 32 columns
                 uint32_t r[32];
                 if (!split) {
                     tmem_ld32(taddr + (uint32_t)c0, r);
@@ -370,18 +380,28 @@ __global__ void __launch_bounds__(kPThreads, 1)
 #pragma unroll
                     for (int sub = 0; sub < 2; ++sub) {
                         const size_t coff = (size_t)((c0 + 16 * sub) >> 4) * (kPBM * 16);
+                        // every split's 4 vectors in flight at once (one L2 round trip),
+                        // then summed in split order 0..S-1 (deterministic)
+                        float4 part[kMaxSplits][4];
+#pragma unroll
+                        for (int sk = 0; sk < kMaxSplits; ++sk)
+                            if (sk < p.splits) {
+                                const float4* sl = reinterpret_cast<const float4*>(slot0 + (size_t)sk * kPBM * kPBN + coff);
+#pragma unroll
+                                for (int k = 0; k < 4; ++k) part[sk][k] = __ldcg(sl + e + 128 * k);
+                            }
                         float4 acc[4];
 #pragma unroll
-                        for (int k = 0; k < 4; ++k)
-                            acc[k] = __ldcg(reinterpret_cast<const float4*>(slot0 + coff) + e + 128 * k);
-                        for (int sk = 1; sk < p.splits; ++sk) {
-                            const float4* sl = reinterpret_cast<const float4*>(slot0 + (size_t)sk * kPBM * kPBN + coff);
+                        for (int k = 0; k < 4; ++k) acc[k] = part[0][k];
 #pragma unroll
-                            for (int k = 0; k < 4; ++k) {
-                                const float4 v = __ldcg(sl + e + 128 * k);
-                                acc[k].x += v.x; acc[k].y += v.y; acc[k].z += v.z; acc[k].w += v.w;
+                        for (int sk = 1; sk < kMaxSplits; ++sk)
+                            if (sk < p.splits) {
+#pragma unroll
+                                for (int k = 0; k < 4; ++k) {
+                                    acc[k].x += part[sk][k].x; acc[k].y += part[sk][k].y;
+                                    acc[k].z += part[sk][k].z; acc[k].w += part[sk][k].w;
+                                }
                             }
-                        }
 #pragma unroll
                         for (int k = 0; k < 4; ++k) {
                             const int i = e + 128 * k;
@@ -485,6 +505,13 @@ __global__ void __launch_bounds__(kPThreads, 1)
                         if (j < nvalid) yrow[nb + j] = (uint16_t)(w[j >> 1] >> ((j & 1) * 16));
                 }
             }
+            if (split) {   // my reads of the partial slots are done; the last reader resets both counters
+                named_bar(1, 32 * kPEpiWarps);
+                if (tid == 64 && atom_add_acq_rel_gpu(p.skcnt + 2 * half + 1, 1u) == (uint32_t)(p.splits - 1)) {
+                    p.skcnt[2 * half] = 0u;
+                    p.skcnt[2 * half + 1] = 0u;
+                }
+            }
             // accumulator buffer drained: hand it back to the MMA warp (the leader's)
             if (!split) {
                 tc_fence_before();
@@ -506,6 +533,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
                     kmax = 0u;
                     const int nend = min(p.N, n0 + h0 + kPBN / 2);
                     for (int n = n0 + h0; n < nend; ++n) {
+                        if (split && ((n - n0) >> 5) % p.splits != ks) continue;   // columns another split stored
                         const uint16_t b = yrow[n];
                         if (nonfinite1<DT>(b)) {
                             ++nf;
@@ -625,6 +653,38 @@ static cudaError_t launch_prefill_dt(const CUtensorMap& mx, const CUtensorMap& m
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+// Clusters (MC = 2: CTA pairs) or CTAs (MC = 1) of the persistent kernel that
+// can be resident at once.  The split-K path makes the splits of a tile wait
+// for each other, so it is planned only when every unit is resident at once.
+template <int MC>
+static int resident_slots() {
+    static int n = [] {
+        auto* k = prefill_gemm_kernel<0, MC>;
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kPSmemBytes) != cudaSuccess) {
+            cudaGetLastError();
+            return 0;
+        }
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)num_sms());
+        cfg.blockDim = dim3(kPThreads);
+        cfg.dynamicSmemBytes = kPSmemBytes;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = MC;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        int c = 0;
+        if (cudaOccupancyMaxActiveClusters(&c, k, &cfg) != cudaSuccess) {
+            cudaGetLastError();
+            return 0;
+        }
+        return c;
+    }();
+    return n;
+}
+
 // K-split plan for the persistent kernel: when the tiles cannot fill the
 // machine (small M: e.g. 512 prompt tokens at N = 4096 give 16 pair-tiles for
 // 74 SM pairs; a 256-trial decode batch gives 43 at N = 11008), split each
@@ -641,23 +701,24 @@ PrefillSplit plan_prefill_split(int32_t M, int32_t N, int32_t K, size_t ws_bytes
     // words) whatever the shape, so one launch's partial slots never alias
     // the next launch's counters
     r.cnt_bytes = (size_t)kSplitCounters * 4;
-    if ((size_t)tilesMp * tilesN > (size_t)kSplitCounters) return r;
+    if ((size_t)tilesMp * tilesN * 2 > (size_t)kSplitCounters) return r;   // two counters per half-tile
     const size_t per_split = (size_t)tilesMp * kPBM * tilesN * kPBN * 4;
-    // Opt-in (FT2_PREFILL_SPLITS = s >= 2, or -1 for the planner below).
-    // Measured (profiles/r1_prefill_splitk.txt): with per-row partial stores
-    // the split was 1.6x SLOWER; with the shared-memory-staged coalesced
-    // slots it is at par (M = 256, 4096^2: 28.7 us unsplit, 28.9 at s = 4),
-    // because the mainloop is latency-bound at ~0.45 us per k-block per CTA
-    // pair either way -- so it stays off until that is fixed.
+    // FT2_PREFILL_SPLITS = s >= 2 forces s, 0 or 1 disables, -1 (default) is
+    // the planner: the largest s <= kMaxSplits with units * s <= slots (one
+    // wave: the splits of a tile wait for each other) and >= 8 k-blocks each.
+    // Round 1 measured the old last-arriver reduction at par with no split
+    // (its reads were serialised per split); the distributed one reads every
+    // split's vectors at once (profiles/r2_prefill_split.txt).
     const char* ev = getenv("FT2_PREFILL_SPLITS");   // read per call: tests toggle it
-    const int env = ev ? atoi(ev) : 0;
+    const int env = ev ? atoi(ev) : -1;
     if (env == 0 || env == 1) return r;
-    double best_t = (double)((units + slots - 1) / slots);
-    for (int s = 2; s <= 8; ++s) {
-        if (nkb < 8 * s) break;
-        if (env > 0 && s != env) continue;
-        const double t = (double)((units * s + slots - 1) / slots) / s;
-        if (t < 0.9 * best_t || (env > 0 && s == env)) { best_t = t; r.splits = s; }
+    // (a tcgen05.alloc kernel reads as 1 CTA/SM to the occupancy API, which is
+    // what this kernel runs at anyway)
+    const int resident = tilesM >= 2 ? resident_slots<2>() : resident_slots<1>();
+    for (int s = 2; s <= kMaxSplits; ++s) {
+        if (nkb < 8 * s || units * s > slots || units * s > resident) break;
+        if (env > 0 && s > env) break;
+        r.splits = s;
     }
     r.need_bytes = r.splits > 1 ? r.cnt_bytes + (size_t)r.splits * per_split : 0;
     while (r.splits > 1 && r.cnt_bytes + (size_t)r.splits * per_split > ws_bytes) --r.splits;
