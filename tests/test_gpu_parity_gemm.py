@@ -253,7 +253,10 @@ def test_gemm_site_overflow_is_never_dropped(ft2, M, N, K, step):
 
 @pytest.mark.parametrize("env", [{"FT2_GEMM_BA": "64"}, {"FT2_GEMM_BA": "128"},
                                  {"FT2_GEMM_BA": "64", "FT2_GEMM_XMC": "1"},
-                                 {"FT2_GEMM_BA": "128", "FT2_GEMM_BN": "16"}])
+                                 {"FT2_GEMM_BA": "128", "FT2_GEMM_BN": "16"},
+                                 {"FT2_GEMM_MMA2": "0"},                      # one MMA issuer (round 1)
+                                 {"FT2_GEMM_BA": "128", "FT2_GEMM_BN": "32", "FT2_GEMM_MMA2": "2"},   # 128-row MMA2
+                                 {"FT2_GEMM_TRIGGER": "1"}, {"FT2_GEMM_TRIGGER": "2"}])
 def test_gemm_tile_variants_in_subprocess(env):
     """The 64- and 128-row feature tiles and the opt-in x multicast (planner
     knobs read once per process) give results within R8's tolerance and
