@@ -226,6 +226,19 @@ __device__ __noinline__ uint2 xor_sites_scan(uint2 w, const GemmK& p, int ga, in
     return w;
 }
 
+// Sum of the NS split-K slots of one float4 (slot r at src + r * step floats),
+// in slot order 0..NS-1 (the same order as the generic loop: bit-identical).
+template <int NS>
+__device__ __forceinline__ float4 sum_slots(const float* src, int step) {
+    float4 part[NS];
+#pragma unroll
+    for (int r = 0; r < NS; ++r) part[r] = *reinterpret_cast<const float4*>(src + r * step);
+    float4 acc = part[0];
+#pragma unroll
+    for (int r = 1; r < NS; ++r) { acc.x += part[r].x; acc.y += part[r].y; acc.z += part[r].z; acc.w += part[r].w; }
+    return acc;
+}
+
 // Check-and-clip of two packed bf16 (R5): NaN -> key(+0), clamp in key space.
 template <int DT>
 __device__ __forceinline__ uint32_t clip2_nocount(uint32_t w, uint32_t kL2, uint32_t kH2) {
@@ -484,7 +497,6 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                         tc_mma(tmem_base, da + (uint64_t)(k * 2), db + (uint64_t)(k * 2), idesc,
                                (i > 0 || k > 0) ? 1u : 0u);
                 }
-                if (i == 2) FT2_TRACE(15);
                 if (p.trigger == 3 && i == (nk - 1) / 2) griddep_launch();   // mid-stream trigger (default)
                 if (p.trigger >= 10 && i == (nk - 1) * (p.trigger - 10) / 8) griddep_launch();   // experiment: eighths
                 // release the stage only if the producer will refill it: a
@@ -621,19 +633,27 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         if (cs) mbar_wait(recv_bar, 0);  // ... and every peer's rows of my slice
         if (tid == 64) FT2_TRACE(6);
         const uint32_t nsite = *site_n;   // > kMaxSitesPerCta: finish4 scans every site
+        if (tid == 64) FT2_TRACE(15);     // (trace builds: the site count read)
 #pragma unroll 1
         for (int v = e; v < nvec; v += 128) {
             // consecutive threads take consecutive rows (coalesced stores in swap-AB mode)
             const int c4 = (int)(((uint32_t)v * inv) >> 20), lr = v - c4 * nrow, la = r0 + lr;
-            float4 part[kMaxSplitK];
             const float* src = recv + lr * C::kRecvStride + c4 * 4;
+            float4 acc;
+            if (splitk == 4) {   // the common split factors: every slot read issued before the sum
+                acc = sum_slots<4>(src, RS * C::kRecvStride);
+            } else if (splitk == 8) {
+                acc = sum_slots<8>(src, RS * C::kRecvStride);
+            } else {
+                float4 part[kMaxSplitK];
 #pragma unroll
-            for (int rr = 0; rr < kMaxSplitK; ++rr)
-                if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
-            float4 acc = part[0];
+                for (int rr = 0; rr < kMaxSplitK; ++rr)
+                    if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
+                acc = part[0];
 #pragma unroll
-            for (int rr = 1; rr < kMaxSplitK; ++rr)
-                if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
+                for (int rr = 1; rr < kMaxSplitK; ++rr)
+                    if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
+            }
             if (tid == 64) FT2_TRACE(11);
             finish4<SWAP, DT>(y, ldy, tileA * BA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
                               (uint32_t)(la * BN + c4 * 4), acc, site_e, site_m, nsite, row_cnt + la, col_cnt + c4 * 4, p);

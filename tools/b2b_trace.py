@@ -100,7 +100,7 @@ for k, v in occ.items():
 if CLK:
     # per-CTA SM-cycle deltas from the moment its producer's PDL wait returned
     # (slot 2), medians over the CTAs of every launch of a shape
-    sl = [0, 1, 2, 3, 12, 15, 13, 4, 5, 14, 8, 9, 6, 11, 7]
+    sl = [0, 1, 2, 3, 12, 13, 4, 5, 14, 8, 9, 6, 15, 11, 7]
     per = {}
     for i in range(len(launches)):
         r = t[i % 128]
