@@ -74,11 +74,23 @@ for (M, N, K) in [(256, 512, 1024), (136, 264, 1024)]:
     ft2.prefill_fused_gemm(x, w, out, bd, ft2.make_workspace(2), seq_offsets=sq, num_seqs=2)
 os.environ.pop("FT2_PREFILL_SPLITS")
 # fused row-parallel all-reduce + check at P = 1 (handshake skipped) through the C ABI directly
-pp = torch.tensor([yd.data_ptr()], dtype=torch.int64, device=dev)
+# (round 2 session e: pointer tables are host arrays; also in place, y aliasing the partial)
 fl = torch.zeros(1, dtype=torch.int32, device=dev)
-fp = torch.tensor([fl.data_ptr()], dtype=torch.int64, device=dev)
 words = torch.zeros(3, dtype=torch.int32, device=dev)
 yo = torch.empty_like(yd)
-ft2.allreduce_protect(pp, 520, 1, 0, fp, words, yo, mode=1, bounds=b[:1].clone(), num_seqs=1, corrected_count=cnt)
+ft2.allreduce_protect([yd.data_ptr()], 520, 1, 0, [fl.data_ptr()], words, yo, mode=1, bounds=b[:1].clone(),
+                      num_seqs=1, corrected_count=cnt)
+ft2.allreduce_protect([yo.data_ptr()], 520, 1, 0, [fl.data_ptr()], words, yo, mode=1,
+                      bounds=torch.tensor([[-0.05, 0.05]], dtype=torch.bfloat16, device=dev), num_seqs=1,
+                      corrected_count=cnt)
+# round 2 session e: the default prefill K split (distributed reduction) at a 512-token shape
+for (M, N, K) in [(512, 1024, 2048)]:
+    x = ft2_synth.gen_bf16_torch((M, K), 8, 1, device=dev)
+    w = ft2_synth.gen_bf16_torch((N, K), 9, 1, scale_log2=-5, device=dev)
+    out = torch.empty((M, N), dtype=torch.bfloat16, device=dev)
+    ft2.protect_fused_gemm(x, w, out, mode=0)
+    sq = torch.arange(0, M + 1, M // 8, dtype=torch.int32, device=dev)
+    bd = torch.zeros((8, 2), dtype=torch.bfloat16, device=dev)
+    ft2.prefill_fused_gemm(x, w, out, bd, ft2.make_workspace(8), seq_offsets=sq, num_seqs=8)
 torch.cuda.synchronize()
 print("sanitize cases: done")
