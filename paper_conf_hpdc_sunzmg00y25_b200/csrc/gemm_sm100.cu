@@ -239,6 +239,43 @@ __device__ __forceinline__ float4 sum_slots(const float* src, int step) {
     return acc;
 }
 
+// Any other split factor, out of line (kept off the common path's code size).
+__device__ __noinline__ float4 sum_slots_any(const float* src, int step, int splitk) {
+    float4 part[kMaxSplitK];
+#pragma unroll
+    for (int r = 0; r < kMaxSplitK; ++r)
+        if (r < splitk) part[r] = *reinterpret_cast<const float4*>(src + r * step);
+    float4 acc = part[0];
+#pragma unroll
+    for (int r = 1; r < kMaxSplitK; ++r)
+        if (r < splitk) { acc.x += part[r].x; acc.y += part[r].y; acc.z += part[r].z; acc.w += part[r].w; }
+    return acc;
+}
+
+// The fault sites that land in this CTA's slice (rows [r0, r1) of the tile at
+// (a0, b0)), gathered into the shared-memory site list (sites beyond
+// kMaxSitesPerCta only raise the count: finish4 then rescans every site).
+// Out of line: only fault-injection runs pass sites.
+template <bool SWAP>
+__device__ __noinline__ void gather_sites(const GemmK& p, int e, int a0, int b0, int BA, int BN, int r0, int r1,
+                                          uint32_t* site_n, uint32_t* site_e, uint32_t* site_m) {
+    for (int i = e; i < p.n_sites; i += 128) {
+        const ft2_fault_site st = p.sites[i];
+        if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
+        const int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) + (p.cur_step == 0 ? (int64_t)st.token : 0);
+        const int64_t n = st.col;
+        if (m < 0 || m >= p.M || n >= p.N) continue;
+        const int64_t la = (SWAP ? n : m) - (int64_t)a0;
+        const int64_t lb = (SWAP ? m : n) - (int64_t)b0;
+        if (la < r0 || la >= r1 || lb < 0 || lb >= BN) continue;
+        const uint32_t idx = atomicAdd(site_n, 1u);
+        if (idx < (uint32_t)kMaxSitesPerCta) {
+            site_e[idx] = (uint32_t)(la * BN + lb);
+            site_m[idx] = st.xor_mask;
+        }
+    }
+}
+
 // Check-and-clip of two packed bf16 (R5): NaN -> key(+0), clamp in key space.
 template <int DT>
 __device__ __forceinline__ uint32_t clip2_nocount(uint32_t w, uint32_t kL2, uint32_t kH2) {
@@ -528,24 +565,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             col_tab[c] = SWAP ? token_entry(p, tileB * BN + c) : feature_entry<DT>(p, tileB * BN + c);
             col_cnt[c] = 0u;
         }
-        if (p.sites != nullptr) {  // fault sites landing in my slice
-            for (int i = e; i < p.n_sites; i += 128) {
-                const ft2_fault_site st = p.sites[i];
-                if ((int)st.step != p.cur_step || (int)st.layer != p.cur_layer) continue;
-                const int64_t m = (p.base_row ? (int64_t)p.base_row[i] : (int64_t)i) +
-                                  (p.cur_step == 0 ? (int64_t)st.token : 0);
-                const int64_t n = st.col;
-                if (m < 0 || m >= p.M || n >= p.N) continue;
-                const int64_t la = (SWAP ? n : m) - (int64_t)tileA * BA;
-                const int64_t lb = (SWAP ? m : n) - (int64_t)tileB * BN;
-                if (la < r0 || la >= r1 || lb < 0 || lb >= BN) continue;
-                const uint32_t idx = atomicAdd(site_n, 1u);
-                if (idx < (uint32_t)kMaxSitesPerCta) {
-                    site_e[idx] = (uint32_t)(la * BN + lb);
-                    site_m[idx] = st.xor_mask;
-                }
-            }
-        }
+        if (p.sites != nullptr)  // fault sites landing in my slice (out of line: campaign runs only)
+            gather_sites<SWAP>(p, e, tileA * BA, tileB * BN, BA, BN, r0, r1, site_n, site_e, site_m);
         // Receive-slot geometry of accumulator row a (independent of the
         // accumulator, so computed while the main loop streams): its owner
         // is the split whose row slice holds a, r0(r) = floor(BA r / splitk)
@@ -645,14 +666,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             } else if (splitk == 8) {
                 acc = sum_slots<8>(src, RS * C::kRecvStride);
             } else {
-                float4 part[kMaxSplitK];
-#pragma unroll
-                for (int rr = 0; rr < kMaxSplitK; ++rr)
-                    if (rr < splitk) part[rr] = *reinterpret_cast<const float4*>(src + rr * RS * C::kRecvStride);
-                acc = part[0];
-#pragma unroll
-                for (int rr = 1; rr < kMaxSplitK; ++rr)
-                    if (rr < splitk) { acc.x += part[rr].x; acc.y += part[rr].y; acc.z += part[rr].z; acc.w += part[rr].w; }
+                acc = sum_slots_any(src, RS * C::kRecvStride, splitk);
             }
             if (tid == 64) FT2_TRACE(11);
             finish4<SWAP, DT>(y, ldy, tileA * BA + la, tileB * BN + c4 * 4, row_tab[la], col_tab + c4 * 4,
