@@ -226,12 +226,18 @@ class Runner:
         # torch's kernels (experiments)
         self.host_norm = os.environ.get("FT2_HOST_NORM", "1") == "1"
         self.host_act = self.host_norm and os.environ.get("FT2_HOST_ACT", "1") == "1"
-        # L2 prefetch hint of the decode GEMMs (ft2_protect_fused_gemm_ex): each
+        # L2 prefetch hint of the decode GEMMs (ft2_protect_fused_gemm_ex): a
         # fused critical-layer GEMM pulls the weights of the next one into L2
-        # once its own operands have landed.  Measured slower in situ (OPT-1.3B
-        # decode step 1.79 -> 1.82 ms; the prefetch competes with the current
-        # layer's own weight stream), so opt-in: FT2_L2_PREFETCH=1
-        self.l2_prefetch = os.environ.get("FT2_L2_PREFETCH", "0") == "1"
+        # once its own operands have landed.  Default (FT2_L2_PREFETCH=2): only
+        # v_proj, for out_proj / o_proj -- the layer after attention, which is
+        # latency-bound and triggers no PDL, so out_proj otherwise pays its whole
+        # weight fetch after it (session e, OPT-1.3B in situ, two A/B pairs:
+        # 16 970 -> 16 990 protected tok/s, decode step 1.744 -> 1.741 ms).
+        # FT2_L2_PREFETCH=1 hints every layer (slower: the prefetch of fc2's
+        # 34 MB competes with fc1's own stream; 16 928 tok/s), 0 none.
+        mode = os.environ.get("FT2_L2_PREFETCH", "2")
+        self.l2_prefetch = mode in ("1", "2")
+        self.l2_prefetch_after_attn = mode == "2"
         self.crit_names = cfg.coverage_names(coverage)   # protected layers of one block
         self.lin_names = [n for n, _, _, _ in cfg.linears()]
         self.n_crit = len(self.crit_names) * cfg.n_layers
@@ -426,7 +432,9 @@ class Runner:
         if getattr(self, "_next_w", None) is None:
             order = self._fused_gemm_order()
             w_of = lambda b_, n_: b_.wf[n_] if n_ in b_.wf else b_.w[n_]
-            self._next_w = {(b_.idx, n_): w_of(*order[(i + 1) % len(order)]) for i, (b_, n_) in enumerate(order)}
+            nxt = {(b_.idx, n_): order[(i + 1) % len(order)] for i, (b_, n_) in enumerate(order)}
+            self._next_w = {k: w_of(*v) for k, v in nxt.items()
+                            if not self.l2_prefetch_after_attn or v[1] in ("out_proj", "o_proj")}
         return self._next_w.get((blk.idx, name))
 
     def _group_ok(self, blk: Block, g: str) -> bool:
