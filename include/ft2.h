@@ -221,6 +221,11 @@ ft2_status ft2_protect(ft2_tensor y, const int32_t* row_to_seq, const void* boun
  *              Split partials are summed in split order: results do not depend
  *              on the workspace (only the timing does) -- except that a
  *              different split count changes the fp32 summation order.
+ *              A split is planned only when every (tile, split) unit of the
+ *              launch fits on the GPU at once (the splits of a tile wait for
+ *              each other): do not run such a call concurrently with other
+ *              kernels that hold SMs indefinitely (persistent kernels on other
+ *              streams); pass NULL, or set FT2_PREFILL_SPLITS=0, to disable it.
  * The kernel is launched with programmatic stream serialization (PDL): its
  * prologue and first weight tiles overlap the previous kernel's tail; it reads
  * x, bias, bounds, sites and writes y, counters, workspace only after the
