@@ -574,6 +574,7 @@ def main():
         # ranges split over the ranks
         del runner
         torch.cuda.empty_cache()
+    if not args.no_extras and not _skip("partitioned"):
         progress("partitioned paths")
         try:
             res["partitioned_paths"] = partitioned_legs(args, dev, rank, world)
@@ -710,20 +711,19 @@ def kernel_rooflines(runner, dev, ft2):
                 xs[K] = ft2_synth.gen_bf16_torch((B, K), 77, K, device=dev)
             y = torch.empty((B, w.shape[0]), dtype=torch.bfloat16, device=dev)
             cid = runner._crit_id(blk.idx, name)
-            launches.append((xs[K], w, b, y, cid))
+            launches.append((xs[K], w, b, y, cid, runner._next_fused_w(blk, name)))
     st = runner.state
     big = torch.full((runner.n_crit, B, 2), 0, dtype=torch.bfloat16, device=dev)
     big[..., 0] = -3.0e38
     big[..., 1] = 3.0e38
 
-    # each GEMM carries the next one's weights as its L2 prefetch hint, as the
-    # runner's decode step does (runner.l2_prefetch)
-    nxt = [launches[(i + 1) % len(launches)][1] if runner.l2_prefetch else None for i in range(len(launches))]
+    # each GEMM carries the L2 prefetch hint the runner's decode step gives it
+    # (runner._next_fused_w: by default only v_proj, for out_proj's weights)
 
     def run_all():
-        for i, (x, w, b, y, cid) in enumerate(launches):
+        for i, (x, w, b, y, cid, pf) in enumerate(launches):
             ft2.protect_fused_gemm(x, w, y, bias=b, mode=1 | 16, bounds=big[cid], num_seqs=B,
-                                   corrected_count=st.corrected[cid], l2_prefetch=nxt[i])
+                                   corrected_count=st.corrected[cid], l2_prefetch=pf)
 
     run_all()
     torch.cuda.synchronize()
@@ -742,7 +742,7 @@ def kernel_rooflines(runner, dev, ft2):
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / R
     nbytes = sum(w.numel() * 2 + x.numel() * 2 + y.numel() * 2 + (b.numel() * 2 if b is not None else 0)
-                 for x, w, b, y, _ in launches)
+                 for x, w, b, y, _, _ in launches)
     per_launch_us = 1000.0 * ms / len(launches)
     ach = nbytes / (ms / 1e3) / 1e9
     traffic = load_traffic()
@@ -752,7 +752,8 @@ def kernel_rooflines(runner, dev, ft2):
             "shapes": f"M={B}; (N,K) per block: " + ", ".join(
                 f"{blk_w.shape[0]}x{blk_w.shape[1]}" for blk_w in [runner.blocks[0].w[n] for n in runner.crit_names]),
             "launches_per_graph": len(launches), "avg_launch_us": per_launch_us,
-            "l2_prefetch_hint": bool(runner.l2_prefetch),
+            "l2_prefetch_hint": ("v_proj -> out_proj only (the runner's default)" if runner.l2_prefetch_after_attn
+                                 else bool(runner.l2_prefetch)),
             "bytes_per_launch_avg": nbytes / len(launches), "peak_source": peak_src,
             "algorithmic_bytes": "N*K*2 (W) + M*K*2 (x) + M*N*2 (y) + N*2 (bias) per launch"}
     # ---- the same kernel streaming (large K, not launch-latency bound): M = 32,
