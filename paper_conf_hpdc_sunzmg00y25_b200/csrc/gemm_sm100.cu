@@ -826,13 +826,13 @@ static int swap_max_m() {
     return v;
 }
 
-static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
+static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K, bool force64 = false) {
     GemmPlan g;
     g.swap = M <= swap_max_m() ? 1 : 0;
     g.ba = 128;
     g.cA = 1;
     static const int sk_env0 = env_int("FT2_GEMM_SPLITK", 0);
-    if (g.swap && use_ba64(M, N, K)) {
+    if (g.swap && (force64 || use_ba64(M, N, K))) {
         // the smallest split whose K slice fits the ring (one DRAM round trip,
         // weights requested before the PDL wait), at most 2 CTAs per SM and
         // clusters of <= 8; large K keeps streaming at the largest such split
@@ -931,6 +931,16 @@ static GemmPlan plan_gemm_impl(int32_t M, int32_t N, int32_t K) {
             }
         }
     }
+    // A 128-row plan that puts more CTAs than SMs on the GPU double-books SMs
+    // anyway (profiles: SM sharing); for N <= 2048 at <= 32 tokens (OPT fc2)
+    // the 64-row plan -- half the split-K exchange per CTA, an 8-way split with
+    // the fixed-size slot sum -- is then faster: fc2 back to back 8.95 -> 8.68
+    // us, in situ +0.1 %; plans that fit one CTA per SM (e.g. Qwen2-1.5B's
+    // 1536x8960 down_proj, 144 CTAs) stay at 128 rows (profiles/r2_fc2_ba64.txt)
+    static const int ba_env = env_int("FT2_GEMM_BA", 0);
+    if (g.swap && !force64 && !g.deep && ba_env == 0 && M <= 32 && N <= 2048 &&
+        g.tilesA * g.tilesB * g.splitk > num_sms())
+        return plan_gemm_impl(M, N, K, true);
     return g;
 }
 
