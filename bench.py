@@ -748,7 +748,9 @@ def kernel_rooflines(runner, dev, ft2):
     traffic = load_traffic()
     gemm_tr = traffic.get("gemm_decode_opt1.3b", {}).get("avg_per_launch_bytes") if runner.cfg.hidden == 2048 else None
     gemm = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
-            "traffic": gemm_tr, "traffic_source": traffic.get("source") if gemm_tr else None, "kernel": "ft2 gemm_kernel (tcgen05, CHECK epilogue)",
+            "traffic": gemm_tr, "traffic_source": traffic.get("source") if gemm_tr else None,
+            "traffic_note": traffic.get("gemm_decode_opt1.3b", {}).get("note") if gemm_tr else None,
+            "kernel": "ft2 gemm_kernel (tcgen05, CHECK epilogue)",
             "shapes": f"M={B}; (N,K) per block: " + ", ".join(
                 f"{blk_w.shape[0]}x{blk_w.shape[1]}" for blk_w in [runner.blocks[0].w[n] for n in runner.crit_names]),
             "launches_per_graph": len(launches), "avg_launch_us": per_launch_us,
